@@ -1,0 +1,221 @@
+"""Pins for the float64 forward oracle: hand-computed values, closed
+forms, and torch float64 modules (test-only cross-check; the oracle itself is NumPy)."""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import forward as F
+from oracle.ir import IRError, parse
+
+
+def f32(a):
+    return np.asarray(a, dtype=np.float32)
+
+
+def bf16_bits(a):
+    t = torch.tensor(np.asarray(a, dtype=np.float32)).to(torch.bfloat16)
+    return t.view(torch.int16).numpy().view(np.uint16)
+
+
+# ---- hand-computed 2-layer toy (SURVEY.md C-P "Forward, MLP/sigmoid") -----------------------
+TOY = """
+param @W1 : {dt}[2,2]
+param @b1 : f32[2]
+param @W2 : {dt}[1,2]
+param @b2 : f32[1]
+%x = input() : {dt}[1,2]
+%h = linear(%x, @W1, @b1) {{act=relu}} : {dt}[1,2]
+%y = linear(%h, @W2, @b2) {{act=sigmoid}} : f32[1,1]
+output %y
+"""
+TOY_Y = 0.029312230751356319  # sigma(-3.5), h = relu([-2.5, 4.5]) = [0, 4.5], z = 2*0 - 4.5 + 1
+
+
+@pytest.mark.parametrize("dt", ["f32", "bf16"])
+def test_toy_mlp_hand_computed(dt):
+    enc = f32 if dt == "f32" else bf16_bits
+    params = {"W1": enc([[1, 2], [3, -1]]), "b1": f32([0.5, -0.5]), "W2": enc([[2, -1]]),
+              "b2": f32([1])}
+    out = F.run(TOY.format(dt=dt), params, {"x": enc([[1, -2]])}, keep_all=True)
+    np.testing.assert_array_equal(out["h"], [[0.0, 4.5]])
+    assert out["y"][0, 0] == pytest.approx(TOY_Y, rel=1e-15)
+    assert 1.0 / (1.0 + math.exp(3.5)) == pytest.approx(TOY_Y, rel=1e-15)
+
+
+# ---- gathers: integer table pattern, exact ----------------------------------------------------
+def _pattern_table(F_, R, D):
+    f, v, k = np.meshgrid(np.arange(F_), np.arange(R), np.arange(D), indexing="ij")
+    return ((7 * v + 3 * k + 11 * f) % 251) - 125
+
+
+def test_gather_concat_and_sum_pattern():
+    F_, R, D, B = 4, 300, 8, 9
+    E = _pattern_table(F_, R, D)
+    rng = np.random.default_rng(0)
+    ids = rng.integers(0, R, size=(B, F_))
+    out = F.gather_concat(ids, f32(E), "f32")
+    for b in range(B):
+        for f in range(F_):
+            for k in range(D):
+                assert out[b, f * D + k] == ((7 * ids[b, f] + 3 * k + 11 * f) % 251) - 125
+    Tw = _pattern_table(F_, R, 1)[:, :, 0]
+    ws = F.gather_sum(ids, bf16_bits(Tw), "bf16", np.array([0.5]))
+    for b in range(B):
+        assert ws[b, 0] == 0.5 + sum(((7 * ids[b, f] + 11 * f) % 251) - 125 for f in range(F_))
+
+
+def test_hash_mod_floor():
+    raw = np.array([[0, 5, 10**12 + 7, 2**31 - 1]], dtype=np.int64)
+    np.testing.assert_array_equal(F.hash_mod(raw, 1000), [[0, 5, (10**12 + 7) % 1000, (2**31 - 1) % 1000]])
+    assert F.hash_mod(np.array([-3]), 10)[0] == 7
+
+
+def test_embed_seq_time_major():
+    E = np.arange(20, dtype=np.float32).reshape(10, 2)
+    tok = np.array([[1, 2, 3], [4, 5, 6]])
+    x = F.embed_seq(tok, E, "f32")
+    assert x.shape == (3, 2, 2)
+    np.testing.assert_array_equal(x[2, 1], E[6])
+
+
+# ---- LSTM / GRU closed forms (weights 0) and torch float64 ---------------------------------------
+def test_lstm_zero_weight_closed_form():
+    H, S, B, E = 3, 7, 2, 4
+    bih = np.array([0.3, -0.2, 0.1, 0.5, 0.7, 0.2, -0.4, 0.6, -0.1, 0.2, 0.3, -0.3])
+    bhh = np.array([0.1] * 12)
+    x = np.random.default_rng(1).normal(size=(S, B, E))
+    h = F.lstm(x, np.zeros((4 * H, E)), np.zeros((4 * H, H)), bih, bhh)
+    bx = bih + bhh
+    sg = lambda v: 1 / (1 + np.exp(-v))
+    i, f, g, o = sg(bx[:H]), sg(bx[H:2 * H]), np.tanh(bx[2 * H:3 * H]), sg(bx[3 * H:])
+    c = i * g * (1 - f ** S) / (1 - f)
+    np.testing.assert_allclose(h, np.broadcast_to(o * np.tanh(c), (B, H)), rtol=1e-13)
+
+
+def test_gru_zero_weight_closed_form():
+    H, S, B, E = 3, 5, 2, 4
+    bih = np.array([0.3, -0.2, 0.1, 0.5, 0.7, 0.2, -0.4, 0.6, -0.1])
+    bhh = np.array([0.2, 0.1, -0.3, 0.05, 0.0, 0.4, 0.3, -0.2, 0.25])
+    x = np.random.default_rng(2).normal(size=(S, B, E))
+    h = F.gru(x, np.zeros((3 * H, E)), np.zeros((3 * H, H)), bih, bhh)
+    sg = lambda v: 1 / (1 + np.exp(-v))
+    r = sg(bih[:H] + bhh[:H])
+    z = sg(bih[H:2 * H] + bhh[H:2 * H])
+    n = np.tanh(bih[2 * H:] + r * bhh[2 * H:])
+    np.testing.assert_allclose(h, np.broadcast_to(n * (1 - z ** S), (B, H)), rtol=1e-13)
+
+
+@pytest.mark.parametrize("kind", ["lstm", "gru"])
+def test_rnn_vs_torch_f64(kind):
+    S, B, E, H = 6, 5, 7, 9
+    torch.manual_seed(0)
+    mod = (torch.nn.LSTM if kind == "lstm" else torch.nn.GRU)(E, H).double()
+    x = torch.randn(S, B, E, dtype=torch.float64)
+    _, st = mod(x)
+    want = (st[0] if kind == "lstm" else st)[0].detach().numpy()
+    fn = F.lstm if kind == "lstm" else F.gru
+    got = fn(x.numpy(), mod.weight_ih_l0.detach().numpy(), mod.weight_hh_l0.detach().numpy(),
+             mod.bias_ih_l0.detach().numpy(), mod.bias_hh_l0.detach().numpy())
+    np.testing.assert_allclose(got, want, rtol=1e-12, atol=1e-14)
+
+
+# ---- conv / BN / pooling ----------------------------------------------------------------------
+def test_conv_center_tap_identity_and_bn_identity():
+    x = np.random.default_rng(3).normal(size=(2, 5, 6, 4))
+    W = np.zeros((4, 3, 3, 4))
+    for c in range(4):
+        W[c, 1, 1, c] = 1.0
+    y = F.conv2d_bn(x, W, np.ones(4), np.zeros(4), np.zeros(4), np.full(4, 1 - 1e-5), 1, 1, "none")
+    np.testing.assert_allclose(y, x, rtol=1e-12, atol=1e-15)
+
+
+@pytest.mark.parametrize("stride,pad,k", [(1, 1, 3), (2, 1, 3), (2, 3, 7), (2, 0, 1)])
+def test_conv_bn_vs_torch_f64(stride, pad, k):
+    rng = np.random.default_rng(4)
+    N, H, W_, C, Co = 2, 11, 9, 3, 5
+    x = rng.normal(size=(N, H, W_, C))
+    Wt = rng.normal(size=(Co, k, k, C))
+    g, b, mu, var = rng.uniform(0.5, 1.5, Co), rng.normal(size=Co), rng.normal(size=Co), rng.uniform(0.5, 1.5, Co)
+    got = F.conv2d_bn(x, Wt, g, b, mu, var, stride, pad, "relu")
+    conv = torch.nn.functional.conv2d(torch.tensor(x).permute(0, 3, 1, 2),
+                                      torch.tensor(Wt).permute(0, 3, 1, 2), stride=stride, padding=pad)
+    bn = torch.nn.functional.batch_norm(conv, torch.tensor(mu), torch.tensor(var), torch.tensor(g),
+                                        torch.tensor(b), training=False, eps=1e-5)
+    want = torch.relu(bn).permute(0, 2, 3, 1).numpy()
+    np.testing.assert_allclose(got, want, rtol=1e-11, atol=1e-12)
+
+
+def test_maxpool_avgpool_vs_torch():
+    x = np.random.default_rng(5).normal(size=(2, 9, 8, 3))
+    got = F.maxpool(x, 3, 2, 1)
+    want = torch.nn.functional.max_pool2d(torch.tensor(x).permute(0, 3, 1, 2), 3, 2, 1).permute(0, 2, 3, 1)
+    np.testing.assert_array_equal(got, want.numpy())
+    np.testing.assert_allclose(F.avgpool(x), x.reshape(2, -1, 3).mean(1), rtol=1e-14)
+
+
+def test_resnet18_small_vs_torch_f64():
+    """The workload's ResNet-18 IR through the oracle == a torch float64 ResNet-18 built here
+    from nn.Conv2d / nn.BatchNorm2d (torchvision BasicBlock topology)."""
+    from paper_conf_ipps_zhanghl21_b200 import workloads as W
+    wl = W.build("c4", small=True, dt="f32")
+    params = {k: s.materialize().numpy() for k, s in wl.params.items()}
+    img = wl.inputs["image"].materialize().numpy()
+    vals = F.run(wl.ir, params, {"image": img, "tok": wl.inputs["tok"].materialize().numpy(),
+                                 "raw": wl.inputs["raw"].materialize().numpy()}, keep_all=True)
+
+    def P(n):
+        return torch.tensor(params[n], dtype=torch.float64)
+
+    def cbn(x, name, stride, pad, relu):
+        y = torch.nn.functional.conv2d(x, P(name + "_W").permute(0, 3, 1, 2), stride=stride, padding=pad)
+        y = torch.nn.functional.batch_norm(y, P(name + "_mean"), P(name + "_var"), P(name + "_gamma"),
+                                           P(name + "_beta"), training=False, eps=1e-5)
+        return torch.relu(y) if relu else y
+
+    x = torch.tensor(img, dtype=torch.float64).permute(0, 3, 1, 2)
+    x = cbn(x, "cnn_stem", 2, 3, True)
+    x = torch.nn.functional.max_pool2d(x, 3, 2, 1)
+    cin = 64
+    for li, cout in enumerate([64, 128, 256, 512]):
+        for bi in range(2):
+            s = 2 if (li > 0 and bi == 0) else 1
+            nm = f"cnn_l{li + 1}b{bi}"
+            y = cbn(x, nm + "_c1", s, 1, True)
+            y = cbn(y, nm + "_c2", 1, 1, False)
+            sc = cbn(x, nm + "_ds", s, 0, False) if (s != 1 or cin != cout) else x
+            x = torch.relu(y + sc)
+            cin = cout
+    want = x.mean(dim=(2, 3)).numpy()
+    np.testing.assert_allclose(vals["cnn_gap"], want, rtol=1e-10, atol=1e-12)
+
+
+# ---- joins --------------------------------------------------------------------------------------
+def test_joins_special_cases():
+    a = np.random.default_rng(6).normal(size=(4, 8))
+    np.testing.assert_allclose(F.cosine_join(a, a)[:, 0], 1.0, rtol=1e-14)
+    np.testing.assert_allclose(F.cosine_join(a, -a)[:, 0], -1.0, rtol=1e-14)
+    assert F.cosine_join(np.zeros((1, 3)), np.ones((1, 3)))[0, 0] == 0.0
+    l = np.full((4, 1), 0.37)
+    np.testing.assert_allclose(F.mean_join([l, l, l]), F.sigmoid(l), rtol=1e-15)
+    np.testing.assert_allclose(F.sum_join([l, -l]), 0.5, rtol=1e-15)
+    s = np.array([[0.25]])
+    np.testing.assert_allclose(F.dot_join(s, np.array([[1.0, 2.0]]), np.array([0.5, -1.0]),
+                                          np.array([0.25])), F.sigmoid(np.array([[0.25 + 0.5 - 2 + 0.25]])))
+    x = F.concat_head([np.array([[1.0]]), np.array([[2.0, 3.0]])], np.array([1.0, 1.0, -1.0]),
+                      np.array([0.0]), "none")
+    assert x[0, 0] == 0.0
+    assert F.sigmoid(np.array([-800.0, 800.0])).tolist() == [0.0, 1.0]
+
+
+# ---- IR reader ------------------------------------------------------------------------------------
+def test_ir_errors():
+    with pytest.raises(IRError):
+        parse("%a = add(%b, %b) : f32[1]\n%b = add(%a, %a) : f32[1]\n")  # cycle
+    with pytest.raises(IRError):
+        parse("%a = linear(%x, @W, @b) : f32[1]\n")  # undefined
+    with pytest.raises(IRError):
+        parse("%a = input() : f16[1]\n")  # bad dtype
+    g = parse("# c\n%x = input() : f32[2,3]\n%y = sigmoid(%x) : f32[2,3]\noutput %y\n")
+    assert [n.op for n in g.nodes] == ["input", "sigmoid"] and g.outputs == [1]

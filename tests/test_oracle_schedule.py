@@ -1,0 +1,235 @@
+"""Pins for the oracle partitioner (C2), makespan model (C3), greedy-correction (C4) and brute
+force (C5): closed forms, invariants, the paper's Table II numbers, the hand-traced
+LPT counter-example, brute-force equality, fallback on chains."""
+import itertools
+import random
+
+import pytest
+
+from oracle.partition import MULTI, SEQ, partition
+from oracle.schedule import Comm, Link, Model, brute_force, schedule
+from paper_conf_ipps_zhanghl21_b200 import workloads as W
+
+ZERO = Comm(Link(0, 0), Link(0, 0))
+
+
+def branches_ir(n, join=False):
+    """n independent opaque branches off one shared input (replicated placeholders)."""
+    lines = ["%x = input() : f32[4,4]"]
+    for i in range(n):
+        lines.append(f"%b{i} = opaque(%x) : f32[4,{i + 1}]")
+    if join:
+        lines.append(f"%y = opaque({', '.join(f'%b{i}' for i in range(n))}) : f32[4,1]")
+        lines.append("output %y")
+    else:
+        lines.append("output " + ", ".join(f"%b{i}" for i in range(n)))
+    return "\n".join(lines) + "\n"
+
+
+# ---- partition ----------------------------------------------------------------------------------
+def test_chain_is_one_sequential_subgraph():
+    ir = "%x = input() : f32[2]\n" + "".join(
+        f"%c{i} = opaque(%{'x' if i == 0 else f'c{i - 1}'}) : f32[2]\n" for i in range(6)) + "output %c5\n"
+    p = partition(ir)
+    assert p.phase_kind == [SEQ] and p.n_sg == 1 and p.node_to_sg == [-1] + [0] * 6
+    assert p.edges == {(-1, 0): 8, (0, -1): 8}
+
+
+def test_diamond_seq_multi_seq():
+    ir = """%x = input() : f32[2,4]
+%a = opaque(%x) : f32[2,4]
+%l = opaque(%a) : f32[2,8]
+%r1 = opaque(%a) : f32[2,2]
+%r2 = opaque(%r1) : f32[2,2]
+%j = opaque(%l, %r2) : f32[2,1]
+output %j
+"""
+    p = partition(ir)
+    assert p.phase_kind == [SEQ, MULTI, SEQ]
+    assert p.sg_nodes == [[1], [2], [3, 4], [5]]
+    assert p.sg_phase == [0, 1, 1, 2]
+    assert p.edges == {(-1, 0): 32, (0, 1): 32, (0, 2): 32, (1, 3): 64, (2, 3): 16, (3, -1): 8}
+    op = partition(ir, "op")
+    assert op.n_sg == 5 and op.sg_phase == [0, 1, 1, 1, 2]
+
+
+def test_residual_block_stays_sequential():
+    ir = """%x = input() : f32[2]
+%a = opaque(%x) : f32[2]
+%b = opaque(%a) : f32[2]
+%c = opaque(%b) : f32[2]
+%d = opaque(%c, %a) : f32[2]
+output %d
+"""
+    p = partition(ir)
+    assert p.phase_kind == [SEQ] and p.n_sg == 1
+
+
+def test_placeholders_and_independent_towers():
+    p = partition(branches_ir(3, join=True))
+    assert p.n_placeholders == 2
+    assert p.phase_kind == [MULTI, SEQ] and p.n_sg == 4
+    assert p.edges[(-1, 0)] == 64 and p.edges[(-1, 2)] == 64
+
+
+@pytest.mark.parametrize("cfg,coarse,op,kinds", [
+    ("c1", 4, 6, [SEQ, MULTI, SEQ]),
+    ("c2", 4, 7, [SEQ, MULTI, SEQ]),
+    ("c3", 3, 5, [MULTI, SEQ]),
+    ("c4", 4, None, [MULTI, SEQ]),
+    ("c5", 9, None, [MULTI, SEQ]),
+])
+def test_config_partitions(cfg, coarse, op, kinds):
+    wl = W.build(cfg, small=True)
+    p = partition(wl.ir)
+    assert p.n_sg == coarse and p.phase_kind == kinds
+    if op is not None:
+        assert partition(wl.ir, "op").n_sg == op
+    # coverage: every compute node in exactly one subgraph; phases alternate
+    assert sorted(v for s in p.sg_nodes for v in s) == sorted(i for i, s in enumerate(p.node_to_sg) if s >= 0)
+    assert all(a != b for a, b in zip(p.phase_kind, p.phase_kind[1:]))
+
+
+# ---- makespan model closed forms ------------------------------------------------------------------
+def test_single_slot_makespan_is_sum():
+    p = partition(W.build("c4", small=True).ir, "op")
+    T = [[1000 + 37 * s] for s in range(p.n_sg)]
+    m = Model(p, T, [0], ZERO)
+    assert m.makespan([0] * p.n_sg) == sum(r[0] for r in T)
+
+
+@pytest.mark.parametrize("n,D", [(5, 2), (7, 3), (8, 4), (3, 4)])
+def test_equal_costs_ceil(n, D):
+    p = partition(branches_ir(n))
+    m = Model(p, [[500] * D for _ in range(n)], [0] * D, ZERO)
+    a = [i % D for i in range(n)]
+    assert m.makespan(a) == -(-n // D) * 500
+    s = schedule(p, [[500] * D for _ in range(n)], [0] * D, ZERO)
+    assert s.makespan == -(-n // D) * 500
+
+
+def test_comm_charged_consumer_side():
+    # x -> a (slot0) ; x -> b (slot1, cross GPU) ; join on slot0 ; 2 GPUs
+    p = partition(branches_ir(2, join=True))
+    comm = Comm(Link(7, 0), Link(100, 2000))   # cross: 100 ns + 2 ps/B... = 2 ns/B
+    m = Model(p, [[10, 10], [20, 20], [5, 5]], [0, 1], comm)
+    # b1 bytes out = 4*2*4 = 32 B ; graph input bytes to b1 = 64 B
+    # sg1 on slot1: ready = 100 + 128 = 228, finish 248; join ready = 248 + 100 + 64 = 412
+    assert m.makespan([0, 1, 0]) == 417
+    assert m.makespan([0, 0, 0]) == 35
+
+
+# ---- Table II fixture -----------------------------------------------------------
+def test_table2_fixture():
+    p = partition(branches_ir(2))           # sg0 = "RNN", sg1 = "CNN"
+    T = [[2_400_000, 6_400_000], [14_900_000, 900_000]]   # slot 0 = "cpu", slot 1 = "gpu"
+    s = schedule(p, T, [0, 1], ZERO)
+    assert s.slot_of == [0, 1] and s.makespan == 2_400_000 and s.fell_back == 0
+    assert brute_force(p, T, [0, 1], ZERO) == (2_400_000, [0, 1])
+
+
+# ---- LPT counter-example (hand-traced) ---------------------------------------------
+def test_lpt_fixture():
+    p = partition(branches_ir(5))
+    T = [[t, t] for t in (7000, 6000, 5000, 4000, 3000)]
+    g = schedule(p, T, [0, 0], ZERO, mode=1, allow_fallback=False)
+    assert g.slot_of == [0, 1, 1, 0, 0] and g.makespan == 14000          # LPT
+    s = schedule(p, T, [0, 0], ZERO)
+    assert s.slot_of == [1, 0, 1, 0, 0] and s.makespan == 13000           # after Step 3
+    assert brute_force(p, T, [0, 0], ZERO)[0] == 13000
+    assert 14000 <= (4 / 3 - 1 / 6) * 13000                               # Graham bound
+
+
+# ---- fallback on a chain --------------------------------------------------------------
+def test_fallback_chain():
+    ir = "%x = input() : f32[2]\n%a = opaque(%x) : f32[2]\n%b = opaque(%a) : f32[2]\noutput %b\n"
+    p = partition(ir, "op")
+    T = [[300, 200], [500, 900]]
+    s = schedule(p, T, [0, 1], Comm(Link(50, 0), Link(50, 0)))
+    assert s.fell_back == 1 and s.makespan == min(800, 1100) and s.slot_of == [0, 0]
+
+
+# ---- serial / fixed modes ------------------------------------------------------------------------
+def test_serial_and_fixed_modes():
+    p = partition(branches_ir(3, join=True))
+    T = [[10, 10], [20, 20], [30, 30], [5, 5]]
+    assert schedule(p, T, [0, 0], ZERO, mode=2).makespan == 65
+    assert schedule(p, T, [0, 0], ZERO, mode=3, fixed=[1, 0, 1, 0]).makespan == 45
+
+
+# ---- brute force equality on paper-like fixtures; invariants on fuzzed DAGs ------------------------
+def random_dag_ir(rng, n_nodes):
+    lines = ["%x = input() : f32[8,8]", "%x2 = input() : f32[8,4]"]
+    names = []
+    for i in range(n_nodes):
+        k = rng.randint(0, min(2, len(names)))
+        srcs = rng.sample(names, k) if k else [rng.choice(["x", "x2"])]
+        lines.append(f"%n{i} = opaque({', '.join('%' + s for s in srcs)}) : f32[8,{rng.randint(1, 64)}]")
+        names.append(f"n{i}")
+    lines.append("output " + ", ".join(f"%{n}" for n in names[-2:]))
+    return "\n".join(lines) + "\n"
+
+
+def check_invariants(p, T, slot_gpu, comm, s):
+    m = Model(p, T, slot_gpu, comm)
+    assert s.makespan == m.makespan(s.slot_of)
+    assert m.critical_path_lb() <= m.phase_cp_sum() <= s.makespan
+    serial = m.makespan([0] * p.n_sg)
+    assert s.makespan <= serial
+    # every dependency respected in the simulated timeline
+    finish, start = {}, {}
+    t = 0
+    for ph in range(p.n_phase):
+        free = [t] * len(slot_gpu)
+        pe = t
+        for sg in m.phases[ph]:
+            d = s.slot_of[sg]
+            ready = m.c(0, d, m.in_bytes[sg]) if m.in_bytes[sg] is not None else 0
+            for u, b in m.preds[sg]:
+                ready = max(ready, finish[u] + m.c(s.slot_of[u], d, b))
+            start[sg] = max(free[d], ready)
+            finish[sg] = start[sg] + T[sg][d]
+            free[d] = finish[sg]
+            pe = max(pe, finish[sg])
+        t = pe
+    for sg in range(p.n_sg):
+        for u, b in m.preds[sg]:
+            assert start[sg] >= finish[u] + m.c(s.slot_of[u], s.slot_of[sg], b)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_fuzz_vs_brute_force(seed):
+    rng = random.Random(seed)
+    ir = random_dag_ir(rng, rng.randint(3, 9))
+    gran = "op" if seed % 2 else "coarse"
+    p = partition(ir, gran)
+    D = rng.choice([2, 3]) if p.n_sg <= 7 else 2
+    slot_gpu = [0] + [rng.randint(0, 1) for _ in range(D - 1)]
+    T = [[rng.randint(1, 50) * 1000 for _ in range(D)] for _ in range(p.n_sg)]
+    comm = Comm(Link(rng.randint(0, 2000), rng.randint(0, 3)), Link(rng.randint(0, 8000), rng.randint(0, 500)))
+    s = schedule(p, T, slot_gpu, comm)
+    check_invariants(p, T, slot_gpu, comm, s)
+    opt, _ = brute_force(p, T, slot_gpu, comm)
+    assert opt <= s.makespan
+
+
+def test_gc_near_optimal_on_paper_like_fixtures():
+    """PAPER.md:88 claims greedy-correction finds the optimum when the subgraph count is small;
+    the explicit fixtures above pin equality.  On random costs over the c1-c3 partitions the
+    heuristic is never below the optimum (sanity of both) and is optimal in most cases; the gap
+    is reported, not required to be 0."""
+    hits = total = 0
+    worst = 1.0
+    for cfg in ("c1", "c2", "c3"):
+        p = partition(W.build(cfg, small=True).ir)
+        rng = random.Random(cfg)
+        for _ in range(20):
+            T = [[rng.randint(1, 30) * 1000, rng.randint(1, 30) * 1000] for _ in range(p.n_sg)]
+            comm = Comm(Link(500, 0), Link(500, 1))
+            s = schedule(p, T, [0, 1], comm)
+            opt = brute_force(p, T, [0, 1], comm)[0]
+            assert s.makespan >= opt
+            hits += s.makespan == opt
+            total += 1
+            worst = max(worst, s.makespan / opt)
+    assert hits / total >= 0.8 and worst < 1.25, (hits, total, worst)
