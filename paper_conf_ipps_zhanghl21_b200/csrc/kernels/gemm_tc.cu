@@ -1,0 +1,308 @@
+// tcgen05 + TMA GEMM tile for sm_100a with fused epilogues.
+//
+//   D[M, N] = A[M, K] * W[N, K]^T      A, W bf16 K-major (row-major [rows, K]); fp32 accumulate
+//
+// One CTA computes one 128 x BN tile.  Warp roles (6 warps):
+//   warp 0      TMA producer: A/W k-blocks of 64 (128-B rows, SWIZZLE_128B) into a STAGES ring
+//   warp 1      TMEM allocator + single-thread tcgen05.mma issuer (UMMA 128 x BN x 16)
+//   warps 2..5  epilogue: tcgen05.ld TMEM -> registers -> fused epilogue -> global
+// Epilogues:
+//   EPI_BIAS_ACT  out = act(acc + bias[n])                      (MLP / projections, A5-A6)
+//   EPI_LSTM      gates = gx + acc; c = f*c + i*g; h = o*tanh(c) (A7, PyTorch i,f,g,o)
+//   EPI_GRU       r,z = sig(gx + acc); n = tanh(gx_n + r*(acc_n + b_hn)); h = (1-z) n + z h (A8)
+// For the RNN epilogues the weight rows are gate-block interleaved per tile: tile columns
+// [g*u, (g+1)*u) hold gate g of hidden units [tile*u, (tile+1)*u), u = BN / G, so one thread
+// owns every gate of its units.
+#include <cudaTypedefs.h>
+
+#include <cstdio>
+
+#include "../common.h"
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace duet {
+
+namespace {
+
+constexpr int BM = 128;
+constexpr int BK = 64;  // bf16: 128 bytes per row = one SWIZZLE_128B atom row
+constexpr int A_STAGE_BYTES = BM * BK * 2;
+
+template <int BN>
+struct TileCfg {
+  static constexpr int B_STAGE_BYTES = BN * BK * 2;
+  static constexpr int STAGES = BN <= 64 ? 8 : (BN <= 128 ? 6 : 4);
+  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr int SMEM = STAGES * (A_STAGE_BYTES + B_STAGE_BYTES) + 1024 + 256;
+};
+
+__device__ __forceinline__ void store16(float* dst, const float* v, int n_valid) {
+  if (n_valid >= 16 && ((uintptr_t)dst & 15) == 0) {
+    float4* d4 = reinterpret_cast<float4*>(dst);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) d4[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+  } else {
+    for (int i = 0; i < 16 && i < n_valid; ++i) dst[i] = v[i];
+  }
+}
+__device__ __forceinline__ void store16(__nv_bfloat16* dst, const float* v, int n_valid) {
+  if (n_valid >= 16 && ((uintptr_t)dst & 15) == 0) {
+    uint32_t w[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      __nv_bfloat162 p = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+      w[i] = *reinterpret_cast<uint32_t*>(&p);
+    }
+    uint4* d4 = reinterpret_cast<uint4*>(dst);
+    d4[0] = make_uint4(w[0], w[1], w[2], w[3]);
+    d4[1] = make_uint4(w[4], w[5], w[6], w[7]);
+  } else {
+    for (int i = 0; i < 16 && i < n_valid; ++i) dst[i] = __float2bfloat16_rn(v[i]);
+  }
+}
+
+template <int BN, int EPI, typename OutT>
+__global__ void __launch_bounds__(192, 1)
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
+                   const TcEpilogue ep, int M, int N, int K) {
+  using Cfg = TileCfg<BN>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + Cfg::STAGES * A_STAGE_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + Cfg::STAGES * Cfg::B_STAGE_BYTES);
+  uint64_t* empty = full + Cfg::STAGES;
+  uint64_t* tmem_full = empty + Cfg::STAGES;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
+
+  const int warp = ptx::warp_id();
+  const int lane = threadIdx.x & 31;
+  const int n0 = blockIdx.x * BN;
+  const int m0 = blockIdx.y * BM;
+  const int nk = (K + BK - 1) / BK;
+
+  if (warp == 0 && lane == 0) {
+    ptx::tma_prefetch(&tmA);
+    ptx::tma_prefetch(&tmW);
+    for (int s = 0; s < Cfg::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    ptx::mbar_init(tmem_full, 1);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) {
+    ptx::tmem_alloc(tmem_slot, Cfg::TMEM_COLS);
+    ptx::tmem_relinquish();
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % Cfg::STAGES;
+        if (kb >= Cfg::STAGES) ptx::mbar_wait(&empty[s], ((kb / Cfg::STAGES) - 1) & 1);
+        ptx::mbar_arrive_expect_tx(&full[s], A_STAGE_BYTES + Cfg::B_STAGE_BYTES);
+        ptx::tma_load_2d(&tmA, &full[s], sA + s * A_STAGE_BYTES, kb * BK, m0);
+        ptx::tma_load_2d(&tmW, &full[s], sB + s * Cfg::B_STAGE_BYTES, kb * BK, n0);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      constexpr uint32_t idesc = ptx::idesc_bf16(BM, BN);
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % Cfg::STAGES;
+        ptx::mbar_wait(&full[s], (kb / Cfg::STAGES) & 1);
+        ptx::tc_fence_after();
+        const uint32_t a_base = ptx::smem_u32(sA + s * A_STAGE_BYTES);
+        const uint32_t b_base = ptx::smem_u32(sB + s * Cfg::B_STAGE_BYTES);
+#pragma unroll
+        for (int k = 0; k < BK / 16; ++k) {
+          ptx::umma_bf16(tmem, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
+                         (kb | k) != 0);
+        }
+        ptx::umma_commit(&empty[s]);
+      }
+      ptx::umma_commit(tmem_full);
+    }
+  } else {
+    // ---------------- epilogue warps 2..5 ----------------
+    const int q = warp & 3;  // TMEM lane quarter this warp may access
+    const int row = m0 + q * 32 + lane;
+    ptx::mbar_wait(tmem_full, 0);
+    ptx::tc_fence_after();
+    const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
+    if constexpr (EPI == EPI_BIAS_ACT) {
+      OutT* out = reinterpret_cast<OutT*>(ep.out);
+#pragma unroll 1
+      for (int c = 0; c < BN / 16; ++c) {
+        float v[16];
+        ptx::tmem_ld16(tq + c * 16, v);
+        const int col0 = n0 + c * 16;
+        if (row < M && col0 < N) {
+          const int nv = min(16, N - col0);
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            float b = (ep.bias && i < nv) ? __ldg(ep.bias + col0 + i) : 0.0f;
+            v[i] = apply_act(v[i] + b, ep.act);
+          }
+          store16(out + (size_t)row * ep.ldo + col0, v, nv);
+        }
+      }
+    } else {
+      // RNN cell epilogue; G gates per unit, u units per tile, gate block g at columns [g*u, (g+1)*u)
+      constexpr int G = (EPI == EPI_LSTM) ? 4 : 3;
+      constexpr int U = BN / G;
+      const int H = ep.H;
+      const int unit0 = blockIdx.x * U;
+#pragma unroll 1
+      for (int jc = 0; jc < U; jc += 16) {
+        float acc[G][16];
+#pragma unroll
+        for (int g = 0; g < G; ++g) ptx::tmem_ld16(tq + g * U + jc, acc[g]);
+        if (row >= M) continue;
+        const float* gx = ep.gx + (size_t)row * N + (size_t)blockIdx.x * BN + jc;
+        float h[16];
+        const int nv = min(16, H - (unit0 + jc));
+        if (nv <= 0) continue;
+        if constexpr (EPI == EPI_LSTM) {
+          float* cst = ep.c_state + (size_t)row * H + unit0 + jc;
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            if (i >= nv) break;
+            float ig = sigmoidf_acc(acc[0][i] + gx[0 * U + i]);
+            float fg = sigmoidf_acc(acc[1][i] + gx[1 * U + i]);
+            float gg = tanhf(acc[2][i] + gx[2 * U + i]);
+            float og = sigmoidf_acc(acc[3][i] + gx[3 * U + i]);
+            float c = fg * cst[i] + ig * gg;
+            cst[i] = c;
+            h[i] = og * tanhf(c);
+          }
+        } else {
+          const __nv_bfloat16* hp = reinterpret_cast<const __nv_bfloat16*>(ep.h_prev) + (size_t)row * H + unit0 + jc;
+          const float* bhn = ep.b_hn + unit0 + jc;
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            if (i >= nv) break;
+            float r = sigmoidf_acc(acc[0][i] + gx[0 * U + i]);
+            float z = sigmoidf_acc(acc[1][i] + gx[1 * U + i]);
+            float n = tanhf(gx[2 * U + i] + r * (acc[2][i] + bhn[i]));
+            h[i] = (1.0f - z) * n + z * __bfloat162float(hp[i]);
+          }
+        }
+        __nv_bfloat16* hn = reinterpret_cast<__nv_bfloat16*>(ep.h_next) + (size_t)row * H + unit0 + jc;
+        store16(hn, h, nv);
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem, Cfg::TMEM_COLS);
+  }
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !p)
+      fail(DUET_ECUDA, "cannot resolve cuTensorMapEncodeTiled");
+    fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }
+  return fn;
+}
+
+template <int BN, int EPI, typename OutT>
+void launch_tc(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, int M, int N, int K,
+               cudaStream_t st) {
+  using Cfg = TileCfg<BN>;
+  auto kern = gemm_tc_kernel<BN, EPI, OutT>;
+  static bool attr_done = false;  // per instantiation; device attribute applies process-wide
+  if (!attr_done) {
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr_done = true;
+  }
+  dim3 grid((N + BN - 1) / BN, (M + BM - 1) / BM);
+  kern<<<grid, 192, Cfg::SMEM, st>>>(a, w, ep, M, N, K);
+  CK(cudaGetLastError());
+}
+
+}  // namespace
+
+CUtensorMap make_tmap_bf16_2d(const void* base, int64_t rows, int64_t cols, int box_rows) {
+  if (((uintptr_t)base & 15) || (cols * 2) % 16)
+    fail(DUET_EUNSUPPORTED, "TMA operand needs 16-byte aligned base and row pitch (K % 8 == 0)");
+  CUtensorMap m;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(cols * 2)};
+  cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = get_encode()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box,
+                            estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) fail(DUET_ECUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
+  return m;
+}
+
+int tc_pick_bn(int M, int N, int num_sms) {
+  // Smallest-waste tile width that still fills the SMs: prefer the widest BN whose tile count
+  // reaches the SM count; else the narrowest (most CTAs).
+  const int cands[] = {256, 128, 64, 32};
+  int mt = (M + BM - 1) / BM;
+  for (int bn : cands) {
+    if (bn > 128 && N < 256) continue;
+    int tiles = mt * ((N + bn - 1) / bn);
+    if (tiles >= num_sms) return bn;
+  }
+  return N <= 16 ? 16 : 32;
+}
+
+void gemm_tc(const void* A, const void* W, int M, int N, int K, int bn, const TcEpilogue& ep, int epi,
+             int out_bf16, cudaStream_t st) {
+  CUtensorMap ta = make_tmap_bf16_2d(A, M, K, BM);
+  CUtensorMap tw = make_tmap_bf16_2d(W, N, K, bn);
+  gemm_tc_maps(ta, tw, M, N, K, bn, ep, epi, out_bf16, st);
+}
+
+void gemm_tc_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
+                  int epi, int out_bf16, cudaStream_t st) {
+#define DUET_TC_CASE(BNV)                                                        \
+  case BNV:                                                                      \
+    if (epi == EPI_BIAS_ACT) {                                                   \
+      if (out_bf16)                                                              \
+        launch_tc<BNV, EPI_BIAS_ACT, __nv_bfloat16>(ta, tw, ep, M, N, K, st);    \
+      else                                                                       \
+        launch_tc<BNV, EPI_BIAS_ACT, float>(ta, tw, ep, M, N, K, st);            \
+      return;                                                                    \
+    }                                                                            \
+    break;
+  switch (bn) {
+    DUET_TC_CASE(16)
+    DUET_TC_CASE(32)
+    DUET_TC_CASE(64)
+    DUET_TC_CASE(128)
+    DUET_TC_CASE(256)
+  }
+#undef DUET_TC_CASE
+  if (epi == EPI_LSTM) {
+    if (bn == 128) return launch_tc<128, EPI_LSTM, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
+    if (bn == 256) return launch_tc<256, EPI_LSTM, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
+    if (bn == 64) return launch_tc<64, EPI_LSTM, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
+  }
+  if (epi == EPI_GRU) {
+    if (bn == 96) return launch_tc<96, EPI_GRU, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
+    if (bn == 192) return launch_tc<192, EPI_GRU, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
+    if (bn == 48) return launch_tc<48, EPI_GRU, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
+  }
+  fail(DUET_EUNSUPPORTED, "no tcgen05 tile for bn=" + std::to_string(bn) + " epi=" + std::to_string(epi));
+}
+
+}  // namespace duet

@@ -1,0 +1,237 @@
+// Branch joins, elementwise ops and pooling.  Joins are one warp per row
+// with a shuffle reduction (coalesced lane-strided reads of each branch's row).
+#include <cuda_bf16.h>
+
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace duet {
+
+namespace {
+
+__device__ __forceinline__ float ldx(const void* p, int64_t i, int bf16) {
+  return bf16 ? __bfloat162float(reinterpret_cast<const __nv_bfloat16*>(p)[i]) : reinterpret_cast<const float*>(p)[i];
+}
+__device__ __forceinline__ void stx(void* p, int64_t i, float v, int bf16) {
+  if (bf16)
+    reinterpret_cast<__nv_bfloat16*>(p)[i] = __float2bfloat16_rn(v);
+  else
+    reinterpret_cast<float*>(p)[i] = v;
+}
+
+__device__ __forceinline__ int row_of_warp() { return blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); }
+
+__global__ void reduce_sum_kernel(const void* x, int bf16, const float* b, float* y, int B, int K) {
+  int row = row_of_warp(), lane = threadIdx.x & 31;
+  if (row >= B) return;
+  float s = 0.0f;
+  for (int k = lane; k < K; k += 32) s += ldx(x, (int64_t)row * K + k, bf16);
+  s = warp_sum(s);
+  if (lane == 0) y[row] = s + b[0];
+}
+
+__global__ void dot_join_kernel(const float* s, const void* a, int bf16, const float* w, const float* b, float* y,
+                                int B, int K) {
+  int row = row_of_warp(), lane = threadIdx.x & 31;
+  if (row >= B) return;
+  float acc = 0.0f;
+  for (int k = lane; k < K; k += 32) acc = fmaf(ldx(a, (int64_t)row * K + k, bf16), w[k], acc);
+  acc = warp_sum(acc);
+  if (lane == 0) y[row] = sigmoidf_acc(s[row] + acc + b[0]);
+}
+
+__global__ void cosine_join_kernel(const void* a, const void* b, int bf16, float* y, int B, int K) {
+  int row = row_of_warp(), lane = threadIdx.x & 31;
+  if (row >= B) return;
+  float ab = 0.0f, aa = 0.0f, bb = 0.0f;
+  for (int k = lane; k < K; k += 32) {
+    float x = ldx(a, (int64_t)row * K + k, bf16), z = ldx(b, (int64_t)row * K + k, bf16);
+    ab = fmaf(x, z, ab);
+    aa = fmaf(x, x, aa);
+    bb = fmaf(z, z, bb);
+  }
+  ab = warp_sum(ab);
+  aa = warp_sum(aa);
+  bb = warp_sum(bb);
+  if (lane == 0) {
+    float den = sqrtf(aa) * sqrtf(bb);
+    y[row] = den > 0.0f ? ab / den : 0.0f;
+  }
+}
+
+struct HeadArgs {
+  const void* p[8];
+  int K[8];
+  int bf16[8];
+  int n;
+};
+
+__global__ void concat_head_kernel(HeadArgs h, const float* w, const float* b, float* y, int B, int act) {
+  int row = row_of_warp(), lane = threadIdx.x & 31;
+  if (row >= B) return;
+  float acc = 0.0f;
+  int off = 0;
+  for (int i = 0; i < h.n; ++i) {
+    for (int k = lane; k < h.K[i]; k += 32) acc = fmaf(ldx(h.p[i], (int64_t)row * h.K[i] + k, h.bf16[i]), w[off + k], acc);
+    off += h.K[i];
+  }
+  acc = warp_sum(acc);
+  if (lane == 0) y[row] = apply_act(acc + b[0], act);
+}
+
+struct LogitArgs {
+  const float* p[16];
+  int n;
+};
+
+__global__ void logit_join_kernel(LogitArgs a, float* y, int B, int mean) {
+  int row = blockIdx.x * blockDim.x + threadIdx.x;
+  if (row >= B) return;
+  float s = 0.0f;
+  for (int i = 0; i < a.n; ++i) s += a.p[i][row];
+  if (mean) s /= (float)a.n;
+  y[row] = sigmoidf_acc(s);
+}
+
+template <typename T>
+__global__ void add_act_kernel(const T* a, const T* b, T* y, int64_t n, int act) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    y[i] = from_f<T>(apply_act(to_f(a[i]) + to_f(b[i]), act));
+}
+
+template <typename T>
+__global__ void sigmoid_kernel(const T* x, T* y, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    y[i] = from_f<T>(sigmoidf_acc(to_f(x[i])));
+}
+
+template <typename T>
+__global__ void maxpool_kernel(const T* x, T* y, int N, int H, int W, int C, int k, int s, int p, int Ho, int Wo) {
+  int64_t total = (int64_t)N * Ho * Wo * C;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    int c = (int)(i % C);
+    int64_t t = i / C;
+    int wo = (int)(t % Wo);
+    t /= Wo;
+    int ho = (int)(t % Ho);
+    int n = (int)(t / Ho);
+    float m = -INFINITY;
+    for (int r = 0; r < k; ++r) {
+      int hi = ho * s - p + r;
+      if (hi < 0 || hi >= H) continue;
+      for (int q = 0; q < k; ++q) {
+        int wi = wo * s - p + q;
+        if (wi < 0 || wi >= W) continue;
+        m = fmaxf(m, to_f(x[(((int64_t)n * H + hi) * W + wi) * C + c]));
+      }
+    }
+    y[i] = from_f<T>(m);
+  }
+}
+
+// global average pool: one thread per (n, c), coalesced over c
+template <typename T>
+__global__ void avgpool_kernel(const T* x, T* y, int N, int HW, int C) {
+  int64_t total = (int64_t)N * C;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    int c = (int)(i % C);
+    int64_t n = i / C;
+    float s = 0.0f;
+    const T* base = x + n * HW * C + c;
+    for (int j = 0; j < HW; ++j) s += to_f(base[(int64_t)j * C]);
+    y[i] = from_f<T>(s / (float)HW);
+  }
+}
+
+int warp_rows_grid(int B) { return (B + 7) / 8; }
+
+}  // namespace
+
+void reduce_sum(const void* x, int x_bf16, const float* b, float* y, int B, int K, cudaStream_t st) {
+  if (!B) return;
+  reduce_sum_kernel<<<warp_rows_grid(B), 256, 0, st>>>(x, x_bf16, b, y, B, K);
+  CK(cudaGetLastError());
+}
+
+void dot_join(const float* s, const void* a, int a_bf16, const float* w, const float* b, float* y, int B, int K,
+              cudaStream_t st) {
+  if (!B) return;
+  dot_join_kernel<<<warp_rows_grid(B), 256, 0, st>>>(s, a, a_bf16, w, b, y, B, K);
+  CK(cudaGetLastError());
+}
+
+void cosine_join(const void* a, const void* b, int bf16, float* y, int B, int K, cudaStream_t st) {
+  if (!B) return;
+  cosine_join_kernel<<<warp_rows_grid(B), 256, 0, st>>>(a, b, bf16, y, B, K);
+  CK(cudaGetLastError());
+}
+
+void concat_head(const void* const* parts, const int* Ks, const int* bf16s, int n, const float* w, const float* b,
+                 float* y, int B, int act, cudaStream_t st) {
+  if (n > 8) fail(DUET_EUNSUPPORTED, "concat_head: at most 8 parts");
+  HeadArgs h{};
+  for (int i = 0; i < n; ++i) {
+    h.p[i] = parts[i];
+    h.K[i] = Ks[i];
+    h.bf16[i] = bf16s[i];
+  }
+  h.n = n;
+  if (!B) return;
+  concat_head_kernel<<<warp_rows_grid(B), 256, 0, st>>>(h, w, b, y, B, act);
+  CK(cudaGetLastError());
+}
+
+void logit_join(const float* const* parts, int n, float* y, int B, int mean, cudaStream_t st) {
+  if (n > 16) fail(DUET_EUNSUPPORTED, "logit join: at most 16 branches");
+  LogitArgs a{};
+  for (int i = 0; i < n; ++i) a.p[i] = parts[i];
+  a.n = n;
+  if (!B) return;
+  logit_join_kernel<<<(B + 255) / 256, 256, 0, st>>>(a, y, B, mean);
+  CK(cudaGetLastError());
+}
+
+void add_act(const void* a, const void* b, void* y, int bf16, int64_t n, int act, cudaStream_t st) {
+  if (!n) return;
+  if (bf16)
+    add_act_kernel<__nv_bfloat16><<<grid_for(n, 256), 256, 0, st>>>((const __nv_bfloat16*)a, (const __nv_bfloat16*)b,
+                                                                  (__nv_bfloat16*)y, n, act);
+  else
+    add_act_kernel<float><<<grid_for(n, 256), 256, 0, st>>>((const float*)a, (const float*)b, (float*)y, n, act);
+  CK(cudaGetLastError());
+}
+
+void sigmoid_ew(const void* x, void* y, int bf16, int64_t n, cudaStream_t st) {
+  if (!n) return;
+  if (bf16)
+    sigmoid_kernel<__nv_bfloat16><<<grid_for(n, 256), 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, n);
+  else
+    sigmoid_kernel<float><<<grid_for(n, 256), 256, 0, st>>>((const float*)x, (float*)y, n);
+  CK(cudaGetLastError());
+}
+
+void maxpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, int k, int s, int p, int Ho, int Wo,
+                  cudaStream_t st) {
+  int64_t total = (int64_t)N * Ho * Wo * C;
+  if (!total) return;
+  if (bf16)
+    maxpool_kernel<__nv_bfloat16><<<grid_for(total, 256), 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, N,
+                                                                       H, W, C, k, s, p, Ho, Wo);
+  else
+    maxpool_kernel<float><<<grid_for(total, 256), 256, 0, st>>>((const float*)x, (float*)y, N, H, W, C, k, s, p, Ho,
+                                                               Wo);
+  CK(cudaGetLastError());
+}
+
+void avgpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, cudaStream_t st) {
+  int64_t total = (int64_t)N * C;
+  if (!total) return;
+  if (bf16)
+    avgpool_kernel<__nv_bfloat16><<<grid_for(total, 256), 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, N,
+                                                                       H * W, C);
+  else
+    avgpool_kernel<float><<<grid_for(total, 256), 256, 0, st>>>((const float*)x, (float*)y, N, H * W, C);
+  CK(cudaGetLastError());
+}
+
+}  // namespace duet

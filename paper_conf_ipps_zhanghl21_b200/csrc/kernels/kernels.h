@@ -1,0 +1,99 @@
+// Host-side launchers of the sm_100a kernels (all enqueue on the given stream, no sync).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <string>
+
+#include "../common.h"
+
+namespace duet {
+
+#define CK(x)                                                                                     \
+  do {                                                                                            \
+    cudaError_t e_ = (x);                                                                         \
+    if (e_ != cudaSuccess)                                                                        \
+      ::duet::fail(DUET_ECUDA, std::string(#x) + ": " + cudaGetErrorString(e_) + " @" __FILE__ ":" + \
+                                   std::to_string(__LINE__));                                     \
+  } while (0)
+
+enum { EPI_BIAS_ACT = 0, EPI_LSTM = 1, EPI_GRU = 2 };
+enum Act { ACT_NONE = 0, ACT_RELU = 1, ACT_SIGMOID = 2, ACT_TANH = 3 };
+
+struct TcEpilogue {
+  // EPI_BIAS_ACT
+  const float* bias = nullptr;
+  void* out = nullptr;
+  int ldo = 0;
+  int act = 0;
+  // EPI_LSTM / EPI_GRU
+  const float* gx = nullptr;   // [M, N] step pre-activations (gate-block layout, biases folded)
+  float* c_state = nullptr;    // LSTM cell state [M, H] fp32
+  const void* h_prev = nullptr;// [M, H] bf16 (GRU z*h term)
+  void* h_next = nullptr;      // [M, H] bf16
+  const float* b_hn = nullptr; // GRU [H]
+  int H = 0;
+};
+
+// ---- tcgen05 GEMM (gemm_tc.cu) ----
+CUtensorMap make_tmap_bf16_2d(const void* base, int64_t rows, int64_t cols, int box_rows);
+int tc_pick_bn(int M, int N, int num_sms);
+void gemm_tc(const void* A, const void* W, int M, int N, int K, int bn, const TcEpilogue& ep, int epi,
+             int out_bf16, cudaStream_t st);
+void gemm_tc_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
+                  int epi, int out_bf16, cudaStream_t st);
+
+// ---- SIMT fallbacks / small kernels (simt.cu) ----
+// Y[M,N] = act(X[M,K] W[N,K]^T + b) ; X/W dtype per flags; fp32 accumulate.
+void gemm_simt(const void* X, int x_bf16, const void* W, int w_bf16, const float* b, void* Y, int y_bf16, int M,
+               int N, int K, int act, cudaStream_t st);
+// Fused small-M MLP (all layers in one CTA per row block). dims[0..L], act on all but last.
+void mlp_small(const void* X, int bf16, const void* const* Ws, const float* const* bs, const int* dims, int L,
+               void* Y, int y_bf16, int M, int act, int last_act, cudaStream_t st);
+// RNN step, SIMT (f32 parity path): gates from h_prev W_hh^T + gx (original PyTorch layout).
+void rnn_step_simt(int kind, const float* gx, const void* Whh, int w_bf16, const float* bhh_n, const void* h_prev,
+                   void* h_next, int h_bf16, float* c_state, int M, int H, cudaStream_t st);
+
+// ---- gathers (gather.cu) ----
+void hash_mod(const int64_t* raw, int32_t* ids, int64_t n, int64_t V, cudaStream_t st);
+void gather_sum(const int32_t* ids, const void* T, int t_bf16, const float* b, float* y, int B, int F, int64_t R,
+                cudaStream_t st);
+void gather_concat(const int32_t* ids, const void* E, int esize, void* X, int B, int F, int64_t R, int D,
+                   cudaStream_t st);
+void embed_seq(const int32_t* tok, const void* E, int esize, void* X, int B, int S, int64_t V, int D,
+               cudaStream_t st);
+void fill_random(void* p, int dtype, int64_t n, int64_t high, uint64_t seed, cudaStream_t st);
+void permute_rows(const void* src, void* dst, const int32_t* src_row_of_dst, int64_t rows_dst, int64_t row_bytes,
+                  cudaStream_t st);
+
+// ---- joins / elementwise / pooling (join.cu) ----
+void reduce_sum(const void* x, int x_bf16, const float* b, float* y, int B, int K, cudaStream_t st);
+void dot_join(const float* s, const void* a, int a_bf16, const float* w, const float* b, float* y, int B, int K,
+              cudaStream_t st);
+void cosine_join(const void* a, const void* b, int bf16, float* y, int B, int K, cudaStream_t st);
+// y = act(sum_i parts_i . w_i + b); parts given as (ptr, K_i, bf16_i)
+void concat_head(const void* const* parts, const int* Ks, const int* bf16s, int n, const float* w, const float* b,
+                 float* y, int B, int act, cudaStream_t st);
+void logit_join(const float* const* parts, int n, float* y, int B, int mean, cudaStream_t st);
+void add_act(const void* a, const void* b, void* y, int bf16, int64_t n, int act, cudaStream_t st);
+void sigmoid_ew(const void* x, void* y, int bf16, int64_t n, cudaStream_t st);
+void maxpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, int k, int s, int p, int Ho,
+                  int Wo, cudaStream_t st);
+void avgpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, cudaStream_t st);
+
+// ---- convolution (conv.cu) ----
+struct ConvShape {
+  int N, H, W, C, Co, kh, kw, stride, pad, Ho, Wo;
+};
+// y = act(conv(x, Wf) + bias (+ residual)); Wf [Co, kh, kw, C] with BN folded; NHWC.
+void conv_fwd(const void* x, const void* Wf, const float* bias, const void* residual, void* y, int bf16,
+              const ConvShape& s, int act, cudaStream_t st);
+// Fold BN into conv weights/bias: Wf = W * g/sqrt(var+eps), bias = beta - mean*g/sqrt(var+eps)
+void fold_bn(const void* W, int bf16, const float* g, const float* beta, const float* mean, const float* var,
+             void* Wf, float* bias, int Co, int64_t per_co, cudaStream_t st);
+
+int num_sms(int device);
+// blocks for a grid-stride kernel: enough for `work` items, capped at per_sm x SM count
+int grid_for(int64_t work, int threads, int per_sm = 8);
+
+}  // namespace duet

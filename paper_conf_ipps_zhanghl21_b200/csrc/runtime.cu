@@ -1,0 +1,834 @@
+// Device runtime: the compiled program of a bound graph, the executor and the profiler.
+//
+//  * Program  — one "compiled subgraph" per IR node ("going through the DL
+//    compilation pipeline"): the node's sm_100a kernels, prepared weights (BN folded, RNN gates
+//    block-interleaved), TMA descriptors and its library-owned output buffer.
+//  * Executor — PAPER.md:82 (§IV-D) spawns two busy-looping processes fed by shared-memory
+//    queues; on a B200 the equivalent is ONE CUDA graph per schedule: every subgraph's kernels are
+//    captured on its slot's stream in schedule order, cross-slot dependencies become event edges
+//    (the sync queue), and a replay is a single cudaGraphLaunch on the home stream.
+//  * Profiler — PAPER.md:80 (§IV-B) / :87 (500 runs): each subgraph is captured alone and timed
+//    with CUDA events (samples of R replays; lower median, int64 ns).
+#include <algorithm>
+#include <cstring>
+#include <functional>
+
+#include "common.h"
+#include "kernels/kernels.h"
+
+namespace duet {
+
+// ------------------------------------------------------------------------------------------------
+// Program
+// ------------------------------------------------------------------------------------------------
+using Ptrs = std::vector<void*>;
+
+struct Op {
+  std::function<void(const Ptrs&, cudaStream_t)> launch;
+  int n_kernels = 0;
+};
+
+struct Program {
+  const Graph* g = nullptr;
+  int device = 0;
+  std::vector<void*> buf;                  // per node: library output buffer (inputs: staging)
+  std::vector<Op> ops;                     // per node
+  std::vector<void*> allocs;               // device memory to free
+  ~Program() {
+    int prev = 0;
+    cudaGetDevice(&prev);
+    cudaSetDevice(device);
+    for (void* p : allocs) cudaFree(p);
+    cudaSetDevice(prev);
+  }
+  void* alloc(int64_t bytes) {
+    void* p = nullptr;
+    if (bytes <= 0) bytes = 16;
+    cudaError_t e = cudaMalloc(&p, (size_t)((bytes + 255) / 256 * 256));
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      fail(e == cudaErrorMemoryAllocation ? DUET_ENOMEM : DUET_ECUDA,
+           std::string("cudaMalloc(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+    }
+    allocs.push_back(p);
+    return p;
+  }
+  void* param(const std::string& name) const {
+    auto it = g->bound.find(name);
+    if (it == g->bound.end()) fail(DUET_EUNBOUND, "parameter @" + name + " is not bound");
+    return it->second.data;
+  }
+};
+
+void destroy_program(Program* p) { delete p; }
+
+namespace {
+
+struct DeviceGuard {
+  int prev = 0;
+  explicit DeviceGuard(int d) {
+    CK(cudaGetDevice(&prev));
+    if (prev != d) CK(cudaSetDevice(d));
+  }
+  ~DeviceGuard() { cudaSetDevice(prev); }
+};
+
+int act_code(const std::string& a) {
+  if (a == "none") return ACT_NONE;
+  if (a == "relu") return ACT_RELU;
+  if (a == "sigmoid") return ACT_SIGMOID;
+  if (a == "tanh") return ACT_TANH;
+  fail(DUET_EPARSE, "unknown activation '" + a + "'");
+}
+
+void need_dtype(const Node& n, int have, int want, const std::string& what) {
+  if (have != want)
+    fail(DUET_EDTYPE, "%" + n.name + ": " + what + " is " + dtype_name(have) + ", expected " + dtype_name(want));
+}
+
+bool is_float(int d) { return d == kF32 || d == kBF16; }
+
+// combined RNN input bias in the (possibly reordered) column layout:
+//   LSTM: b_ih + b_hh for all gates; GRU: b_ih + b_hh for r,z; b_ih only for n (b_hn is applied
+//   inside r*(...), PyTorch convention).
+__global__ void rnn_bias_kernel(const float* bih, const float* bhh, const int32_t* old_of_new, float* out, int n_new,
+                                int H, int is_gru) {
+  int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n_new) return;
+  int o = old_of_new[i];
+  if (o < 0) {
+    out[i] = 0.0f;
+    return;
+  }
+  float b = bih[o];
+  if (!(is_gru && o >= 2 * H)) b += bhh[o];
+  out[i] = b;
+}
+
+int rnn_step_bn(int kind, int B, int H, int sms) {
+  // tile width for the recurrent step: LSTM u in {16,32,64} (BN = 4u), GRU u in {16,32,64} (BN = 3u)
+  const int G = kind == EPI_LSTM ? 4 : 3;
+  const int mt = (B + 127) / 128;
+  int best = 0;
+  for (int u : {64, 32, 16}) {
+    int tiles = mt * ((H + u - 1) / u);
+    best = G * u;
+    if (tiles >= sms / 2) return G * u;  // enough CTAs: keep the wider tile
+  }
+  return best;  // u = 16: most CTAs
+}
+
+void build_op(Program& P, const Node& n, Op& op) {
+  const Graph& g = *P.g;
+  auto argn = [&](int i) -> const Node& { return g.nodes[n.arg_nodes.at(i)]; };
+  auto pdecl = [&](int i) -> const ParamDecl& { return g.params.at(n.params.at(i)); };
+  auto nargs = [&](size_t k, size_t p) {
+    if (n.arg_nodes.size() != k || n.params.size() != p)
+      fail(DUET_EPARSE, "%" + n.name + " = " + n.op + ": wrong number of arguments");
+  };
+  const int me = n.id;
+  const int sms = num_sms(P.device);
+
+  if (n.op == "input") return;
+  if (n.op == "opaque") fail(DUET_EUNSUPPORTED, "%" + n.name + ": opaque nodes have no kernel");
+
+  if (n.op == "hash_mod") {
+    nargs(1, 0);
+    need_dtype(n, argn(0).dtype, kI64, "input");
+    need_dtype(n, n.dtype, kI32, "output");
+    const int in = n.arg_nodes[0];
+    const int64_t V = n.attr_int("V", 0), cnt = n.numel();
+    if (V <= 0 || V > INT32_MAX) fail(DUET_EINVAL, "%" + n.name + ": V out of range");
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { hash_mod((const int64_t*)T[in], (int32_t*)T[me], cnt, V, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "gather_sum") {
+    nargs(1, 2);
+    need_dtype(n, argn(0).dtype, kI32, "ids");
+    need_dtype(n, n.dtype, kF32, "output");
+    const auto& t = pdecl(0);
+    if (t.shape.size() != 2 || argn(0).shape.size() != 2 || t.shape[0] != argn(0).shape[1])
+      fail(DUET_ESHAPE, "%" + n.name + ": table must be [F, R] with F = ids.shape[1]");
+    const int in = n.arg_nodes[0], B = (int)argn(0).shape[0], F = (int)argn(0).shape[1];
+    const int64_t R = t.shape[1];
+    const int tb = t.dtype == kBF16;
+    void* T0 = P.param(n.params[0]);
+    const float* b = (const float*)P.param(n.params[1]);
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      gather_sum((const int32_t*)T[in], T0, tb, b, (float*)T[me], B, F, R, st);
+    };
+    op.n_kernels = 1;
+  } else if (n.op == "gather_concat") {
+    nargs(1, 1);
+    need_dtype(n, argn(0).dtype, kI32, "ids");
+    const auto& e = pdecl(0);
+    need_dtype(n, n.dtype, e.dtype, "output");
+    if (e.shape.size() != 3 || e.shape[0] != argn(0).shape[1])
+      fail(DUET_ESHAPE, "%" + n.name + ": table must be [F, R, D]");
+    const int in = n.arg_nodes[0], B = (int)argn(0).shape[0], F = (int)argn(0).shape[1], D = (int)e.shape[2];
+    const int64_t R = e.shape[1];
+    const int es = dtype_bytes(e.dtype);
+    void* E = P.param(n.params[0]);
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      gather_concat((const int32_t*)T[in], E, es, T[me], B, F, R, D, st);
+    };
+    op.n_kernels = 1;
+  } else if (n.op == "embed_seq") {
+    nargs(1, 1);
+    need_dtype(n, argn(0).dtype, kI32, "tokens");
+    const auto& e = pdecl(0);
+    need_dtype(n, n.dtype, e.dtype, "output");
+    const int in = n.arg_nodes[0], B = (int)argn(0).shape[0], S = (int)argn(0).shape[1], D = (int)e.shape[1];
+    const int64_t V = e.shape[0];
+    const int es = dtype_bytes(e.dtype);
+    void* E = P.param(n.params[0]);
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      embed_seq((const int32_t*)T[in], E, es, T[me], B, S, V, D, st);
+    };
+    op.n_kernels = 1;
+  } else if (n.op == "linear") {
+    nargs(1, 2);
+    const Node& x = argn(0);
+    const auto& w = pdecl(0);
+    if (w.shape.size() != 2 || x.shape.size() != 2 || w.shape[1] != x.shape[1] || n.shape[1] != w.shape[0])
+      fail(DUET_ESHAPE, "%" + n.name + ": linear shapes");
+    const int in = n.arg_nodes[0], M = (int)x.shape[0], K = (int)x.shape[1], N = (int)w.shape[0];
+    const int act = act_code(n.attr_str("act", "none"));
+    void* W = P.param(n.params[0]);
+    const float* b = (const float*)P.param(n.params[1]);
+    const int xb = x.dtype == kBF16, wb = w.dtype == kBF16, yb = n.dtype == kBF16;
+    if (xb && wb && K % 8 == 0 && N >= 16) {
+      const int bn = tc_pick_bn(M, N, sms);
+      CUtensorMap tw = make_tmap_bf16_2d(W, N, K, bn);
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        CUtensorMap ta = make_tmap_bf16_2d(T[in], M, K, 128);
+        TcEpilogue ep;
+        ep.bias = b;
+        ep.out = T[me];
+        ep.ldo = N;
+        ep.act = act;
+        gemm_tc_maps(ta, tw, M, N, K, bn, ep, EPI_BIAS_ACT, yb, st);
+      };
+    } else {
+      op.launch = [=](const Ptrs& T, cudaStream_t st) { gemm_simt(T[in], xb, W, wb, b, T[me], yb, M, N, K, act, st); };
+    }
+    op.n_kernels = 1;
+  } else if (n.op == "mlp") {
+    if (n.arg_nodes.size() != 1 || n.params.size() < 2 || n.params.size() % 2)
+      fail(DUET_EPARSE, "%" + n.name + ": mlp(%x, @W0, @b0, ...)");
+    const Node& x = argn(0);
+    const int L = (int)n.params.size() / 2;
+    std::vector<int> dims{(int)x.shape[1]};
+    std::vector<void*> Ws;
+    std::vector<const float*> bs;
+    int wdt = pdecl(0).dtype;
+    for (int l = 0; l < L; ++l) {
+      const auto& w = pdecl(2 * l);
+      if (w.shape.size() != 2 || w.shape[1] != dims.back()) fail(DUET_ESHAPE, "%" + n.name + ": mlp layer shapes");
+      need_dtype(n, w.dtype, wdt, "weights");
+      dims.push_back((int)w.shape[0]);
+      Ws.push_back(P.param(n.params[2 * l]));
+      bs.push_back((const float*)P.param(n.params[2 * l + 1]));
+    }
+    need_dtype(n, x.dtype, wdt, "input");
+    const int in = n.arg_nodes[0], M = (int)x.shape[0];
+    const int act = act_code(n.attr_str("act", "relu")), last = act_code(n.attr_str("last_act", "none"));
+    const int xb = x.dtype == kBF16, yb = n.dtype == kBF16;
+    if (M <= 64) {
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        std::vector<const void*> w(Ws.begin(), Ws.end());
+        mlp_small(T[in], xb, w.data(), bs.data(), dims.data(), L, T[me], yb, M, act, last, st);
+      };
+      op.n_kernels = 1;
+    } else {
+      std::vector<void*> mids;
+      for (int l = 0; l + 1 < L; ++l) mids.push_back(P.alloc((int64_t)M * dims[l + 1] * dtype_bytes(x.dtype)));
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        const void* cur = T[in];
+        for (int l = 0; l < L; ++l) {
+          void* out = (l + 1 == L) ? T[me] : mids[l];
+          int ob = (l + 1 == L) ? yb : xb;
+          gemm_simt(cur, xb, Ws[l], xb, bs[l], out, ob, M, dims[l + 1], dims[l], l + 1 == L ? last : act, st);
+          cur = out;
+        }
+      };
+      op.n_kernels = L;
+    }
+  } else if (n.op == "reduce_sum") {
+    nargs(1, 1);
+    need_dtype(n, n.dtype, kF32, "output");
+    const Node& x = argn(0);
+    const int in = n.arg_nodes[0], B = (int)x.shape[0], K = (int)x.shape[1], xb = x.dtype == kBF16;
+    const float* b = (const float*)P.param(n.params[0]);
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { reduce_sum(T[in], xb, b, (float*)T[me], B, K, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "lstm" || n.op == "gru") {
+    nargs(1, 4);
+    const int kind = n.op == "lstm" ? EPI_LSTM : EPI_GRU;
+    const int G = kind == EPI_LSTM ? 4 : 3;
+    const Node& x = argn(0);
+    const auto& wih = pdecl(0);
+    const auto& whh = pdecl(1);
+    if (x.shape.size() != 3) fail(DUET_ESHAPE, "%" + n.name + ": input must be [S, B, E]");
+    const int S = (int)x.shape[0], B = (int)x.shape[1], E = (int)x.shape[2], H = (int)whh.shape[1];
+    if (wih.shape[0] != G * H || wih.shape[1] != E || whh.shape[0] != G * H || n.shape[1] != H || n.shape[0] != B)
+      fail(DUET_ESHAPE, "%" + n.name + ": rnn weight shapes");
+    need_dtype(n, wih.dtype, whh.dtype, "W_ih");
+    need_dtype(n, x.dtype, wih.dtype, "input");
+    need_dtype(n, n.dtype, x.dtype, "output");
+    const int in = n.arg_nodes[0];
+    void* Wih = P.param(n.params[0]);
+    void* Whh = P.param(n.params[1]);
+    const float* bih = (const float*)P.param(n.params[2]);
+    const float* bhh = (const float*)P.param(n.params[3]);
+    const bool tc = x.dtype == kBF16 && E % 8 == 0 && H % 8 == 0;
+    const int es = dtype_bytes(x.dtype);
+    // column layout of the gate pre-activations
+    int bn = tc ? rnn_step_bn(kind, B, H, sms) : 0;
+    const int U = tc ? bn / G : H;
+    const int tiles = tc ? (H + U - 1) / U : 1;
+    const int Np = tc ? tiles * bn : G * H;
+    std::vector<int32_t> old_of_new(Np);
+    for (int r = 0; r < Np; ++r) {
+      if (!tc) {
+        old_of_new[r] = r;
+        continue;
+      }
+      int t = r / bn, rem = r % bn, gate = rem / U, j = t * U + rem % U;
+      old_of_new[r] = j < H ? gate * H + j : -1;
+    }
+    int32_t* d_map = (int32_t*)P.alloc((int64_t)Np * 4);
+    CK(cudaMemcpy(d_map, old_of_new.data(), (size_t)Np * 4, cudaMemcpyHostToDevice));
+    float* bias = (float*)P.alloc((int64_t)Np * 4);
+    rnn_bias_kernel<<<(Np + 255) / 256, 256>>>(bih, bhh, d_map, bias, Np, H, kind == EPI_GRU);
+    CK(cudaGetLastError());
+    const float* bhn = bhh + 2 * H;
+    float* gx = (float*)P.alloc((int64_t)S * B * Np * 4);
+    void* hb[2] = {P.alloc((int64_t)B * H * es), P.alloc((int64_t)B * H * es)};
+    float* cst = (float*)P.alloc((int64_t)B * H * 4);
+    if (tc) {
+      void* Wih_r = P.alloc((int64_t)Np * E * es);
+      void* Whh_r = P.alloc((int64_t)Np * H * es);
+      permute_rows(Wih, Wih_r, d_map, Np, (int64_t)E * es, 0);
+      permute_rows(Whh, Whh_r, d_map, Np, (int64_t)H * es, 0);
+      CK(cudaDeviceSynchronize());
+      const int bn_in = tc_pick_bn(S * B, Np, sms);
+      CUtensorMap t_wih = make_tmap_bf16_2d(Wih_r, Np, E, bn_in);
+      CUtensorMap t_whh = make_tmap_bf16_2d(Whh_r, Np, H, bn);
+      CUtensorMap t_h[2] = {make_tmap_bf16_2d(hb[0], B, H, 128), make_tmap_bf16_2d(hb[1], B, H, 128)};
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        CK(cudaMemsetAsync(hb[1], 0, (size_t)B * H * es, st));
+        if (kind == EPI_LSTM) CK(cudaMemsetAsync(cst, 0, (size_t)B * H * 4, st));
+        CUtensorMap tx = make_tmap_bf16_2d(T[in], (int64_t)S * B, E, 128);
+        TcEpilogue ep;
+        ep.bias = bias;
+        ep.out = gx;
+        ep.ldo = Np;
+        ep.act = ACT_NONE;
+        gemm_tc_maps(tx, t_wih, S * B, Np, E, bn_in, ep, EPI_BIAS_ACT, 0, st);
+        for (int t = 0; t < S; ++t) {
+          TcEpilogue e2;
+          e2.gx = gx + (size_t)t * B * Np;
+          e2.c_state = cst;
+          e2.h_prev = hb[(t + 1) & 1];
+          e2.h_next = (t == S - 1) ? T[me] : hb[t & 1];
+          e2.b_hn = bhn;
+          e2.H = H;
+          gemm_tc_maps(t_h[(t + 1) & 1], t_whh, B, Np, H, bn, e2, kind, 1, st);
+        }
+      };
+    } else {
+      const int xb = x.dtype == kBF16;
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        CK(cudaMemsetAsync(hb[1], 0, (size_t)B * H * es, st));
+        if (kind == EPI_LSTM) CK(cudaMemsetAsync(cst, 0, (size_t)B * H * 4, st));
+        gemm_simt(T[in], xb, Wih, xb, bias, gx, 0, S * B, G * H, E, ACT_NONE, st);
+        for (int t = 0; t < S; ++t) {
+          void* hn = (t == S - 1) ? T[me] : hb[t & 1];
+          rnn_step_simt(kind, gx + (size_t)t * B * G * H, Whh, xb, bhn, hb[(t + 1) & 1], hn, xb, cst, B, H, st);
+        }
+      };
+    }
+    op.n_kernels = 1 + S;
+  } else if (n.op == "conv2d_bn") {
+    nargs(1, 5);
+    const Node& x = argn(0);
+    const auto& w = pdecl(0);
+    if (x.shape.size() != 4 || w.shape.size() != 4 || w.shape[3] != x.shape[3])
+      fail(DUET_ESHAPE, "%" + n.name + ": conv shapes");
+    need_dtype(n, x.dtype, w.dtype, "input");
+    need_dtype(n, n.dtype, x.dtype, "output");
+    ConvShape s{(int)x.shape[0], (int)x.shape[1], (int)x.shape[2], (int)x.shape[3], (int)w.shape[0], (int)w.shape[1],
+                (int)w.shape[2], (int)n.attr_int("stride", 1), (int)n.attr_int("pad", 0), 0, 0};
+    s.Ho = (s.H + 2 * s.pad - s.kh) / s.stride + 1;
+    s.Wo = (s.W + 2 * s.pad - s.kw) / s.stride + 1;
+    if (n.shape != std::vector<int64_t>{s.N, s.Ho, s.Wo, s.Co}) fail(DUET_ESHAPE, "%" + n.name + ": conv output shape");
+    const int bf = x.dtype == kBF16, act = act_code(n.attr_str("act", "none"));
+    const int64_t per_co = (int64_t)s.kh * s.kw * s.C;
+    void* Wf = P.alloc((int64_t)s.Co * per_co * dtype_bytes(w.dtype));
+    float* bias = (float*)P.alloc((int64_t)s.Co * 4);
+    fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
+            (const float*)P.param(n.params[3]), (const float*)P.param(n.params[4]), Wf, bias, s.Co, per_co, 0);
+    const int in = n.arg_nodes[0];
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { conv_fwd(T[in], Wf, bias, nullptr, T[me], bf, s, act, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "add") {
+    nargs(2, 0);
+    need_dtype(n, argn(0).dtype, n.dtype, "a");
+    need_dtype(n, argn(1).dtype, n.dtype, "b");
+    if (argn(0).numel() != n.numel() || argn(1).numel() != n.numel()) fail(DUET_ESHAPE, "%" + n.name + ": add shapes");
+    const int a = n.arg_nodes[0], b = n.arg_nodes[1], bf = n.dtype == kBF16;
+    const int act = act_code(n.attr_str("act", "none"));
+    const int64_t cnt = n.numel();
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { add_act(T[a], T[b], T[me], bf, cnt, act, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "sigmoid") {
+    nargs(1, 0);
+    need_dtype(n, argn(0).dtype, n.dtype, "input");
+    const int a = n.arg_nodes[0], bf = n.dtype == kBF16;
+    const int64_t cnt = n.numel();
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { sigmoid_ew(T[a], T[me], bf, cnt, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "maxpool") {
+    nargs(1, 0);
+    const Node& x = argn(0);
+    need_dtype(n, x.dtype, n.dtype, "input");
+    const int a = n.arg_nodes[0], bf = n.dtype == kBF16;
+    const int N = (int)x.shape[0], H = (int)x.shape[1], W = (int)x.shape[2], C = (int)x.shape[3];
+    const int k = (int)n.attr_int("k", 3), s = (int)n.attr_int("stride", 2), p = (int)n.attr_int("pad", 1);
+    const int Ho = (H + 2 * p - k) / s + 1, Wo = (W + 2 * p - k) / s + 1;
+    if (n.shape != std::vector<int64_t>{N, Ho, Wo, C}) fail(DUET_ESHAPE, "%" + n.name + ": maxpool output shape");
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { maxpool_nhwc(T[a], T[me], bf, N, H, W, C, k, s, p, Ho, Wo, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "avgpool") {
+    nargs(1, 0);
+    const Node& x = argn(0);
+    need_dtype(n, x.dtype, n.dtype, "input");
+    const int a = n.arg_nodes[0], bf = n.dtype == kBF16;
+    const int N = (int)x.shape[0], H = (int)x.shape[1], W = (int)x.shape[2], C = (int)x.shape[3];
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { avgpool_nhwc(T[a], T[me], bf, N, H, W, C, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "dot_join") {
+    nargs(2, 2);
+    need_dtype(n, argn(0).dtype, kF32, "wide logit");
+    need_dtype(n, n.dtype, kF32, "output");
+    const Node& a = argn(1);
+    const int s = n.arg_nodes[0], ai = n.arg_nodes[1], B = (int)a.shape[0], K = (int)a.shape[1];
+    const int ab = a.dtype == kBF16;
+    const float* w = (const float*)P.param(n.params[0]);
+    const float* b = (const float*)P.param(n.params[1]);
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      dot_join((const float*)T[s], T[ai], ab, w, b, (float*)T[me], B, K, st);
+    };
+    op.n_kernels = 1;
+  } else if (n.op == "cosine_join") {
+    nargs(2, 0);
+    need_dtype(n, argn(1).dtype, argn(0).dtype, "b");
+    need_dtype(n, n.dtype, kF32, "output");
+    const int a = n.arg_nodes[0], b = n.arg_nodes[1], B = (int)argn(0).shape[0], K = (int)argn(0).shape[1];
+    const int bf = argn(0).dtype == kBF16;
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { cosine_join(T[a], T[b], bf, (float*)T[me], B, K, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "concat_head") {
+    if (n.params.size() != 2 || n.arg_nodes.empty()) fail(DUET_EPARSE, "%" + n.name + ": concat_head(%a..., @w, @b)");
+    need_dtype(n, n.dtype, kF32, "output");
+    std::vector<int> ins, Ks, bfs;
+    int64_t tot = 0;
+    for (size_t i = 0; i < n.arg_nodes.size(); ++i) {
+      ins.push_back(n.arg_nodes[i]);
+      Ks.push_back((int)argn(i).shape[1]);
+      bfs.push_back(argn(i).dtype == kBF16);
+      tot += Ks.back();
+    }
+    if (pdecl(0).numel() != tot) fail(DUET_ESHAPE, "%" + n.name + ": head weight length != concat width");
+    const int B = (int)n.shape[0], act = act_code(n.attr_str("act", "sigmoid"));
+    const float* w = (const float*)P.param(n.params[0]);
+    const float* b = (const float*)P.param(n.params[1]);
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      std::vector<const void*> parts;
+      for (int i : ins) parts.push_back(T[i]);
+      concat_head(parts.data(), Ks.data(), bfs.data(), (int)ins.size(), w, b, (float*)T[me], B, act, st);
+    };
+    op.n_kernels = 1;
+  } else if (n.op == "sum_join" || n.op == "mean_join") {
+    if (!n.params.empty() || n.arg_nodes.empty()) fail(DUET_EPARSE, "%" + n.name + ": logit join arguments");
+    need_dtype(n, n.dtype, kF32, "output");
+    std::vector<int> ins(n.arg_nodes.begin(), n.arg_nodes.end());
+    for (size_t i = 0; i < ins.size(); ++i) need_dtype(n, argn(i).dtype, kF32, "branch logit");
+    const int B = (int)n.shape[0], mean = n.op == "mean_join";
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      std::vector<const float*> parts;
+      for (int i : ins) parts.push_back((const float*)T[i]);
+      logit_join(parts.data(), (int)parts.size(), (float*)T[me], B, mean, st);
+    };
+    op.n_kernels = 1;
+  } else {
+    fail(DUET_EUNSUPPORTED, "%" + n.name + ": no kernel for operator '" + n.op + "'");
+  }
+}
+
+std::shared_ptr<Program> ensure_program(Graph* g) {
+  if (g->prog) return g->prog;
+  for (auto& name : g->param_order)
+    if (!g->bound.count(name)) fail(DUET_EUNBOUND, "parameter @" + name + " is not bound");
+  int dev = 0;
+  if (!g->bound.empty())
+    dev = g->bound.begin()->second.device;
+  else
+    CK(cudaGetDevice(&dev));
+  DeviceGuard dg(dev);
+  auto P = std::make_shared<Program>();
+  P->g = g;
+  P->device = dev;
+  P->buf.resize(g->nodes.size(), nullptr);
+  for (auto& n : g->nodes) P->buf[n.id] = P->alloc(n.nbytes());
+  P->ops.resize(g->nodes.size());
+  for (auto& n : g->nodes) build_op(*P, n, P->ops[n.id]);
+  CK(cudaDeviceSynchronize());
+  g->prog = P;
+  return P;
+}
+
+void launch_subgraph(const Program& P, const Partition& part, int s, const Ptrs& T, cudaStream_t st) {
+  for (int v : part.sg_nodes[s])
+    if (P.ops[v].launch) P.ops[v].launch(T, st);
+}
+
+int64_t tensor_numel(const duet_tensor& t) {
+  int64_t n = 1;
+  for (int i = 0; i < t.ndim; ++i) n *= t.shape[i];
+  return n;
+}
+
+void check_tensor(const Node& n, const duet_tensor& t, const char* what) {
+  if ((int)t.dtype != n.dtype)
+    fail(DUET_EDTYPE, std::string(what) + " %" + n.name + ": dtype " + dtype_name(t.dtype) + " != " + dtype_name(n.dtype));
+  if (t.ndim != (int)n.shape.size()) fail(DUET_ESHAPE, std::string(what) + " %" + n.name + ": rank mismatch");
+  for (int i = 0; i < t.ndim; ++i)
+    if (t.shape[i] != n.shape[i]) fail(DUET_ESHAPE, std::string(what) + " %" + n.name + ": shape mismatch");
+  if (!t.data && n.numel() > 0) fail(DUET_EINVAL, std::string(what) + " %" + n.name + ": NULL data");
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------------------
+// Executor
+// ------------------------------------------------------------------------------------------------
+struct ExecEntry {
+  std::vector<void*> key;
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  std::vector<cudaEvent_t> events;
+};
+
+struct ExecCache {
+  int device = 0;
+  std::vector<ExecEntry> entries;
+  int64_t launches = 0;
+  std::weak_ptr<Program> prog;
+  ~ExecCache() {
+    int prev = 0;
+    cudaGetDevice(&prev);
+    cudaSetDevice(device);
+    for (auto& e : entries) {
+      if (e.exec) cudaGraphExecDestroy(e.exec);
+      if (e.graph) cudaGraphDestroy(e.graph);
+      for (auto ev : e.events) cudaEventDestroy(ev);
+    }
+    cudaSetDevice(prev);
+  }
+};
+
+void destroy_exec(ExecCache* e) { delete e; }
+
+static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<cudaStream_t>& streams,
+                         const Ptrs& T, int64_t* launches) {
+  const Partition& part = *S.p;
+  ExecEntry E;
+  cudaStream_t home = streams[0];
+  const int n = part.n_sg();
+  auto mk = [&]() {
+    cudaEvent_t ev;
+    CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    E.events.push_back(ev);
+    return ev;
+  };
+  std::vector<cudaEvent_t> done(n);
+  for (int s = 0; s < n; ++s) done[s] = mk();
+  cudaEvent_t fork = mk();
+  // subgraph-level predecessors
+  std::vector<std::vector<int>> preds(n);
+  for (auto& kv : part.edges)
+    if (kv.first.first >= 0 && kv.first.second >= 0) preds[kv.first.second].push_back(kv.first.first);
+  int64_t nk = 0;
+  CK(cudaStreamBeginCapture(home, cudaStreamCaptureModeRelaxed));
+  try {
+    CK(cudaEventRecord(fork, home));
+    std::vector<char> forked(streams.size(), 0);
+    std::vector<int> last_on(streams.size(), -1);
+    for (int s : S.order) {
+      const int d = S.slot_of[s];
+      cudaStream_t st = streams[d];
+      // slot index of the first slot that uses this stream handle (aliases share a queue)
+      int q = d;
+      for (int k = 0; k < (int)streams.size(); ++k)
+        if (streams[k] == st) {
+          q = k;
+          break;
+        }
+      if (st != home && !forked[q]) {
+        CK(cudaStreamWaitEvent(st, fork, 0));
+        forked[q] = 1;
+      }
+      for (int u : preds[s])
+        if (streams[S.slot_of[u]] != st) CK(cudaStreamWaitEvent(st, done[u], 0));
+      launch_subgraph(P, part, s, T, st);
+      for (int v : part.sg_nodes[s]) nk += P.ops[v].n_kernels;
+      CK(cudaEventRecord(done[s], st));
+      last_on[q] = s;
+    }
+    for (size_t q = 0; q < streams.size(); ++q)
+      if (last_on[q] >= 0 && streams[q] != home) CK(cudaStreamWaitEvent(home, done[last_on[q]], 0));
+  } catch (...) {
+    cudaGraph_t junk = nullptr;
+    cudaStreamEndCapture(home, &junk);
+    if (junk) cudaGraphDestroy(junk);
+    cudaGetLastError();
+    for (auto ev : E.events) cudaEventDestroy(ev);
+    throw;
+  }
+  CK(cudaStreamEndCapture(home, &E.graph));
+  CK(cudaGraphInstantiate(&E.exec, E.graph, 0));
+  *launches = nk;
+  return E;
+}
+
+void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_tensor* in, int n_in, duet_tensor* out,
+                  int n_out) {
+  const Graph* gc = S->p->g;
+  Graph* g = const_cast<Graph*>(gc);
+  auto P = ensure_program(g);
+  if (n_slots != S->pr->n_slots) fail(DUET_EINVAL, "n_slots differs from the profile's slot count");
+  std::vector<cudaStream_t> streams;
+  for (int d = 0; d < n_slots; ++d) {
+    if (slots[d].gpu != P->device)
+      fail(DUET_EUNSUPPORTED, "slot on another GPU: this build runs one GPU per process (multi-GPU = ranks)");
+    if (!slots[d].stream) fail(DUET_EINVAL, "slot stream is NULL (the legacy default stream cannot be captured)");
+    streams.push_back((cudaStream_t)slots[d].stream);
+  }
+  if (n_in != (int)g->input_nodes.size()) fail(DUET_EINVAL, "wrong number of inputs");
+  if (n_out != (int)g->outputs.size()) fail(DUET_EINVAL, "wrong number of outputs");
+  DeviceGuard dg(P->device);
+  cudaStream_t home = streams[0];
+  Ptrs T = P->buf;
+  for (int i = 0; i < n_in; ++i) {
+    const Node& nd = g->nodes[g->input_nodes[i]];
+    check_tensor(nd, in[i], "input");
+    if (in[i].device >= 0) {
+      if (in[i].device != P->device) fail(DUET_EUNSUPPORTED, "input on another GPU");
+      T[nd.id] = in[i].data;
+    } else {
+      CK(cudaMemcpyAsync(P->buf[nd.id], in[i].data, (size_t)nd.nbytes(), cudaMemcpyHostToDevice, home));
+    }
+  }
+  for (int i = 0; i < n_out; ++i) {
+    const Node& nd = g->nodes[g->outputs[i]];
+    check_tensor(nd, out[i], "output");
+    if (out[i].device >= 0) {
+      if (out[i].device != P->device) fail(DUET_EUNSUPPORTED, "output on another GPU");
+      T[nd.id] = out[i].data;
+    }
+  }
+  if (!S->exec || S->exec->prog.lock() != P) {
+    S->exec = std::make_shared<ExecCache>();
+    S->exec->device = P->device;
+    S->exec->prog = P;
+  }
+  std::vector<void*> key(T.begin(), T.end());
+  for (auto st : streams) key.push_back((void*)st);
+  ExecEntry* hit = nullptr;
+  for (auto& e : S->exec->entries)
+    if (e.key == key) hit = &e;
+  if (!hit) {
+    int64_t nk = 0;
+    ExecEntry E = capture(*P, *S, streams, T, &nk);
+    E.key = key;
+    S->exec->launches = nk;
+    if (S->exec->entries.size() >= 8) {
+      auto& old = S->exec->entries.front();
+      cudaGraphExecDestroy(old.exec);
+      cudaGraphDestroy(old.graph);
+      for (auto ev : old.events) cudaEventDestroy(ev);
+      S->exec->entries.erase(S->exec->entries.begin());
+    }
+    S->exec->entries.push_back(std::move(E));
+    hit = &S->exec->entries.back();
+  }
+  CK(cudaGraphLaunch(hit->exec, home));
+  for (int i = 0; i < n_out; ++i) {
+    const Node& nd = g->nodes[g->outputs[i]];
+    if (out[i].device < 0)
+      CK(cudaMemcpyAsync(out[i].data, P->buf[nd.id], (size_t)nd.nbytes(), cudaMemcpyDeviceToHost, home));
+  }
+}
+
+int64_t schedule_launch_count(const Schedule* s) {
+  if (!s->exec) fail(DUET_ESTATE, "launch count is known after the first duet_run");
+  return s->exec->launches;
+}
+
+void node_run(Graph* g, const std::string& name, const duet_tensor* args, int n_args, duet_tensor* out, void* stream) {
+  auto it = g->by_name.find(name);
+  if (it == g->by_name.end()) fail(DUET_EINVAL, "no node %" + name);
+  const Node& nd = g->nodes[it->second];
+  auto P = ensure_program(g);
+  if (n_args != (int)nd.arg_nodes.size()) fail(DUET_EINVAL, "node_run: wrong number of arguments");
+  DeviceGuard dg(P->device);
+  Ptrs T = P->buf;
+  for (int i = 0; i < n_args; ++i) {
+    const Node& a = g->nodes[nd.arg_nodes[i]];
+    check_tensor(a, args[i], "argument");
+    if (args[i].device != P->device) fail(DUET_EINVAL, "node_run: arguments must be device tensors on the graph's GPU");
+    T[a.id] = args[i].data;
+  }
+  check_tensor(nd, *out, "output");
+  if (out->device != P->device) fail(DUET_EINVAL, "node_run: output must be a device tensor");
+  T[nd.id] = out->data;
+  if (!P->ops[nd.id].launch) fail(DUET_EINVAL, "node %" + name + " has no kernel");
+  P->ops[nd.id].launch(T, (cudaStream_t)stream);
+}
+
+// ------------------------------------------------------------------------------------------------
+// Profiler
+// ------------------------------------------------------------------------------------------------
+namespace {
+
+__global__ void tiny_kernel(int* p) {
+  if (threadIdx.x == 0 && p) atomicAdd(p, 1);
+}
+
+// Synthetic but representative data in the input staging buffers: uniformly distributed ids so
+// gathers touch the whole table (zeros would hit one cached row), N(0,1)-scaled floats.
+void fill_inputs(const Program& P, cudaStream_t st) {
+  const Graph& g = *P.g;
+  for (int id : g.input_nodes) {
+    const Node& n = g.nodes[id];
+    int64_t high = 0;
+    for (auto& c : g.nodes)
+      for (size_t k = 0; k < c.arg_nodes.size(); ++k)
+        if (c.arg_nodes[k] == id && c.op == "embed_seq") high = g.params.at(c.params[0]).shape[0];
+    if (n.dtype == kI32 && high == 0) high = 1;
+    fill_random(P.buf[id], n.dtype, n.numel(), high, 0x5EED + id, st);
+  }
+}
+
+int64_t lower_median(std::vector<double> v) {
+  std::sort(v.begin(), v.end());
+  double m = v[(v.size() - 1) / 2];
+  return (int64_t)(m + 0.5);
+}
+
+}  // namespace
+
+Profile* profile_on_device(const Partition* p, const duet_slot* slots, int n_slots, const duet_profile_opts* o) {
+  Graph* g = const_cast<Graph*>(p->g);
+  auto P = ensure_program(g);
+  duet_profile_opts opts{20, 500, 20, 0};
+  if (o) opts = *o;
+  if (opts.samples < 1 || opts.reps_per_sample < 1 || opts.warmup < 0) fail(DUET_EINVAL, "bad profile options");
+  for (int d = 0; d < n_slots; ++d)
+    if (slots[d].gpu != P->device) fail(DUET_EUNSUPPORTED, "profiling slots on another GPU is not supported");
+  DeviceGuard dg(P->device);
+  cudaStream_t st;
+  CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+  std::unique_ptr<Profile> pr(new Profile());
+  pr->p = p;
+  pr->n_slots = n_slots;
+  for (int d = 0; d < n_slots; ++d) pr->slot_gpu.push_back(slots[d].gpu);
+  const int n = p->n_sg();
+  pr->t_ns.assign((size_t)n * n_slots, 0);
+  std::vector<cudaEvent_t> ev(opts.samples + 1);
+  try {
+    for (auto& e : ev) CK(cudaEventCreate(&e));
+    fill_inputs(*P, st);
+    // one serial pass so every intermediate buffer holds real data
+    for (int s = 0; s < n; ++s) launch_subgraph(*P, *p, s, P->buf, st);
+    CK(cudaStreamSynchronize(st));
+    for (int s = 0; s < n; ++s) {
+      cudaGraph_t gr;
+      cudaGraphExec_t ex;
+      CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed));
+      launch_subgraph(*P, *p, s, P->buf, st);
+      CK(cudaStreamEndCapture(st, &gr));
+      CK(cudaGraphInstantiate(&ex, gr, 0));
+      for (int w = 0; w < opts.warmup; ++w) CK(cudaGraphLaunch(ex, st));
+      CK(cudaEventRecord(ev[0], st));
+      for (int k = 0; k < opts.samples; ++k) {
+        for (int r = 0; r < opts.reps_per_sample; ++r) CK(cudaGraphLaunch(ex, st));
+        CK(cudaEventRecord(ev[k + 1], st));
+      }
+      CK(cudaStreamSynchronize(st));
+      std::vector<double> ns;
+      for (int k = 0; k < opts.samples; ++k) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, ev[k], ev[k + 1]));
+        ns.push_back(ms * 1e6 / opts.reps_per_sample);
+      }
+      int64_t t = lower_median(ns);
+      for (int d = 0; d < n_slots; ++d) pr->t_ns[(size_t)s * n_slots + d] = t;
+      cudaGraphExecDestroy(ex);
+      cudaGraphDestroy(gr);
+    }
+    if (opts.calibrate_comm && n_slots > 1) {
+      // alpha_same = extra latency of a cross-stream dependency inside a graph (Fig. 5)
+      cudaStream_t s2;
+      CK(cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking));
+      cudaEvent_t e1, e2;
+      CK(cudaEventCreateWithFlags(&e1, cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&e2, cudaEventDisableTiming));
+      auto time_graph = [&](bool cross) {
+        cudaGraph_t gr;
+        cudaGraphExec_t ex;
+        CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed));
+        for (int i = 0; i < 8; ++i) {
+          if (cross) {
+            CK(cudaEventRecord(e1, st));
+            CK(cudaStreamWaitEvent(s2, e1, 0));
+            tiny_kernel<<<1, 32, 0, s2>>>(nullptr);
+            CK(cudaEventRecord(e2, s2));
+            CK(cudaStreamWaitEvent(st, e2, 0));
+          } else {
+            tiny_kernel<<<1, 32, 0, st>>>(nullptr);
+          }
+          tiny_kernel<<<1, 32, 0, st>>>(nullptr);
+        }
+        CK(cudaStreamEndCapture(st, &gr));
+        CK(cudaGraphInstantiate(&ex, gr, 0));
+        for (int w = 0; w < 20; ++w) CK(cudaGraphLaunch(ex, st));
+        CK(cudaEventRecord(ev[0], st));
+        for (int k = 0; k < 200; ++k) CK(cudaGraphLaunch(ex, st));
+        CK(cudaEventRecord(ev[1], st));
+        CK(cudaStreamSynchronize(st));
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, ev[0], ev[1]));
+        cudaGraphExecDestroy(ex);
+        cudaGraphDestroy(gr);
+        return ms * 1e6 / 200.0 / 16.0;  // per dependency edge (2 edges per iteration)
+      };
+      double same = time_graph(false), cross = time_graph(true);
+      pr->comm.same_gpu.alpha_ns = std::max<int64_t>(0, (int64_t)((cross - same) + 0.5));
+      cudaEventDestroy(e1);
+      cudaEventDestroy(e2);
+      cudaStreamDestroy(s2);
+    }
+  } catch (...) {
+    for (auto e : ev)
+      if (e) cudaEventDestroy(e);
+    cudaStreamDestroy(st);
+    throw;
+  }
+  for (auto e : ev) cudaEventDestroy(e);
+  CK(cudaStreamDestroy(st));
+  return pr.release();
+}
+
+}  // namespace duet
