@@ -106,9 +106,13 @@ __global__ void __launch_bounds__(192, 1)
       for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % Cfg::STAGES;
         if (kb >= Cfg::STAGES) ptx::mbar_wait(&empty[s], ((kb / Cfg::STAGES) - 1) & 1);
-        ptx::mbar_arrive_expect_tx(&full[s], A_STAGE_BYTES + Cfg::B_STAGE_BYTES);
-        ptx::tma_load_2d(&tmA, &full[s], sA + s * A_STAGE_BYTES, kb * BK, m0);
-        ptx::tma_load_2d(&tmW, &full[s], sB + s * Cfg::B_STAGE_BYTES, kb * BK, n0);
+        if (ep.dbg & 2) {
+          ptx::mbar_arrive(&full[s]);
+        } else {
+          ptx::mbar_arrive_expect_tx(&full[s], A_STAGE_BYTES + Cfg::B_STAGE_BYTES);
+          ptx::tma_load_2d(&tmA, &full[s], sA + s * A_STAGE_BYTES, kb * BK, m0);
+          ptx::tma_load_2d(&tmW, &full[s], sB + s * Cfg::B_STAGE_BYTES, kb * BK, n0);
+        }
       }
     }
   } else if (warp == 1) {
@@ -122,6 +126,7 @@ __global__ void __launch_bounds__(192, 1)
         const uint32_t b_base = ptx::smem_u32(sB + s * Cfg::B_STAGE_BYTES);
 #pragma unroll
         for (int k = 0; k < BK / 16; ++k) {
+          if (ep.dbg & 1) break;
           ptx::umma_bf16(tmem, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
                          (kb | k) != 0);
         }
@@ -133,7 +138,12 @@ __global__ void __launch_bounds__(192, 1)
     // ---------------- epilogue warps 2..5 ----------------
     const int q = warp & 3;  // TMEM lane quarter this warp may access
     const int row = m0 + q * 32 + lane;
-    ptx::mbar_wait(tmem_full, 0);
+    if (ep.dbg & 4) {
+      const uint32_t a = ptx::smem_u32(tmem_full);
+      while (!ptx::mbar_try_wait(a, 0)) __nanosleep(256);
+    } else {
+      ptx::mbar_wait(tmem_full, 0);
+    }
     ptx::tc_fence_after();
     const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
     if constexpr (EPI == EPI_BIAS_ACT) {

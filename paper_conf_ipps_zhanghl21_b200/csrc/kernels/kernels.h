@@ -33,6 +33,7 @@ struct TcEpilogue {
   void* h_next = nullptr;      // [M, H] bf16
   const float* b_hn = nullptr; // GRU [H]
   int H = 0;
+  int dbg = 0;  // micro-benchmark switches: 1 = skip UMMA, 2 = skip TMA, 4 = epilogue backoff
 };
 
 // ---- tcgen05 GEMM (gemm_tc.cu) ----

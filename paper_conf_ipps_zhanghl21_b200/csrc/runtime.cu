@@ -197,7 +197,10 @@ void build_op(Program& P, const Node& n, Op& op) {
     const float* b = (const float*)P.param(n.params[1]);
     const int xb = x.dtype == kBF16, wb = w.dtype == kBF16, yb = n.dtype == kBF16;
     if (xb && wb && K % 8 == 0 && N >= 16) {
-      const int bn = tc_pick_bn(M, N, sms);
+      const char* dbg_env = getenv("DUET_GEMM_DBG");
+      const int dbg = dbg_env ? atoi(dbg_env) : 0;
+      const char* bn_env = getenv("DUET_GEMM_BN");
+      const int bn = bn_env ? atoi(bn_env) : tc_pick_bn(M, N, sms);
       CUtensorMap tw = make_tmap_bf16_2d(W, N, K, bn);
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         CUtensorMap ta = make_tmap_bf16_2d(T[in], M, K, 128);
@@ -206,6 +209,7 @@ void build_op(Program& P, const Node& n, Op& op) {
         ep.out = T[me];
         ep.ldo = N;
         ep.act = act;
+        ep.dbg = dbg;
         gemm_tc_maps(ta, tw, M, N, K, bn, ep, EPI_BIAS_ACT, yb, st);
       };
     } else {

@@ -1,0 +1,145 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the float64 oracle on the same seeded inputs.
+
+Bar (BASELINE.json:5): relative error <= 1e-5 (fp32) / 2e-2 (bf16 inputs, fp32
+accumulate); bit-exact for integer / byte work (hashing, gathers).  Sizes span several tiles with
+ragged tails; the full c2 size (the bench workload) is checked on sampled rows."""
+import numpy as np
+import pytest
+import torch
+
+from oracle import forward as OF
+from paper_conf_ipps_zhanghl21_b200 import duet
+from paper_conf_ipps_zhanghl21_b200 import workloads as W
+from paper_conf_ipps_zhanghl21_b200.harness import Session, materialize
+from tests.helpers import TOL, lazy_rows, oracle_arrays, rel_err, to_np
+
+pytestmark = pytest.mark.gpu
+
+FAST_PROFILE = dict(warmup=2, samples=5, reps=2)
+
+
+def _single_node_graph(op_line, params, inputs):
+    lines = [f"param @{k} : {dt}[{','.join(map(str, s))}]" for k, (dt, s) in params.items()]
+    lines += [f"%{k} = input() : {dt}[{','.join(map(str, s))}]" for k, (dt, s) in inputs.items()]
+    lines += [op_line, "output %y"]
+    return "\n".join(lines) + "\n"
+
+
+def _rand(shape, dt, scale=1.0, seed=0):
+    g = torch.Generator().manual_seed(seed)
+    t = (torch.rand(shape, generator=g, dtype=torch.float64) * 2 - 1) * scale
+    return t.to(torch.float32).to(torch.bfloat16 if dt == "bf16" else torch.float32)
+
+
+@pytest.mark.parametrize("M,N,K,dt,out", [
+    (128, 128, 64, "bf16", "bf16"),
+    (300, 136, 320, "bf16", "bf16"),
+    (2048, 1024, 1664, "bf16", "bf16"),
+    (77, 48, 72, "bf16", "f32"),
+    (513, 272, 200, "bf16", "f32"),
+    (300, 136, 320, "f32", "f32"),
+    (5, 3, 7, "f32", "f32"),
+])
+def test_linear_node(M, N, K, dt, out):
+    ir = _single_node_graph(f"%y = linear(%x, @W, @b) {{act=relu}} : {out}[{M},{N}]",
+                            {"W": (dt, (N, K)), "b": ("f32", (N,))}, {"x": (dt, (M, K))})
+    x = _rand((M, K), dt, 1.0, 1)
+    Wt = _rand((N, K), dt, 1.0 / np.sqrt(K), 2)
+    b = _rand((N,), "f32", 0.1, 3)
+    g = duet.Graph(ir)
+    g.bind_all({"W": Wt.cuda(), "b": b.cuda()})
+    y = torch.empty((M, N), dtype=torch.bfloat16 if out == "bf16" else torch.float32, device="cuda")
+    g.node_run("y", [x.cuda()], y)
+    torch.cuda.synchronize()
+    want = OF.linear(OF.to_f64(to_np(x), dt), OF.to_f64(to_np(Wt), dt), OF.to_f64(to_np(b), "f32"), "relu")
+    err = rel_err(y.float().cpu().numpy(), want)
+    assert err <= (TOL["f32"] if dt == "f32" else 1e-2), err
+
+
+def test_gathers_and_hash_bit_exact():
+    wl = W.build("c2", small=True)
+    params = materialize(wl.params, "cuda")
+    raw = wl.inputs["raw"].materialize("cuda")
+    g = duet.Graph(wl.ir)
+    g.bind_all(params)
+    B, F = raw.shape
+    ids = torch.empty((B, F), dtype=torch.int32, device="cuda")
+    g.node_run("ids", [raw], ids)
+    X = torch.empty((B, F * 64), dtype=torch.bfloat16, device="cuda")
+    g.node_run("deep_x", [ids], X)
+    wide = torch.empty((B, 1), dtype=torch.float32, device="cuda")
+    g.node_run("wide", [ids], wide)
+    torch.cuda.synchronize()
+    V = 1000
+    o_ids = OF.hash_mod(to_np(raw), V)
+    np.testing.assert_array_equal(ids.cpu().numpy(), o_ids)
+    E = to_np(params["deep_E"])
+    np.testing.assert_array_equal(to_np(X), E[np.arange(F)[None, :], o_ids].reshape(B, -1))
+    o_wide = OF.gather_sum(o_ids, to_np(params["wide_T"]), "bf16", to_np(params["wide_b"]).astype(np.float64))
+    assert rel_err(wide.cpu().numpy(), o_wide) < 1e-6
+
+
+def _oracle_outputs(wl, params, inputs):
+    return OF.run(wl.ir, oracle_arrays(params), oracle_arrays(inputs))
+
+
+CASES = [("c1", "f32"), ("c1", "bf16"), ("c2", "bf16"), ("c2", "f32"), ("c3", "bf16"), ("c3", "f32"),
+         ("c4", "bf16"), ("c4", "f32"), ("c5", "bf16")]
+
+
+@pytest.mark.parametrize("cfg,dt", CASES)
+def test_config_small_parity(cfg, dt):
+    wl = W.build(cfg, small=True, dt=dt)
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    want = _oracle_outputs(wl, sess.params, dict(zip(wl.inputs, inputs)))
+    results = {}
+    for mode in (duet.GREEDY_CORRECTION, duet.SERIAL):
+        outs = sess.outputs()
+        sess.run(sess.schedule(mode), inputs, outs)
+        torch.cuda.synchronize()
+        results[mode] = [o.float().cpu().numpy() for o in outs]
+        for (name, _, _), y in zip(wl.outputs, results[mode]):
+            err = rel_err(y, want[name])
+            print(f"[parity] {cfg} {dt} mode={mode} {name}: rel err {err:.3e}")
+            assert err <= TOL[dt], (cfg, dt, mode, err)
+    # same kernels, any placement -> bit-identical outputs
+    for a, b in zip(results[duet.GREEDY_CORRECTION], results[duet.SERIAL]):
+        np.testing.assert_array_equal(a, b)
+
+
+def test_host_buffers_e2e_equal_device():
+    wl = W.build("c2", small=True)
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    s = sess.schedule()
+    dev_out = sess.outputs()
+    sess.run(s, inputs, dev_out)
+    host_in = [t.cpu().pin_memory() for t in inputs]
+    host_out = sess.outputs(device=False)
+    sess.run(s, host_in, host_out)
+    sess.home.synchronize()
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(dev_out[0].cpu().numpy(), host_out[0].numpy())
+    assert s.launch_count() >= 6
+
+
+def test_c2_full_size_sampled():
+    """The bench workload (BASELINE.json:8 at full size) in the bench's launch configuration;
+    the oracle evaluates 96 sampled rows (rows are independent), reading only the table rows they
+    touch."""
+    wl = W.build("c2")
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    outs = sess.outputs()
+    sess.run(sess.schedule(), inputs, outs)
+    torch.cuda.synchronize()
+    rows = np.random.default_rng(0).choice(wl.batch, 96, replace=False)
+    rows[:2] = [0, wl.batch - 1]
+    oparams = {}
+    for k, spec in wl.params.items():
+        oparams[k] = lazy_rows(spec) if spec.numel > 10_000_000 else to_np(sess.params[k])
+    oin = {"raw": to_np(inputs[0])[rows]}
+    want = OF.run(wl.ir, oparams, oin)["y"]
+    got = outs[0].cpu().numpy()[rows]
+    assert rel_err(got, want) <= TOL["bf16"]
