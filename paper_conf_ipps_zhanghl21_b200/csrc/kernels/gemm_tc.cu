@@ -34,33 +34,8 @@ struct TileCfg {
   static constexpr int B_STAGE_BYTES = BN * BK * 2;
   static constexpr int STAGES = BN <= 64 ? 8 : (BN <= 128 ? 6 : 4);
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
-  static constexpr int SMEM = STAGES * (A_STAGE_BYTES + B_STAGE_BYTES) + 1024 + 256;
+  static constexpr int SMEM = STAGES * (A_STAGE_BYTES + B_STAGE_BYTES) + 1024 + 256 + BN * 4;
 };
-
-__device__ __forceinline__ void store16(float* dst, const float* v, int n_valid) {
-  if (n_valid >= 16 && ((uintptr_t)dst & 15) == 0) {
-    float4* d4 = reinterpret_cast<float4*>(dst);
-#pragma unroll
-    for (int i = 0; i < 4; ++i) d4[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-  } else {
-    for (int i = 0; i < 16 && i < n_valid; ++i) dst[i] = v[i];
-  }
-}
-__device__ __forceinline__ void store16(__nv_bfloat16* dst, const float* v, int n_valid) {
-  if (n_valid >= 16 && ((uintptr_t)dst & 15) == 0) {
-    uint32_t w[8];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      __nv_bfloat162 p = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
-      w[i] = *reinterpret_cast<uint32_t*>(&p);
-    }
-    uint4* d4 = reinterpret_cast<uint4*>(dst);
-    d4[0] = make_uint4(w[0], w[1], w[2], w[3]);
-    d4[1] = make_uint4(w[4], w[5], w[6], w[7]);
-  } else {
-    for (int i = 0; i < 16 && i < n_valid; ++i) dst[i] = __float2bfloat16_rn(v[i]);
-  }
-}
 
 template <int BN, int EPI, typename OutT>
 __global__ void __launch_bounds__(192, 1)
@@ -75,6 +50,7 @@ __global__ void __launch_bounds__(192, 1)
   uint64_t* empty = full + Cfg::STAGES;
   uint64_t* tmem_full = empty + Cfg::STAGES;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
+  float* s_bias = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(full) + 256);
 
   const int warp = ptx::warp_id();
   const int lane = threadIdx.x & 31;
@@ -138,6 +114,11 @@ __global__ void __launch_bounds__(192, 1)
     // ---------------- epilogue warps 2..5 ----------------
     const int q = warp & 3;  // TMEM lane quarter this warp may access
     const int row = m0 + q * 32 + lane;
+    if constexpr (EPI == EPI_BIAS_ACT) {
+      const int et = threadIdx.x - 64;
+      for (int c = et; c < BN; c += 128) s_bias[c] = (ep.bias && n0 + c < N) ? ep.bias[n0 + c] : 0.0f;
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+    }
     if (ep.dbg & 4) {
       const uint32_t a = ptx::smem_u32(tmem_full);
       while (!ptx::mbar_try_wait(a, 0)) __nanosleep(256);
@@ -147,20 +128,17 @@ __global__ void __launch_bounds__(192, 1)
     ptx::tc_fence_after();
     const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
     if constexpr (EPI == EPI_BIAS_ACT) {
-      OutT* out = reinterpret_cast<OutT*>(ep.out);
+      OutT* out = reinterpret_cast<OutT*>(ep.out) + (size_t)row * ep.ldo;
+      const int act = ep.act;
 #pragma unroll 1
       for (int c = 0; c < BN / 16; ++c) {
         float v[16];
         ptx::tmem_ld16(tq + c * 16, v);
         const int col0 = n0 + c * 16;
         if (row < M && col0 < N) {
-          const int nv = min(16, N - col0);
 #pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            float b = (ep.bias && i < nv) ? __ldg(ep.bias + col0 + i) : 0.0f;
-            v[i] = apply_act(v[i] + b, ep.act);
-          }
-          store16(out + (size_t)row * ep.ldo + col0, v, nv);
+          for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i] + s_bias[c * 16 + i], act);
+          store_row16_any(out + col0, v, N - col0);
         }
       }
     } else {
@@ -205,7 +183,7 @@ __global__ void __launch_bounds__(192, 1)
           }
         }
         __nv_bfloat16* hn = reinterpret_cast<__nv_bfloat16*>(ep.h_next) + (size_t)row * H + unit0 + jc;
-        store16(hn, h, nv);
+        store_row16_any(hn, h, nv);
       }
     }
   }

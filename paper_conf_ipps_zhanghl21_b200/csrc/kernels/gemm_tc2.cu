@@ -1,0 +1,183 @@
+// CTA-pair tcgen05 GEMM (cta_group::2, UMMA 256 x BN x 16) for the MLP / projection GEMMs.
+//
+//   D[M, N] = act(A[M, K] * W[N, K]^T + bias)     A, W bf16 K-major; fp32 accumulate in TMEM
+//
+// A cluster of 2 CTAs (same TPC) computes one 256 x BN tile: CTA r loads rows [m0 + 128 r, +128) of
+// A and rows [n0 + r BN/2, +BN/2) of W into its own shared memory (TMA, SWIZZLE_128B); both CTAs'
+// copies complete on the LEADER's full barrier; the leader's single MMA thread issues
+// tcgen05.mma.cta_group::2, which reads A/B halves from both CTAs' shared memory and writes each
+// CTA's 128 accumulator rows into that CTA's TMEM; tcgen05.commit multicasts stage-free and
+// accumulator-ready to both CTAs.  Versus the single-CTA tile this halves the W bytes each SM
+// pulls from L2 per FLOP and doubles the work per MMA instruction.
+#include "../common.h"
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace duet {
+
+namespace {
+
+constexpr int BM2 = 128;  // rows per CTA (256 per pair)
+constexpr int BK2 = 64;
+constexpr int A2_BYTES = BM2 * BK2 * 2;
+
+template <int BN>
+struct Cfg2 {
+  static constexpr int BH = BN / 2;  // W rows per CTA
+  static constexpr int B_BYTES = BH * BK2 * 2;
+  static constexpr int STAGE = A2_BYTES + B_BYTES;
+  static constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
+  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr int SMEM = STAGES * STAGE + 1024 + 256 + BN * 4;
+};
+
+template <int BN, typename OutT>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
+    gemm2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
+                 const TcEpilogue ep, int M, int N, int K) {
+  using C = Cfg2<BN>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + C::STAGES * A2_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tmem_full = empty + C::STAGES;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
+  float* s_bias = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(full) + 256);
+
+  const int warp = ptx::warp_id();
+  const int lane = threadIdx.x & 31;
+  const uint32_t rank = ptx::cluster_ctarank();
+  const int tile_n = blockIdx.x >> 1;
+  const int n0 = tile_n * BN;
+  const int m0 = blockIdx.y * (2 * BM2) + (int)rank * BM2;  // this CTA's rows
+  const int nk = (K + BK2 - 1) / BK2;
+
+  if (warp == 0 && lane == 0) {
+    ptx::tma_prefetch(&tmA);
+    ptx::tma_prefetch(&tmW);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    ptx::mbar_init(tmem_full, 1);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) {
+    ptx::tmem_alloc_2sm(tmem_slot, C::TMEM_COLS);
+    ptx::tmem_relinquish_2sm();
+  }
+  ptx::tc_fence_before();
+  ptx::cluster_sync();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // full barriers live in the leader CTA; both CTAs' copies complete there
+      const uint32_t full_leader0 = ptx::mapa(ptx::smem_u32(&full[0]), 0);
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % C::STAGES;
+        if (kb >= C::STAGES) ptx::mbar_wait(&empty[s], ((kb / C::STAGES) - 1) & 1);
+        const uint32_t fb = full_leader0 + s * 8;
+        if (ep.dbg & 2) {
+          if (rank == 0) ptx::mbar_arrive(&full[s]);
+          continue;
+        }
+        if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
+        ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES, kb * BK2, m0);
+        ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES, kb * BK2, n0 + (int)rank * C::BH);
+      }
+    }
+  } else if (warp == 1) {
+    if (rank == 0 && lane == 0) {
+      constexpr uint32_t idesc = ptx::idesc_bf16(2 * BM2, BN);
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % C::STAGES;
+        ptx::mbar_wait(&full[s], (kb / C::STAGES) & 1);
+        ptx::tc_fence_after();
+        const uint32_t a_base = ptx::smem_u32(sA + s * A2_BYTES);
+        const uint32_t b_base = ptx::smem_u32(sB + s * C::B_BYTES);
+#pragma unroll
+        for (int k = 0; k < BK2 / 16; ++k)
+          if (!(ep.dbg & 1)) ptx::umma_bf16_2sm(tmem, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
+                             (kb | k) != 0);
+        ptx::umma_commit_2sm(&empty[s], 0x3);
+      }
+      ptx::umma_commit_2sm(tmem_full, 0x3);
+    }
+  } else {
+    // epilogue warps 2..5: stage this tile's bias in smem while the mainloop runs
+    const int et = threadIdx.x - 64;
+    for (int c = et; c < BN; c += 128) s_bias[c] = (ep.bias && n0 + c < N) ? ep.bias[n0 + c] : 0.0f;
+    asm volatile("bar.sync 1, 128;" ::: "memory");
+    const int q = warp & 3;
+    const int row = m0 + q * 32 + lane;
+    ptx::mbar_wait(tmem_full, 0);
+    ptx::tc_fence_after();
+    const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
+    OutT* out = reinterpret_cast<OutT*>(ep.out) + (size_t)row * ep.ldo;
+    const int act = ep.act;
+#pragma unroll 1
+    for (int c = 0; c < BN / 16; ++c) {
+      if (ep.dbg & 8) break;
+      float v[16];
+      ptx::tmem_ld16(tq + c * 16, v);
+      if (ep.dbg & 16) continue;
+      const int col0 = n0 + c * 16;
+      if (row < M && col0 < N) {
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i] + s_bias[c * 16 + i], act);
+        store_row16_any(out + col0, v, N - col0);
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  ptx::cluster_sync();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc_2sm(tmem, C::TMEM_COLS);
+  }
+}
+
+template <int BN, typename OutT>
+void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, int M, int N, int K, cudaStream_t st) {
+  using C = Cfg2<BN>;
+  auto kern = gemm2_kernel<BN, OutT>;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
+    attr = true;
+  }
+  dim3 grid(2 * ((N + BN - 1) / BN), (M + 2 * BM2 - 1) / (2 * BM2));
+  kern<<<grid, 192, C::SMEM, st>>>(a, w, ep, M, N, K);
+  CK(cudaGetLastError());
+}
+
+}  // namespace
+
+int tc2_pick_bn(int M, int N, int K, int sms) {
+  // Widest tile that still occupies ~80% of the SM pairs (measured on B200):
+  // wide tiles cut L2->SMEM traffic per FLOP, but idle SMs cost more when the grid is small.
+  (void)K;
+  const int tm = (M + 255) / 256;
+  const int pairs = sms / 2;
+  for (int bn : {256, 128, 64}) {
+    if (bn > N && bn > 64) continue;
+    if (tm * ((N + bn - 1) / bn) * 5 >= pairs * 4) return bn;
+  }
+  return 64;
+}
+
+void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
+                   int out_bf16, cudaStream_t st) {
+  switch (bn) {
+    case 64: return out_bf16 ? launch2<64, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<64, float>(ta, tw, ep, M, N, K, st);
+    case 128: return out_bf16 ? launch2<128, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<128, float>(ta, tw, ep, M, N, K, st);
+    case 256: return out_bf16 ? launch2<256, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<256, float>(ta, tw, ep, M, N, K, st);
+  }
+  fail(DUET_EUNSUPPORTED, "gemm_tc2: bn must be 64, 128 or 256");
+}
+
+}  // namespace duet

@@ -44,6 +44,11 @@ void gemm_tc(const void* A, const void* W, int M, int N, int K, int bn, const Tc
 void gemm_tc_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
                   int epi, int out_bf16, cudaStream_t st);
 
+// CTA-pair GEMM (gemm_tc2.cu): 256 x bn tiles, bn in {64,128,256}; W map box rows = bn / 2.
+int tc2_pick_bn(int M, int N, int K, int num_sms);
+void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
+                   int out_bf16, cudaStream_t st);
+
 // ---- SIMT fallbacks / small kernels (simt.cu) ----
 // Y[M,N] = act(X[M,K] W[N,K]^T + b) ; X/W dtype per flags; fp32 accumulate.
 void gemm_simt(const void* X, int x_bf16, const void* W, int w_bf16, const float* b, void* Y, int y_bf16, int M,

@@ -196,7 +196,25 @@ void build_op(Program& P, const Node& n, Op& op) {
     void* W = P.param(n.params[0]);
     const float* b = (const float*)P.param(n.params[1]);
     const int xb = x.dtype == kBF16, wb = w.dtype == kBF16, yb = n.dtype == kBF16;
-    if (xb && wb && K % 8 == 0 && N >= 16) {
+    const char* gemm_env = getenv("DUET_GEMM");  // 1 = force the single-CTA tile (comparisons)
+    const bool pair = !(gemm_env && atoi(gemm_env) == 1) && M > 128;
+    if (xb && wb && K % 8 == 0 && N >= 16 && pair) {
+      const char* bn_env = getenv("DUET_GEMM_BN");
+      const int bn = bn_env ? atoi(bn_env) : tc2_pick_bn(M, N, K, sms);
+      const char* dbg_env = getenv("DUET_GEMM_DBG");
+      const int dbg2 = dbg_env ? atoi(dbg_env) : 0;
+      CUtensorMap tw = make_tmap_bf16_2d(W, N, K, bn / 2);
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        CUtensorMap ta = make_tmap_bf16_2d(T[in], M, K, 128);
+        TcEpilogue ep;
+        ep.bias = b;
+        ep.out = T[me];
+        ep.ldo = N;
+        ep.act = act;
+        ep.dbg = dbg2;
+        gemm_tc2_maps(ta, tw, M, N, K, bn, ep, yb, st);
+      };
+    } else if (xb && wb && K % 8 == 0 && N >= 16) {
       const char* dbg_env = getenv("DUET_GEMM_DBG");
       const int dbg = dbg_env ? atoi(dbg_env) : 0;
       const char* bn_env = getenv("DUET_GEMM_BN");
@@ -315,8 +333,8 @@ void build_op(Program& P, const Node& n, Op& op) {
       permute_rows(Wih, Wih_r, d_map, Np, (int64_t)E * es, 0);
       permute_rows(Whh, Whh_r, d_map, Np, (int64_t)H * es, 0);
       CK(cudaDeviceSynchronize());
-      const int bn_in = tc_pick_bn(S * B, Np, sms);
-      CUtensorMap t_wih = make_tmap_bf16_2d(Wih_r, Np, E, bn_in);
+      const int bn_in = tc2_pick_bn(S * B, Np, E, sms);
+      CUtensorMap t_wih = make_tmap_bf16_2d(Wih_r, Np, E, bn_in / 2);
       CUtensorMap t_whh = make_tmap_bf16_2d(Whh_r, Np, H, bn);
       CUtensorMap t_h[2] = {make_tmap_bf16_2d(hb[0], B, H, 128), make_tmap_bf16_2d(hb[1], B, H, 128)};
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
@@ -328,7 +346,7 @@ void build_op(Program& P, const Node& n, Op& op) {
         ep.out = gx;
         ep.ldo = Np;
         ep.act = ACT_NONE;
-        gemm_tc_maps(tx, t_wih, S * B, Np, E, bn_in, ep, EPI_BIAS_ACT, 0, st);
+        gemm_tc2_maps(tx, t_wih, S * B, Np, E, bn_in, ep, 0, st);
         for (int t = 0; t < S; ++t) {
           TcEpilogue e2;
           e2.gx = gx + (size_t)t * B * Np;
@@ -760,14 +778,16 @@ Profile* profile_on_device(const Partition* p, const duet_slot* slots, int n_slo
     for (int s = 0; s < n; ++s) {
       cudaGraph_t gr;
       cudaGraphExec_t ex;
+      // R back-to-back copies of the subgraph inside ONE graph: a sample is one graph launch, so
+      // the per-launch overhead of cudaGraphLaunch is amortised over R subgraph executions.
       CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed));
-      launch_subgraph(*P, *p, s, P->buf, st);
+      for (int r = 0; r < opts.reps_per_sample; ++r) launch_subgraph(*P, *p, s, P->buf, st);
       CK(cudaStreamEndCapture(st, &gr));
       CK(cudaGraphInstantiate(&ex, gr, 0));
-      for (int w = 0; w < opts.warmup; ++w) CK(cudaGraphLaunch(ex, st));
+      for (int w = 0; w < std::max(1, opts.warmup / std::max(1, opts.reps_per_sample)) + 1; ++w) CK(cudaGraphLaunch(ex, st));
       CK(cudaEventRecord(ev[0], st));
       for (int k = 0; k < opts.samples; ++k) {
-        for (int r = 0; r < opts.reps_per_sample; ++r) CK(cudaGraphLaunch(ex, st));
+        CK(cudaGraphLaunch(ex, st));
         CK(cudaEventRecord(ev[k + 1], st));
       }
       CK(cudaStreamSynchronize(st));
