@@ -90,13 +90,14 @@ __global__ void __launch_bounds__(256) conv_simt_kernel(const void* __restrict__
 }
 
 __global__ void fold_bn_kernel(const void* W, int bf16, const float* g, const float* beta, const float* mean,
-                               const float* var, void* Wf, float* bias, int Co, int64_t per_co) {
-  int64_t total = (int64_t)Co * per_co;
+                               const float* var, void* Wf, float* bias, int Co, int64_t per_co, int64_t ldw) {
+  int64_t total = (int64_t)Co * ldw;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    int co = (int)(i / per_co);
+    int co = (int)(i / ldw);
+    int64_t k = i - (int64_t)co * ldw;
     float sc = g[co] / sqrtf(var[co] + 1e-5f);
-    stx(Wf, i, ldx(W, i, bf16) * sc, bf16);
-    if (i % per_co == 0) bias[co] = beta[co] - mean[co] * sc;
+    stx(Wf, i, k < per_co ? ldx(W, (int64_t)co * per_co + k, bf16) * sc : 0.0f, bf16);
+    if (k == 0) bias[co] = beta[co] - mean[co] * sc;
   }
 }
 
@@ -112,9 +113,9 @@ void conv_fwd(const void* x, const void* Wf, const float* bias, const void* resi
 }
 
 void fold_bn(const void* W, int bf16, const float* g, const float* beta, const float* mean, const float* var, void* Wf,
-             float* bias, int Co, int64_t per_co, cudaStream_t st) {
-  fold_bn_kernel<<<grid_for((int64_t)Co * per_co, 256), 256, 0, st>>>(W, bf16, g, beta, mean, var, Wf, bias, Co,
-                                                                     per_co);
+             float* bias, int Co, int64_t per_co, int64_t ldw, cudaStream_t st) {
+  fold_bn_kernel<<<grid_for((int64_t)Co * ldw, 256), 256, 0, st>>>(W, bf16, g, beta, mean, var, Wf, bias, Co,
+                                                                  per_co, ldw);
   CK(cudaGetLastError());
 }
 

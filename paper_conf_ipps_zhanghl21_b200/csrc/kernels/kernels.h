@@ -93,10 +93,15 @@ struct ConvShape {
 };
 // y = act(conv(x, Wf) + bias (+ residual)); Wf [Co, kh, kw, C] with BN folded; NHWC.
 void conv_fwd(const void* x, const void* Wf, const float* bias, const void* residual, void* y, int bf16,
-              const ConvShape& s, int act, cudaStream_t st);
-// Fold BN into conv weights/bias: Wf = W * g/sqrt(var+eps), bias = beta - mean*g/sqrt(var+eps)
+              const ConvShape& s, int act, cudaStream_t st);  // CUDA-core path, Wf rows dense
+// Fold BN into conv weights/bias: Wf = W * g/sqrt(var+eps), bias = beta - mean*g/sqrt(var+eps).
+// Wf rows are ldw >= per_co elements apart; the padding is zero-filled.
 void fold_bn(const void* W, int bf16, const float* g, const float* beta, const float* mean, const float* var,
-             void* Wf, float* bias, int Co, int64_t per_co, cudaStream_t st);
+             void* Wf, float* bias, int Co, int64_t per_co, int64_t ldw, cudaStream_t st);
+// tcgen05 implicit-GEMM conv (conv_tc.cu); tw = TMA map of Wf [Co, ldw] with box rows = bn.
+int conv_tc_pick_bn(const ConvShape& s, int num_sms);
+void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
+             const ConvShape& s, int K, int act, int bn, cudaStream_t st);
 
 int num_sms(int device);
 // blocks for a grid-stride kernel: enough for `work` items, capped at per_sm x SM count

@@ -34,6 +34,8 @@ struct Program {
   std::vector<void*> buf;                  // per node: library output buffer (inputs: staging)
   std::vector<Op> ops;                     // per node
   std::vector<void*> allocs;               // device memory to free
+  std::map<int, std::pair<int, int>> fuse_res;  // conv node -> (residual node, add node it writes)
+  std::set<int> fused_adds;
   ~Program() {
     int prev = 0;
     cudaGetDevice(&prev);
@@ -384,17 +386,40 @@ void build_op(Program& P, const Node& n, Op& op) {
     s.Ho = (s.H + 2 * s.pad - s.kh) / s.stride + 1;
     s.Wo = (s.W + 2 * s.pad - s.kw) / s.stride + 1;
     if (n.shape != std::vector<int64_t>{s.N, s.Ho, s.Wo, s.Co}) fail(DUET_ESHAPE, "%" + n.name + ": conv output shape");
-    const int bf = x.dtype == kBF16, act = act_code(n.attr_str("act", "none"));
+    const int bf = x.dtype == kBF16;
+    int act = act_code(n.attr_str("act", "none"));
     const int64_t per_co = (int64_t)s.kh * s.kw * s.C;
-    void* Wf = P.alloc((int64_t)s.Co * per_co * dtype_bytes(w.dtype));
+    const bool tc = bf && s.Co % 16 == 0;
+    const int64_t ldw = tc ? (per_co + 7) / 8 * 8 : per_co;
+    void* Wf = P.alloc((int64_t)s.Co * ldw * dtype_bytes(w.dtype));
     float* bias = (float*)P.alloc((int64_t)s.Co * 4);
     fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
-            (const float*)P.param(n.params[3]), (const float*)P.param(n.params[4]), Wf, bias, s.Co, per_co, 0);
+            (const float*)P.param(n.params[3]), (const float*)P.param(n.params[4]), Wf, bias, s.Co, per_co, ldw, 0);
     const int in = n.arg_nodes[0];
-    op.launch = [=](const Ptrs& T, cudaStream_t st) { conv_fwd(T[in], Wf, bias, nullptr, T[me], bf, s, act, st); };
+    // residual fusion (planned in ensure_program): write act(conv + bias + res) into the add's buffer
+    int res = -1, dst = me;
+    auto fz = P.fuse_res.find(me);
+    if (fz != P.fuse_res.end()) {
+      res = fz->second.first;
+      dst = fz->second.second;
+      act = act_code(g.nodes[dst].attr_str("act", "none"));
+    }
+    if (tc) {
+      const int bn = conv_tc_pick_bn(s, sms);
+      CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, bn);
+      const int K = (int)per_co;
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        conv_tc(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, K, act, bn, st);
+      };
+    } else {
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        conv_fwd(T[in], Wf, bias, res >= 0 ? T[res] : nullptr, T[dst], bf, s, act, st);
+      };
+    }
     op.n_kernels = 1;
   } else if (n.op == "add") {
     nargs(2, 0);
+    if (P.fused_adds.count(me)) return;  // computed by the fused conv epilogue
     need_dtype(n, argn(0).dtype, n.dtype, "a");
     need_dtype(n, argn(1).dtype, n.dtype, "b");
     if (argn(0).numel() != n.numel() || argn(1).numel() != n.numel()) fail(DUET_ESHAPE, "%" + n.name + ": add shapes");
@@ -488,6 +513,30 @@ void build_op(Program& P, const Node& n, Op& op) {
   }
 }
 
+// add(%a, %b){act} whose later operand (topological rank) is a conv2d_bn with act=none consumed
+// only by this add: the conv's epilogue adds the other operand and applies the add's activation,
+// writing the add's buffer (ResNet BasicBlock tail; no extra HBM round trip).
+void plan_residual_fusion(Program& P) {
+  const Graph& g = *P.g;
+  std::vector<int> rank(g.nodes.size());
+  for (size_t i = 0; i < g.topo.size(); ++i) rank[g.topo[i]] = (int)i;
+  std::vector<int> n_cons(g.nodes.size(), 0);
+  for (auto& n : g.nodes)
+    for (int u : n.inputs) n_cons[u]++;
+  std::set<int> outs(g.outputs.begin(), g.outputs.end());
+  for (auto& n : g.nodes) {
+    if (n.op != "add" || n.arg_nodes.size() != 2 || n.arg_nodes[0] == n.arg_nodes[1]) continue;
+    int a = n.arg_nodes[0], b = n.arg_nodes[1];
+    int late = rank[a] > rank[b] ? a : b, other = late == a ? b : a;
+    const Node& c = g.nodes[late];
+    if (c.op != "conv2d_bn" || c.attr_str("act", "none") != "none" || n_cons[late] != 1 || outs.count(late)) continue;
+    if (c.dtype != kBF16 || n.dtype != kBF16 || c.shape != n.shape || g.nodes[other].shape != n.shape) continue;
+    if (c.shape.size() != 4 || c.shape[3] % 16) continue;
+    P.fuse_res[late] = {other, n.id};
+    P.fused_adds.insert(n.id);
+  }
+}
+
 std::shared_ptr<Program> ensure_program(Graph* g) {
   if (g->prog) return g->prog;
   for (auto& name : g->param_order)
@@ -504,6 +553,7 @@ std::shared_ptr<Program> ensure_program(Graph* g) {
   P->buf.resize(g->nodes.size(), nullptr);
   for (auto& n : g->nodes) P->buf[n.id] = P->alloc(n.nbytes());
   P->ops.resize(g->nodes.size());
+  plan_residual_fusion(*P);
   for (auto& n : g->nodes) build_op(*P, n, P->ops[n.id]);
   CK(cudaDeviceSynchronize());
   g->prog = P;

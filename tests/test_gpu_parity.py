@@ -143,3 +143,34 @@ def test_c2_full_size_sampled():
     want = OF.run(wl.ir, oparams, oin)["y"]
     got = outs[0].cpu().numpy()[rows]
     assert rel_err(got, want) <= TOL["bf16"]
+
+
+@pytest.mark.parametrize("N,H,W,C,Co,k,stride,pad", [
+    (2, 23, 19, 3, 64, 7, 2, 3),      # stem: scalar im2col path (C % 64 != 0), K padded to 8
+    (3, 14, 14, 64, 64, 3, 1, 1),     # 3x3, vector path, ragged M tile
+    (2, 15, 13, 128, 256, 3, 2, 1),   # stride 2, Co = 256
+    (2, 9, 9, 64, 128, 1, 2, 0),      # 1x1 downsample
+])
+def test_conv_node(N, H, W, C, Co, k, stride, pad):
+    Ho, Wo = (H + 2 * pad - k) // stride + 1, (W + 2 * pad - k) // stride + 1
+    ir = _single_node_graph(
+        f"%y = conv2d_bn(%x, @W, @g, @b, @m, @v) {{stride={stride}, pad={pad}, act=relu}} : bf16[{N},{Ho},{Wo},{Co}]",
+        {"W": ("bf16", (Co, k, k, C)), "g": ("f32", (Co,)), "b": ("f32", (Co,)), "m": ("f32", (Co,)),
+         "v": ("f32", (Co,))}, {"x": ("bf16", (N, H, W, C))})
+    x = _rand((N, H, W, C), "bf16", 1.0, 5)
+    Wt = _rand((Co, k, k, C), "bf16", (2.0 / (k * k * C)) ** 0.5, 6)
+    g_ = (_rand((Co,), "f32", 0.5, 7) + 1.0)
+    b_ = _rand((Co,), "f32", 0.1, 8)
+    m_ = _rand((Co,), "f32", 0.1, 9)
+    v_ = (_rand((Co,), "f32", 0.5, 10) + 1.0)
+    g = duet.Graph(ir)
+    g.bind_all({"W": Wt.cuda(), "g": g_.cuda(), "b": b_.cuda(), "m": m_.cuda(), "v": v_.cuda()})
+    y = torch.empty((N, Ho, Wo, Co), dtype=torch.bfloat16, device="cuda")
+    g.node_run("y", [x.cuda()], y)
+    torch.cuda.synchronize()
+    f = lambda t, d: OF.to_f64(to_np(t), d)
+    want = OF.conv2d_bn(f(x, "bf16"), f(Wt, "bf16"), f(g_, "f32"), f(b_, "f32"), f(m_, "f32"), f(v_, "f32"),
+                        stride, pad, "relu")
+    err = rel_err(y.float().cpu().numpy(), want)
+    print(f"[parity] conv {N}x{H}x{W}x{C}->{Co} k{k}s{stride}: rel err {err:.3e}")
+    assert err <= TOL["bf16"], err
