@@ -101,7 +101,60 @@ __global__ void fold_bn_kernel(const void* W, int bf16, const float* g, const fl
   }
 }
 
+// one thread per output row m: decode (n, ho, wo) once, walk k = (r, q, c) with incremental
+// counters (no per-element division), write the row as 16-B stores
+__global__ void im2col_kernel(const __nv_bfloat16* __restrict__ x, __nv_bfloat16* __restrict__ cols, ConvShape s,
+                              int ldk) {
+  const int K = s.kh * s.kw * s.C;
+  const int M = s.N * s.Ho * s.Wo;
+  const uint16_t* xs = reinterpret_cast<const uint16_t*>(x);
+  for (int m = blockIdx.x * blockDim.x + threadIdx.x; m < M; m += gridDim.x * blockDim.x) {
+    const int wo = m % s.Wo;
+    const int q0 = m / s.Wo;
+    const int ho = q0 % s.Ho;
+    const int n = q0 / s.Ho;
+    const int hb = ho * s.stride - s.pad, wb = wo * s.stride - s.pad;
+    uint4* dst = reinterpret_cast<uint4*>(cols + (int64_t)m * ldk);
+    int c = 0, q = 0, r = 0;
+    for (int k0 = 0; k0 < ldk; k0 += 8) {
+      uint32_t w[4];
+#pragma unroll
+      for (int e = 0; e < 8; e += 2) {
+        uint32_t pair = 0;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int k = k0 + e + h;
+          uint32_t v = 0;
+          if (k < K) {
+            const int hi = hb + r, wi = wb + q;
+            if ((unsigned)hi < (unsigned)s.H && (unsigned)wi < (unsigned)s.W)
+              v = xs[(((int64_t)n * s.H + hi) * s.W + wi) * s.C + c];
+            if (++c == s.C) {
+              c = 0;
+              if (++q == s.kw) {
+                q = 0;
+                ++r;
+              }
+            }
+          }
+          pair |= v << (16 * h);
+        }
+        w[e / 2] = pair;
+      }
+      dst[k0 / 8] = make_uint4(w[0], w[1], w[2], w[3]);
+    }
+  }
+}
+
 }  // namespace
+
+void im2col(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStream_t st) {
+  const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
+  if (!M) return;
+  if (M >= INT32_MAX || ldk % 8) fail(DUET_EUNSUPPORTED, "im2col: M < 2^31 and ldk % 8 == 0 required");
+  im2col_kernel<<<grid_for(M, 128, 16), 128, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)cols, s, (int)ldk);
+  CK(cudaGetLastError());
+}
 
 void conv_fwd(const void* x, const void* Wf, const float* bias, const void* residual, void* y, int bf16,
               const ConvShape& s, int act, cudaStream_t st) {

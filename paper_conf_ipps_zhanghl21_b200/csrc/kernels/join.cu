@@ -145,6 +145,40 @@ __global__ void avgpool_kernel(const T* x, T* y, int N, int HW, int C) {
 
 int warp_rows_grid(int B) { return (B + 7) / 8; }
 
+// NHWC bf16 maxpool, 8 channels (16 B) per thread, 32-bit index math (C % 8 == 0)
+__global__ void maxpool8_kernel(const uint4* __restrict__ x, uint4* __restrict__ y, int N, int H, int W, int C8, int k,
+                                int s, int p, int Ho, int Wo) {
+  const int total = N * Ho * Wo * C8;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += gridDim.x * blockDim.x) {
+    int c8 = i % C8;
+    int t = i / C8;
+    int wo = t % Wo;
+    t /= Wo;
+    int ho = t % Ho;
+    int n = t / Ho;
+    float m[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) m[e] = -INFINITY;
+    for (int r = 0; r < k; ++r) {
+      int hi = ho * s - p + r;
+      if (hi < 0 || hi >= H) continue;
+      for (int q = 0; q < k; ++q) {
+        int wi = wo * s - p + q;
+        if (wi < 0 || wi >= W) continue;
+        uint4 v = __ldg(x + ((n * H + hi) * W + wi) * C8 + c8);
+        const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(&v);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) m[e] = fmaxf(m[e], __bfloat162float(b[e]));
+      }
+    }
+    uint4 o;
+    __nv_bfloat16* ob = reinterpret_cast<__nv_bfloat16*>(&o);
+#pragma unroll
+    for (int e = 0; e < 8; ++e) ob[e] = __float2bfloat16_rn(m[e]);
+    y[i] = o;
+  }
+}
+
 }  // namespace
 
 void reduce_sum(const void* x, int x_bf16, const float* b, float* y, int B, int K, cudaStream_t st) {
@@ -214,6 +248,13 @@ void maxpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, 
                   cudaStream_t st) {
   int64_t total = (int64_t)N * Ho * Wo * C;
   if (!total) return;
+  if (bf16 && C % 8 == 0 && total / 8 < INT32_MAX && (int64_t)N * H * W * C / 8 < INT32_MAX &&
+      ((uintptr_t)x % 16) == 0 && ((uintptr_t)y % 16) == 0) {
+    maxpool8_kernel<<<grid_for(total / 8, 256, 16), 256, 0, st>>>((const uint4*)x, (uint4*)y, N, H, W, C / 8, k, s, p,
+                                                                  Ho, Wo);
+    CK(cudaGetLastError());
+    return;
+  }
   if (bf16)
     maxpool_kernel<__nv_bfloat16><<<grid_for(total, 256), 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, N,
                                                                        H, W, C, k, s, p, Ho, Wo);

@@ -102,6 +102,10 @@ void fold_bn(const void* W, int bf16, const float* g, const float* beta, const f
 int conv_tc_pick_bn(const ConvShape& s, int num_sms);
 void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
              const ConvShape& s, int K, int act, int bn, cudaStream_t st);
+bool conv_tma_ok(const ConvShape& s);
+// Explicit im2col (layers with C % 64 != 0): cols[m, k] = x[n, ho*s-p+r, wo*s-p+q, c], k = (r, q, c),
+// rows padded to ldk (zeros), bf16.
+void im2col(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStream_t st);
 
 int num_sms(int device);
 // blocks for a grid-stride kernel: enough for `work` items, capped at per_sm x SM count

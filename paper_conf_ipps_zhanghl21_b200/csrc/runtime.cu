@@ -389,12 +389,6 @@ void build_op(Program& P, const Node& n, Op& op) {
     const int bf = x.dtype == kBF16;
     int act = act_code(n.attr_str("act", "none"));
     const int64_t per_co = (int64_t)s.kh * s.kw * s.C;
-    const bool tc = bf && s.Co % 16 == 0;
-    const int64_t ldw = tc ? (per_co + 7) / 8 * 8 : per_co;
-    void* Wf = P.alloc((int64_t)s.Co * ldw * dtype_bytes(w.dtype));
-    float* bias = (float*)P.alloc((int64_t)s.Co * 4);
-    fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
-            (const float*)P.param(n.params[3]), (const float*)P.param(n.params[4]), Wf, bias, s.Co, per_co, ldw, 0);
     const int in = n.arg_nodes[0];
     // residual fusion (planned in ensure_program): write act(conv + bias + res) into the add's buffer
     int res = -1, dst = me;
@@ -404,19 +398,45 @@ void build_op(Program& P, const Node& n, Op& op) {
       dst = fz->second.second;
       act = act_code(g.nodes[dst].attr_str("act", "none"));
     }
-    if (tc) {
+    // bf16 paths: C % 64 == 0 -> persistent TMA-im2col implicit GEMM; otherwise (the 3-channel
+    // stem) explicit im2col [M, ldk] + the CTA-pair GEMM with the folded BN as its bias.
+    const bool tma = bf && s.Co % 16 == 0 && conv_tma_ok(s);
+    const bool cols = bf && !tma && s.Co >= 16 && s.Co % 8 == 0 && res < 0;
+    const int64_t ldw = (tma || cols) ? (per_co + 7) / 8 * 8 : per_co;
+    void* Wf = P.alloc((int64_t)s.Co * ldw * dtype_bytes(w.dtype));
+    float* bias = (float*)P.alloc((int64_t)s.Co * 4);
+    fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
+            (const float*)P.param(n.params[3]), (const float*)P.param(n.params[4]), Wf, bias, s.Co, per_co, ldw, 0);
+    if (tma) {
       const int bn = conv_tc_pick_bn(s, sms);
       CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, bn);
       const int K = (int)per_co;
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         conv_tc(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, K, act, bn, st);
       };
+      op.n_kernels = 1;
+    } else if (cols) {
+      const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
+      void* colbuf = P.alloc(M * ldw * 2);
+      const int bn = tc2_pick_bn((int)M, s.Co, (int)ldw, sms);
+      CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, bn / 2);
+      CUtensorMap ta = make_tmap_bf16_2d(colbuf, M, ldw, 128);
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        im2col(T[in], colbuf, s, ldw, st);
+        TcEpilogue ep;
+        ep.bias = bias;
+        ep.out = T[dst];
+        ep.ldo = s.Co;
+        ep.act = act;
+        gemm_tc2_maps(ta, tw, (int)M, s.Co, (int)ldw, bn, ep, 1, st);
+      };
+      op.n_kernels = 2;
     } else {
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         conv_fwd(T[in], Wf, bias, res >= 0 ? T[res] : nullptr, T[dst], bf, s, act, st);
       };
+      op.n_kernels = 1;
     }
-    op.n_kernels = 1;
   } else if (n.op == "add") {
     nargs(2, 0);
     if (P.fused_adds.count(me)) return;  // computed by the fused conv epilogue
@@ -669,7 +689,9 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
     throw;
   }
   CK(cudaStreamEndCapture(home, &E.graph));
-  CK(cudaGraphInstantiate(&E.exec, E.graph, 0));
+  // per-node priorities: kernels captured from a higher-priority slot stream keep it inside the
+  // graph, so a latency-bound branch gets SMs first when a co-running branch's CTAs retire
+  CK(cudaGraphInstantiate(&E.exec, E.graph, cudaGraphInstantiateFlagUseNodePriority));
   *launches = nk;
   return E;
 }

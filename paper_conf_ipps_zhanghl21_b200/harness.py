@@ -23,7 +23,11 @@ class Session:
         self.graph = duet.Graph(wl.ir)
         self.graph.bind_all(self.params)
         self.part = self.graph.partition(granularity)
-        self.streams = [torch.cuda.Stream(device=device) for _ in range(n_slots)]
+        # slot 0 (home: inputs, outputs, the critical path after Step 1) at normal priority; the other
+        # slots at high priority so their (typically latency-bound) kernels are not starved by a
+        # co-running throughput branch
+        lo, hi = torch.cuda.Stream.priority_range() if hasattr(torch.cuda.Stream, "priority_range") else (0, -1)
+        self.streams = [torch.cuda.Stream(device=device, priority=0 if i == 0 else -1) for i in range(n_slots)]
         self.slots = [(device, s) for s in self.streams]
         if table is not None:
             self.prof = self.part.profile_from_table([device] * n_slots, table, comm or ((0, 0), (0, 0)))
