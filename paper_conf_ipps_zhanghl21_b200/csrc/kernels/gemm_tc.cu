@@ -153,33 +153,82 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll
         for (int g = 0; g < G; ++g) ptx::tmem_ld16(tq + g * U + jc, acc[g]);
         if (row >= M) continue;
-        const float* gx = ep.gx + (size_t)row * N + (size_t)blockIdx.x * BN + jc;
-        float h[16];
         const int nv = min(16, H - (unit0 + jc));
         if (nv <= 0) continue;
+        const float* gx = ep.gx + (size_t)row * N + (size_t)blockIdx.x * BN + jc;
+        float h[16];
+        // all loads first (16-B vectors), then the cell math: no dependent global loads in the loop
+        float gxv[G][16];
+#pragma unroll
+        for (int g = 0; g < G; ++g)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const float4 t = __ldg(reinterpret_cast<const float4*>(gx + g * U) + i);
+            gxv[g][4 * i] = t.x;
+            gxv[g][4 * i + 1] = t.y;
+            gxv[g][4 * i + 2] = t.z;
+            gxv[g][4 * i + 3] = t.w;
+          }
         if constexpr (EPI == EPI_LSTM) {
           float* cst = ep.c_state + (size_t)row * H + unit0 + jc;
+          float cv[16];
+          if (nv == 16) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+              const float4 t = reinterpret_cast<const float4*>(cst)[i];
+              cv[4 * i] = t.x;
+              cv[4 * i + 1] = t.y;
+              cv[4 * i + 2] = t.z;
+              cv[4 * i + 3] = t.w;
+            }
+          } else {
+#pragma unroll
+            for (int i = 0; i < 16; ++i) cv[i] = i < nv ? cst[i] : 0.0f;
+          }
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
-            if (i >= nv) break;
-            float ig = sigmoidf_acc(acc[0][i] + gx[0 * U + i]);
-            float fg = sigmoidf_acc(acc[1][i] + gx[1 * U + i]);
-            float gg = tanhf(acc[2][i] + gx[2 * U + i]);
-            float og = sigmoidf_acc(acc[3][i] + gx[3 * U + i]);
-            float c = fg * cst[i] + ig * gg;
-            cst[i] = c;
-            h[i] = og * tanhf(c);
+            const float ig = sigmoidf_acc(acc[0][i] + gxv[0][i]);
+            const float fg = sigmoidf_acc(acc[1][i] + gxv[1][i]);
+            const float gg = tanhf(acc[2][i] + gxv[2][i]);
+            const float og = sigmoidf_acc(acc[3][i] + gxv[3][i]);
+            cv[i] = fg * cv[i] + ig * gg;
+            h[i] = og * tanhf(cv[i]);
+          }
+          if (nv == 16) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+              reinterpret_cast<float4*>(cst)[i] = make_float4(cv[4 * i], cv[4 * i + 1], cv[4 * i + 2], cv[4 * i + 3]);
+          } else {
+#pragma unroll
+            for (int i = 0; i < 16; ++i)
+              if (i < nv) cst[i] = cv[i];
           }
         } else {
           const __nv_bfloat16* hp = reinterpret_cast<const __nv_bfloat16*>(ep.h_prev) + (size_t)row * H + unit0 + jc;
           const float* bhn = ep.b_hn + unit0 + jc;
+          float hpv[16], bv[16];
+          if (nv == 16) {
+            const uint4 p0 = *reinterpret_cast<const uint4*>(hp);
+            const uint4 p1 = *reinterpret_cast<const uint4*>(hp + 8);
+            const __nv_bfloat16* b0 = reinterpret_cast<const __nv_bfloat16*>(&p0);
+            const __nv_bfloat16* b1 = reinterpret_cast<const __nv_bfloat16*>(&p1);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              hpv[i] = __bfloat162float(b0[i]);
+              hpv[8 + i] = __bfloat162float(b1[i]);
+            }
+          } else {
+#pragma unroll
+            for (int i = 0; i < 16; ++i) hpv[i] = i < nv ? __bfloat162float(hp[i]) : 0.0f;
+          }
+#pragma unroll
+          for (int i = 0; i < 16; ++i) bv[i] = i < nv ? __ldg(bhn + i) : 0.0f;
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
-            if (i >= nv) break;
-            float r = sigmoidf_acc(acc[0][i] + gx[0 * U + i]);
-            float z = sigmoidf_acc(acc[1][i] + gx[1 * U + i]);
-            float n = tanhf(gx[2 * U + i] + r * (acc[2][i] + bhn[i]));
-            h[i] = (1.0f - z) * n + z * __bfloat162float(hp[i]);
+            const float r = sigmoidf_acc(acc[0][i] + gxv[0][i]);
+            const float z = sigmoidf_acc(acc[1][i] + gxv[1][i]);
+            const float n = tanhf(gxv[2][i] + r * (acc[2][i] + bv[i]));
+            h[i] = (1.0f - z) * n + z * hpv[i];
           }
         }
         __nv_bfloat16* hn = reinterpret_cast<__nv_bfloat16*>(ep.h_next) + (size_t)row * H + unit0 + jc;
