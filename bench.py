@@ -245,18 +245,15 @@ def main():
     if args.impl == "reference":
         return reference_arm(args)
     import torch
-    import torch.distributed as dist
 
     from paper_conf_ipps_zhanghl21_b200 import duet
+    from paper_conf_ipps_zhanghl21_b200 import multirank as MR
     from paper_conf_ipps_zhanghl21_b200 import workloads as W
     from paper_conf_ipps_zhanghl21_b200.harness import Session, materialize
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    rank, world, local = MR.env()
     torch.cuda.set_device(local)
+    MR.init("nccl", torch.device(f"cuda:{local}"))
     dev = f"cuda:{local}"
 
     wl = W.build(args.config, dt=args.dtype)
@@ -279,19 +276,14 @@ def main():
     t_serial = time_steps(torch, step_serial, home, args.steps, args.warmup, flush)
 
     # --- timed region (DUET) ---
-    if world > 1:
-        dist.barrier()
+    MR.barrier()
     torch.cuda.synchronize()
     finish_clocks, _, clk_err = clock_sampler(local)
     t_duet = time_steps(torch, step_duet, home, args.steps, args.warmup, flush)
     clocks = finish_clocks() if finish_clocks else clk_err
     torch.cuda.synchronize()
-    total_ms = sum(t_duet)
-    if world > 1:
-        t = torch.tensor([total_ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
-        dist.barrier()
+    total_ms = MR.max_over_ranks(sum(t_duet))
+    MR.barrier()
 
     # --- end to end through the C ABI with pinned host buffers ---
     host_in = [t.cpu().pin_memory() for t in inputs]
@@ -301,14 +293,10 @@ def main():
         duet_s.run(sess.slots, host_in, host_out)
 
     t_e2e = time_steps(torch, step_e2e, home, args.steps, args.warmup, flush)
-    e2e_ms = sum(t_e2e)
-    if world > 1:
-        t = torch.tensor([e2e_ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_ms = float(t.item())
+    e2e_ms = MR.max_over_ranks(sum(t_e2e))
 
     if rank != 0:
-        dist.destroy_process_group()
+        MR.finalize()
         return
 
     n_launch = duet_s.launch_count()
@@ -379,8 +367,7 @@ def main():
         "clocks": clocks,
     }
     print(json.dumps(line), flush=True)
-    if world > 1:
-        dist.destroy_process_group()
+    MR.finalize()
 
 
 if __name__ == "__main__":
