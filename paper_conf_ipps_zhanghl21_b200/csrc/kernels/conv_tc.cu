@@ -94,6 +94,8 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
 
   if (warp == 0) {
     if (lane == 0) {
@@ -221,8 +223,7 @@ void launch_conv_tma(const CUtensorMap& tx, const CUtensorMap& tw, const ConvArg
   int dev = 0;
   cudaGetDevice(&dev);
   const int grid = (int)std::min<int64_t>(tiles, num_sms(dev));
-  kern<<<grid, 192, C::SMEM, st>>>(tx, tw, a);
-  CK(cudaGetLastError());
+  launch_pdl(kern, dim3(grid), dim3(192), C::SMEM, st, tx, tw, a);
 }
 
 

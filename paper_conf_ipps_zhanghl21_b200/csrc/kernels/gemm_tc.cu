@@ -8,11 +8,14 @@
 //   warps 2..5  epilogue: tcgen05.ld TMEM -> registers -> fused epilogue -> global
 // Epilogues:
 //   EPI_BIAS_ACT  out = act(acc + bias[n])                      (MLP / projections, A5-A6)
-//   EPI_LSTM      gates = gx + acc; c = f*c + i*g; h = o*tanh(c) (A7, PyTorch i,f,g,o)
-//   EPI_GRU       r,z = sig(gx + acc); n = tanh(gx_n + r*(acc_n + b_hn)); h = (1-z) n + z h (A8)
+//   EPI_LSTM      fused step: a = [x_t | h_{t-1}] [W_ih | W_hh]^T + b; c = f*c + i*g; h = o*tanh(c)
+//                 (A6+A7, PyTorch gate order i,f,g,o)
+//   EPI_GRU       fused step with 4 gate blocks r, z, n_x = W_in x + b_in, n_h = W_hn h + b_hn:
+//                 n = tanh(n_x + r*n_h); h = (1-z) n + z h (A6+A8)
 // For the RNN epilogues the weight rows are gate-block interleaved per tile: tile columns
-// [g*u, (g+1)*u) hold gate g of hidden units [tile*u, (tile+1)*u), u = BN / G, so one thread
-// owns every gate of its units.
+// [g*u, (g+1)*u) hold gate block g of hidden units [tile*u, (tile+1)*u), u = BN / 4, so one thread
+// owns every gate of its units, and the input projection is part of the K loop (no G_x buffer;
+// DESIGN.md "Data layout").
 #include <cudaTypedefs.h>
 
 #include <cstdio>
@@ -40,7 +43,7 @@ struct TileCfg {
 template <int BN, int EPI, typename OutT>
 __global__ void __launch_bounds__(192, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
-                   const TcEpilogue ep, int M, int N, int K) {
+                   const __grid_constant__ CUtensorMap tmX, const TcEpilogue ep, int M, int N, int K) {
   using Cfg = TileCfg<BN>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -61,6 +64,7 @@ __global__ void __launch_bounds__(192, 1)
   if (warp == 0 && lane == 0) {
     ptx::tma_prefetch(&tmA);
     ptx::tma_prefetch(&tmW);
+    if (ep.kx) ptx::tma_prefetch(&tmX);
     for (int s = 0; s < Cfg::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
@@ -76,6 +80,8 @@ __global__ void __launch_bounds__(192, 1)
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  ptx::pdl_wait();     // A / gx / c_state / h_prev come from the previous kernel in the stream
+  ptx::pdl_trigger();
 
   if (warp == 0) {
     if (lane == 0) {
@@ -86,7 +92,10 @@ __global__ void __launch_bounds__(192, 1)
           ptx::mbar_arrive(&full[s]);
         } else {
           ptx::mbar_arrive_expect_tx(&full[s], A_STAGE_BYTES + Cfg::B_STAGE_BYTES);
-          ptx::tma_load_2d(&tmA, &full[s], sA + s * A_STAGE_BYTES, kb * BK, m0);
+          if (kb < ep.kx)  // fused RNN step: x_t part of K
+            ptx::tma_load_2d(&tmX, &full[s], sA + s * A_STAGE_BYTES, kb * BK, ep.x_row0 + m0);
+          else
+            ptx::tma_load_2d(&tmA, &full[s], sA + s * A_STAGE_BYTES, (kb - ep.kx) * BK, m0);
           ptx::tma_load_2d(&tmW, &full[s], sB + s * Cfg::B_STAGE_BYTES, kb * BK, n0);
         }
       }
@@ -114,7 +123,7 @@ __global__ void __launch_bounds__(192, 1)
     // ---------------- epilogue warps 2..5 ----------------
     const int q = warp & 3;  // TMEM lane quarter this warp may access
     const int row = m0 + q * 32 + lane;
-    if constexpr (EPI == EPI_BIAS_ACT) {
+    {  // bias tile -> smem (both epilogue kinds)
       const int et = threadIdx.x - 64;
       for (int c = et; c < BN; c += 128) s_bias[c] = (ep.bias && n0 + c < N) ? ep.bias[n0 + c] : 0.0f;
       asm volatile("bar.sync 1, 128;" ::: "memory");
@@ -142,8 +151,8 @@ __global__ void __launch_bounds__(192, 1)
         }
       }
     } else {
-      // RNN cell epilogue; G gates per unit, u units per tile, gate block g at columns [g*u, (g+1)*u)
-      constexpr int G = (EPI == EPI_LSTM) ? 4 : 3;
+      // RNN cell epilogue; 4 gate blocks of U units per tile: block g at columns [g*U, (g+1)*U)
+      constexpr int G = 4;
       constexpr int U = BN / G;
       const int H = ep.H;
       const int unit0 = blockIdx.x * U;
@@ -155,20 +164,11 @@ __global__ void __launch_bounds__(192, 1)
         if (row >= M) continue;
         const int nv = min(16, H - (unit0 + jc));
         if (nv <= 0) continue;
-        const float* gx = ep.gx + (size_t)row * N + (size_t)blockIdx.x * BN + jc;
-        float h[16];
-        // all loads first (16-B vectors), then the cell math: no dependent global loads in the loop
-        float gxv[G][16];
 #pragma unroll
         for (int g = 0; g < G; ++g)
 #pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const float4 t = __ldg(reinterpret_cast<const float4*>(gx + g * U) + i);
-            gxv[g][4 * i] = t.x;
-            gxv[g][4 * i + 1] = t.y;
-            gxv[g][4 * i + 2] = t.z;
-            gxv[g][4 * i + 3] = t.w;
-          }
+          for (int i = 0; i < 16; ++i) acc[g][i] += s_bias[g * U + jc + i];
+        float h[16];
         if constexpr (EPI == EPI_LSTM) {
           float* cst = ep.c_state + (size_t)row * H + unit0 + jc;
           float cv[16];
@@ -187,10 +187,10 @@ __global__ void __launch_bounds__(192, 1)
           }
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
-            const float ig = sigmoidf_acc(acc[0][i] + gxv[0][i]);
-            const float fg = sigmoidf_acc(acc[1][i] + gxv[1][i]);
-            const float gg = tanhf(acc[2][i] + gxv[2][i]);
-            const float og = sigmoidf_acc(acc[3][i] + gxv[3][i]);
+            const float ig = sigmoidf_acc(acc[0][i]);
+            const float fg = sigmoidf_acc(acc[1][i]);
+            const float gg = tanhf(acc[2][i]);
+            const float og = sigmoidf_acc(acc[3][i]);
             cv[i] = fg * cv[i] + ig * gg;
             h[i] = og * tanhf(cv[i]);
           }
@@ -205,8 +205,7 @@ __global__ void __launch_bounds__(192, 1)
           }
         } else {
           const __nv_bfloat16* hp = reinterpret_cast<const __nv_bfloat16*>(ep.h_prev) + (size_t)row * H + unit0 + jc;
-          const float* bhn = ep.b_hn + unit0 + jc;
-          float hpv[16], bv[16];
+          float hpv[16];
           if (nv == 16) {
             const uint4 p0 = *reinterpret_cast<const uint4*>(hp);
             const uint4 p1 = *reinterpret_cast<const uint4*>(hp + 8);
@@ -222,12 +221,10 @@ __global__ void __launch_bounds__(192, 1)
             for (int i = 0; i < 16; ++i) hpv[i] = i < nv ? __bfloat162float(hp[i]) : 0.0f;
           }
 #pragma unroll
-          for (int i = 0; i < 16; ++i) bv[i] = i < nv ? __ldg(bhn + i) : 0.0f;
-#pragma unroll
           for (int i = 0; i < 16; ++i) {
-            const float r = sigmoidf_acc(acc[0][i] + gxv[0][i]);
-            const float z = sigmoidf_acc(acc[1][i] + gxv[1][i]);
-            const float n = tanhf(gxv[2][i] + r * (acc[2][i] + bv[i]));
+            const float r = sigmoidf_acc(acc[0][i]);
+            const float z = sigmoidf_acc(acc[1][i]);
+            const float n = tanhf(acc[2][i] + r * acc[3][i]);  // (W_in x + b_in) + r * (W_hn h + b_hn)
             h[i] = (1.0f - z) * n + z * hpv[i];
           }
         }
@@ -258,8 +255,8 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 }
 
 template <int BN, int EPI, typename OutT>
-void launch_tc(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, int M, int N, int K,
-               cudaStream_t st) {
+void launch_tc(const CUtensorMap& a, const CUtensorMap& w, const CUtensorMap& x, const TcEpilogue& ep, int M, int N,
+               int K, cudaStream_t st) {
   using Cfg = TileCfg<BN>;
   auto kern = gemm_tc_kernel<BN, EPI, OutT>;
   static bool attr_done = false;  // per instantiation; device attribute applies process-wide
@@ -268,11 +265,56 @@ void launch_tc(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep,
     attr_done = true;
   }
   dim3 grid((N + BN - 1) / BN, (M + BM - 1) / BM);
-  kern<<<grid, 192, Cfg::SMEM, st>>>(a, w, ep, M, N, K);
-  CK(cudaGetLastError());
+  launch_pdl(kern, grid, dim3(192), Cfg::SMEM, st, a, w, x, ep, M, N, K);
+}
+
+// Fused recurrent weights: row r' = tile*BN + g*U + j' <-> (gate block g, unit j = tile*U + j');
+// columns [0, E) from W_ih, [E, Ep) zero, [Ep, Ep+H) from W_hh.  LSTM blocks i,f,g,o take PyTorch
+// gate g of both matrices; GRU blocks r, z take gate 0/1 of both, n_x = (W_in | 0), n_h = (0 | W_hn).
+__global__ void rnn_pack_kernel(int kind, const __nv_bfloat16* __restrict__ Wih, const __nv_bfloat16* __restrict__ Whh,
+                                const float* __restrict__ bih, const float* __restrict__ bhh,
+                                __nv_bfloat16* __restrict__ Wcat, float* __restrict__ bias, int E, int Ep, int H,
+                                int U, int BN, int64_t rows) {
+  const int Kc = Ep + H;
+  const int64_t total = rows * Kc;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / Kc;
+    const int k = (int)(i - r * Kc);
+    const int tile = (int)(r / BN), rem = (int)(r % BN), g = rem / U, j = tile * U + rem % U;
+    float v = 0.0f;
+    if (j < H) {
+      const int src_gate = (kind == 2 && g == 3) ? 2 : g;  // GRU n_h uses PyTorch gate n (index 2)
+      const bool use_x = !(kind == 2 && g == 3);
+      const bool use_h = !(kind == 2 && g == 2);
+      if (k < E) {
+        if (use_x) v = __bfloat162float(Wih[((int64_t)src_gate * H + j) * E + k]);
+      } else if (k >= Ep) {
+        if (use_h) v = __bfloat162float(Whh[((int64_t)src_gate * H + j) * H + (k - Ep)]);
+      }
+      if (k == 0) {
+        float b;
+        if (kind == 2 && g == 2) b = bih[2 * H + j];        // b_in
+        else if (kind == 2 && g == 3) b = bhh[2 * H + j];   // b_hn
+        else b = bih[src_gate * H + j] + bhh[src_gate * H + j];
+        bias[r] = b;
+      }
+    } else if (k == 0) {
+      bias[r] = 0.0f;
+    }
+    Wcat[i] = __float2bfloat16_rn(v);
+  }
 }
 
 }  // namespace
+
+void rnn_pack(int kind, const void* Wih, const void* Whh, const float* bih, const float* bhh, void* Wcat, float* bias,
+              int E, int Ep, int H, int U, int BN, int tiles, cudaStream_t st) {
+  const int64_t rows = (int64_t)tiles * BN;
+  rnn_pack_kernel<<<grid_for(rows * (Ep + H), 256), 256, 0, st>>>(
+      kind, (const __nv_bfloat16*)Wih, (const __nv_bfloat16*)Whh, bih, bhh, (__nv_bfloat16*)Wcat, bias, E, Ep, H, U,
+      BN, rows);
+  CK(cudaGetLastError());
+}
 
 CUtensorMap make_tmap_bf16_2d(const void* base, int64_t rows, int64_t cols, int box_rows) {
   if (((uintptr_t)base & 15) || (cols * 2) % 16)
@@ -310,14 +352,15 @@ void gemm_tc(const void* A, const void* W, int M, int N, int K, int bn, const Tc
 }
 
 void gemm_tc_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
-                  int epi, int out_bf16, cudaStream_t st) {
+                  int epi, int out_bf16, cudaStream_t st, const CUtensorMap* tx) {
+  const CUtensorMap& tmx = tx ? *tx : ta;
 #define DUET_TC_CASE(BNV)                                                        \
   case BNV:                                                                      \
     if (epi == EPI_BIAS_ACT) {                                                   \
       if (out_bf16)                                                              \
-        launch_tc<BNV, EPI_BIAS_ACT, __nv_bfloat16>(ta, tw, ep, M, N, K, st);    \
+        launch_tc<BNV, EPI_BIAS_ACT, __nv_bfloat16>(ta, tw, tmx, ep, M, N, K, st);    \
       else                                                                       \
-        launch_tc<BNV, EPI_BIAS_ACT, float>(ta, tw, ep, M, N, K, st);            \
+        launch_tc<BNV, EPI_BIAS_ACT, float>(ta, tw, tmx, ep, M, N, K, st);            \
       return;                                                                    \
     }                                                                            \
     break;
@@ -330,14 +373,14 @@ void gemm_tc_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, in
   }
 #undef DUET_TC_CASE
   if (epi == EPI_LSTM) {
-    if (bn == 128) return launch_tc<128, EPI_LSTM, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
-    if (bn == 256) return launch_tc<256, EPI_LSTM, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
-    if (bn == 64) return launch_tc<64, EPI_LSTM, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
+    if (bn == 128) return launch_tc<128, EPI_LSTM, __nv_bfloat16>(ta, tw, tmx, ep, M, N, K, st);
+    if (bn == 256) return launch_tc<256, EPI_LSTM, __nv_bfloat16>(ta, tw, tmx, ep, M, N, K, st);
+    if (bn == 64) return launch_tc<64, EPI_LSTM, __nv_bfloat16>(ta, tw, tmx, ep, M, N, K, st);
   }
   if (epi == EPI_GRU) {
-    if (bn == 96) return launch_tc<96, EPI_GRU, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
-    if (bn == 192) return launch_tc<192, EPI_GRU, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
-    if (bn == 48) return launch_tc<48, EPI_GRU, __nv_bfloat16>(ta, tw, ep, M, N, K, st);
+    if (bn == 128) return launch_tc<128, EPI_GRU, __nv_bfloat16>(ta, tw, tmx, ep, M, N, K, st);
+    if (bn == 256) return launch_tc<256, EPI_GRU, __nv_bfloat16>(ta, tw, tmx, ep, M, N, K, st);
+    if (bn == 64) return launch_tc<64, EPI_GRU, __nv_bfloat16>(ta, tw, tmx, ep, M, N, K, st);
   }
   fail(DUET_EUNSUPPORTED, "no tcgen05 tile for bn=" + std::to_string(bn) + " epi=" + std::to_string(epi));
 }

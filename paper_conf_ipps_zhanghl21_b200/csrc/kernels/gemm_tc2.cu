@@ -72,6 +72,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
   ptx::cluster_sync();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
 
   if (warp == 0) {
     if (lane == 0) {
@@ -151,8 +153,7 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, i
     attr = true;
   }
   dim3 grid(2 * ((N + BN - 1) / BN), (M + 2 * BM2 - 1) / (2 * BM2));
-  kern<<<grid, 192, C::SMEM, st>>>(a, w, ep, M, N, K);
-  CK(cudaGetLastError());
+  launch_pdl(kern, grid, dim3(192), C::SMEM, st, a, w, ep, M, N, K);
 }
 
 }  // namespace

@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <string>
+#include <utility>
 
 #include "../common.h"
 
@@ -26,13 +27,15 @@ struct TcEpilogue {
   void* out = nullptr;
   int ldo = 0;
   int act = 0;
-  // EPI_LSTM / EPI_GRU
-  const float* gx = nullptr;   // [M, N] step pre-activations (gate-block layout, biases folded)
+  // EPI_LSTM / EPI_GRU (fused step: K = [x_t (kx k-blocks, zero-padded to 64) | h_{t-1}], gate
+  // pre-activation = acc + bias; gate-block layout, G = 4 blocks for both LSTM (i,f,g,o) and GRU
+  // (r, z, n_x, n_h))
   float* c_state = nullptr;    // LSTM cell state [M, H] fp32
   const void* h_prev = nullptr;// [M, H] bf16 (GRU z*h term)
   void* h_next = nullptr;      // [M, H] bf16
-  const float* b_hn = nullptr; // GRU [H]
   int H = 0;
+  int kx = 0;                  // k-blocks read from the X map (x_t) before switching to A (h)
+  int x_row0 = 0;              // row offset of x_t in the X map ([S*B, E] time-major)
   int dbg = 0;  // micro-benchmark switches: 1 = skip UMMA, 2 = skip TMA, 4 = epilogue backoff
 };
 
@@ -42,7 +45,11 @@ int tc_pick_bn(int M, int N, int num_sms);
 void gemm_tc(const void* A, const void* W, int M, int N, int K, int bn, const TcEpilogue& ep, int epi,
              int out_bf16, cudaStream_t st);
 void gemm_tc_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
-                  int epi, int out_bf16, cudaStream_t st);
+                  int epi, int out_bf16, cudaStream_t st, const CUtensorMap* tx = nullptr);
+// Pack the fused, gate-block-interleaved recurrent weights / bias (runtime.cu builds them once):
+//   Wcat[r', :] = [W_ih-part (E, zero-padded to Ep) | W_hh-part (H)], bias[r'].
+void rnn_pack(int kind, const void* Wih, const void* Whh, const float* bih, const float* bhh, void* Wcat, float* bias,
+              int E, int Ep, int H, int U, int BN, int tiles, cudaStream_t st);
 
 // CTA-pair GEMM (gemm_tc2.cu): 256 x bn tiles, bn in {64,128,256}; W map box rows = bn / 2.
 int tc2_pick_bn(int M, int N, int K, int num_sms);
@@ -108,6 +115,23 @@ bool conv_tma_ok(const ConvShape& s);
 void im2col(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStream_t st);
 
 int num_sms(int device);
+
+// Launch with the programmatic-stream-serialization attribute (PDL): the kernel must execute
+// griddepcontrol.wait before touching data produced by the preceding kernel in the stream.
+template <typename... KArgs, typename... Args>
+void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  CK(cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...));
+}
 // blocks for a grid-stride kernel: enough for `work` items, capped at per_sm x SM count
 int grid_for(int64_t work, int threads, int per_sm = 8);
 

@@ -109,7 +109,8 @@ __global__ void rnn_bias_kernel(const float* bih, const float* bhh, const int32_
 
 int rnn_step_bn(int kind, int B, int H, int sms) {
   // tile width for the recurrent step: LSTM u in {16,32,64} (BN = 4u), GRU u in {16,32,64} (BN = 3u)
-  const int G = kind == EPI_LSTM ? 4 : 3;
+  (void)kind;
+  const int G = 4;  // fused step: 4 gate blocks for LSTM and GRU
   const int mt = (B + 127) / 128;
   int best = 0;
   for (int u : {64, 32, 16}) {
@@ -306,61 +307,52 @@ void build_op(Program& P, const Node& n, Op& op) {
     const float* bhh = (const float*)P.param(n.params[3]);
     const bool tc = x.dtype == kBF16 && E % 8 == 0 && H % 8 == 0;
     const int es = dtype_bytes(x.dtype);
-    // column layout of the gate pre-activations
-    int bn = tc ? rnn_step_bn(kind, B, H, sms) : 0;
-    const int U = tc ? bn / G : H;
-    const int tiles = tc ? (H + U - 1) / U : 1;
-    const int Np = tc ? tiles * bn : G * H;
-    std::vector<int32_t> old_of_new(Np);
-    for (int r = 0; r < Np; ++r) {
-      if (!tc) {
-        old_of_new[r] = r;
-        continue;
-      }
-      int t = r / bn, rem = r % bn, gate = rem / U, j = t * U + rem % U;
-      old_of_new[r] = j < H ? gate * H + j : -1;
-    }
-    int32_t* d_map = (int32_t*)P.alloc((int64_t)Np * 4);
-    CK(cudaMemcpy(d_map, old_of_new.data(), (size_t)Np * 4, cudaMemcpyHostToDevice));
-    float* bias = (float*)P.alloc((int64_t)Np * 4);
-    rnn_bias_kernel<<<(Np + 255) / 256, 256>>>(bih, bhh, d_map, bias, Np, H, kind == EPI_GRU);
-    CK(cudaGetLastError());
-    const float* bhn = bhh + 2 * H;
-    float* gx = (float*)P.alloc((int64_t)S * B * Np * 4);
     void* hb[2] = {P.alloc((int64_t)B * H * es), P.alloc((int64_t)B * H * es)};
     float* cst = (float*)P.alloc((int64_t)B * H * 4);
     if (tc) {
-      void* Wih_r = P.alloc((int64_t)Np * E * es);
-      void* Whh_r = P.alloc((int64_t)Np * H * es);
-      permute_rows(Wih, Wih_r, d_map, Np, (int64_t)E * es, 0);
-      permute_rows(Whh, Whh_r, d_map, Np, (int64_t)H * es, 0);
+      // fused step (kernels/gemm_tc.cu EPI_LSTM/EPI_GRU): K = [x_t (E, padded to Ep) | h_{t-1} (H)],
+      // 4 gate blocks per tile; no G_x buffer and no separate input-projection GEMM
+      const int bn = rnn_step_bn(kind, B, H, sms);
+      const int U = bn / 4;
+      const int tiles = (H + U - 1) / U;
+      const int Np = tiles * bn;
+      const int Ep = (E + 63) / 64 * 64;
+      const int Kc = Ep + H;
+      void* Wcat = P.alloc((int64_t)Np * Kc * 2);
+      float* bias = (float*)P.alloc((int64_t)Np * 4);
+      rnn_pack(kind, Wih, Whh, bih, bhh, Wcat, bias, E, Ep, H, U, bn, tiles, 0);
       CK(cudaDeviceSynchronize());
-      const int bn_in = tc2_pick_bn(S * B, Np, E, sms);
-      CUtensorMap t_wih = make_tmap_bf16_2d(Wih_r, Np, E, bn_in / 2);
-      CUtensorMap t_whh = make_tmap_bf16_2d(Whh_r, Np, H, bn);
+      CUtensorMap t_w = make_tmap_bf16_2d(Wcat, Np, Kc, bn);
       CUtensorMap t_h[2] = {make_tmap_bf16_2d(hb[0], B, H, 128), make_tmap_bf16_2d(hb[1], B, H, 128)};
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         CK(cudaMemsetAsync(hb[1], 0, (size_t)B * H * es, st));
         if (kind == EPI_LSTM) CK(cudaMemsetAsync(cst, 0, (size_t)B * H * 4, st));
         CUtensorMap tx = make_tmap_bf16_2d(T[in], (int64_t)S * B, E, 128);
-        TcEpilogue ep;
-        ep.bias = bias;
-        ep.out = gx;
-        ep.ldo = Np;
-        ep.act = ACT_NONE;
-        gemm_tc2_maps(tx, t_wih, S * B, Np, E, bn_in, ep, 0, st);
         for (int t = 0; t < S; ++t) {
           TcEpilogue e2;
-          e2.gx = gx + (size_t)t * B * Np;
+          e2.bias = bias;
           e2.c_state = cst;
           e2.h_prev = hb[(t + 1) & 1];
           e2.h_next = (t == S - 1) ? T[me] : hb[t & 1];
-          e2.b_hn = bhn;
           e2.H = H;
-          gemm_tc_maps(t_h[(t + 1) & 1], t_whh, B, Np, H, bn, e2, kind, 1, st);
+          e2.kx = Ep / 64;
+          e2.x_row0 = t * B;
+          // t = 0: h_{-1} = 0, so only the x_t part of K contributes
+          gemm_tc_maps(t_h[(t + 1) & 1], t_w, B, Np, t == 0 ? Ep : Kc, bn, e2, kind, 1, st, &tx);
         }
       };
+      op.n_kernels = S;
     } else {
+      // fp32 parity path (original PyTorch layout): G_x = x W_ih^T + folded bias, then SIMT steps
+      std::vector<int32_t> ident(G * H);
+      for (int r = 0; r < G * H; ++r) ident[r] = r;
+      int32_t* d_map = (int32_t*)P.alloc((int64_t)G * H * 4);
+      CK(cudaMemcpy(d_map, ident.data(), (size_t)G * H * 4, cudaMemcpyHostToDevice));
+      float* bias = (float*)P.alloc((int64_t)G * H * 4);
+      rnn_bias_kernel<<<(G * H + 255) / 256, 256>>>(bih, bhh, d_map, bias, G * H, H, kind == EPI_GRU);
+      CK(cudaGetLastError());
+      const float* bhn = bhh + 2 * H;
+      float* gx = (float*)P.alloc((int64_t)S * B * G * H * 4);
       const int xb = x.dtype == kBF16;
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         CK(cudaMemsetAsync(hb[1], 0, (size_t)B * H * es, st));
@@ -371,8 +363,8 @@ void build_op(Program& P, const Node& n, Op& op) {
           rnn_step_simt(kind, gx + (size_t)t * B * G * H, Whh, xb, bhn, hb[(t + 1) & 1], hn, xb, cst, B, H, st);
         }
       };
+      op.n_kernels = 1 + S;
     }
-    op.n_kernels = 1 + S;
   } else if (n.op == "conv2d_bn") {
     nargs(1, 5);
     const Node& x = argn(0);

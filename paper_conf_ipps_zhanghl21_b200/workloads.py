@@ -319,9 +319,33 @@ SMALL = {
 }
 
 
-def build(name: str, small: bool = False, dt: str | None = None, **kw) -> Workload:
+def with_branch_outputs(wl: Workload) -> Workload:
+    """Also expose every branch result feeding the final join as a graph output (parity tests check
+    each branch, not only the join)."""
+    import re
+    lines = wl.ir.splitlines()
+    decl = {}
+    for ln in lines:
+        m = re.match(r"^%([\w.]+) = (\w+)\((.*?)\).*: (\w+)\[([0-9,]*)\]$", ln)
+        if m:
+            decl[m.group(1)] = (m.group(2), [a.strip()[1:] for a in m.group(3).split(",") if a.strip().startswith("%")],
+                                m.group(4), tuple(int(x) for x in m.group(5).split(",")))
+    join = wl.outputs[0][0]
+    extra = [a for a in decl[join][1] if a not in [o[0] for o in wl.outputs]]
+    out_idx = next(i for i, ln in enumerate(lines) if ln.startswith("output "))
+    lines[out_idx] += "".join(f", %{a}" for a in extra)
+    outs = list(wl.outputs) + [(a, decl[a][2], decl[a][3]) for a in extra]
+    # duet_run / the oracle order outputs by node declaration order
+    order = {nm: i for i, nm in enumerate(decl)}
+    outs.sort(key=lambda o: order[o[0]])
+    return Workload(wl.name, "\n".join(lines) + "\n", wl.params, wl.inputs, outs, wl.batch, dict(wl.meta))
+
+
+def build(name: str, small: bool = False, dt: str | None = None, branch_outputs: bool = False,
+          **kw) -> Workload:
     args = dict(SMALL[name]) if small else {}
     args.update(kw)
     if dt is not None:
         args["dt"] = dt
-    return CONFIGS[name](**args)
+    wl = CONFIGS[name](**args)
+    return with_branch_outputs(wl) if branch_outputs else wl

@@ -89,7 +89,7 @@ CASES = [("c1", "f32"), ("c1", "bf16"), ("c2", "bf16"), ("c2", "f32"), ("c3", "b
 
 @pytest.mark.parametrize("cfg,dt", CASES)
 def test_config_small_parity(cfg, dt):
-    wl = W.build(cfg, small=True, dt=dt)
+    wl = W.build(cfg, small=True, dt=dt, branch_outputs=True)
     sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
     inputs = list(materialize(wl.inputs, "cuda").values())
     want = _oracle_outputs(wl, sess.params, dict(zip(wl.inputs, inputs)))
@@ -174,3 +174,33 @@ def test_conv_node(N, H, W, C, Co, k, stride, pad):
     err = rel_err(y.float().cpu().numpy(), want)
     print(f"[parity] conv {N}x{H}x{W}x{C}->{Co} k{k}s{stride}: rel err {err:.3e}")
     assert err <= TOL["bf16"], err
+
+
+@pytest.mark.parametrize("kind,S,B,E,H,dt", [
+    ("lstm", 7, 300, 64, 48, "bf16"),    # ragged B (3 M tiles), H not a multiple of the unit tile
+    ("lstm", 5, 64, 40, 136, "bf16"),    # E padded to 64, H > one tile
+    ("gru", 6, 200, 64, 72, "bf16"),
+    ("gru", 4, 130, 24, 256, "bf16"),
+    ("lstm", 5, 33, 24, 40, "f32"),      # CUDA-core parity path
+    ("gru", 5, 33, 24, 40, "f32"),
+])
+def test_rnn_node(kind, S, B, E, H, dt):
+    G = 4 if kind == "lstm" else 3
+    ir = _single_node_graph(
+        f"%y = {kind}(%x, @Wih, @Whh, @bih, @bhh) : {dt}[{B},{H}]",
+        {"Wih": (dt, (G * H, E)), "Whh": (dt, (G * H, H)), "bih": ("f32", (G * H,)), "bhh": ("f32", (G * H,))},
+        {"x": (dt, (S, B, E))})
+    sc = 1.0 / np.sqrt(H)
+    x = _rand((S, B, E), dt, 1.0, 11)
+    Wih, Whh = _rand((G * H, E), dt, sc, 12), _rand((G * H, H), dt, sc, 13)
+    bih, bhh = _rand((G * H,), "f32", sc, 14), _rand((G * H,), "f32", sc, 15)
+    g = duet.Graph(ir)
+    g.bind_all({"Wih": Wih.cuda(), "Whh": Whh.cuda(), "bih": bih.cuda(), "bhh": bhh.cuda()})
+    y = torch.empty((B, H), dtype=torch.bfloat16 if dt == "bf16" else torch.float32, device="cuda")
+    g.node_run("y", [x.cuda()], y)
+    torch.cuda.synchronize()
+    f = lambda t, d: OF.to_f64(to_np(t), d)
+    want = (OF.lstm if kind == "lstm" else OF.gru)(f(x, dt), f(Wih, dt), f(Whh, dt), f(bih, "f32"), f(bhh, "f32"))
+    err = rel_err(y.float().cpu().numpy(), want)
+    print(f"[parity] {kind} S{S} B{B} E{E} H{H} {dt}: rel err {err:.3e}")
+    assert err <= TOL[dt], err
