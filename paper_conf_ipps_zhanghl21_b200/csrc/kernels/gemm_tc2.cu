@@ -18,13 +18,16 @@ namespace duet {
 namespace {
 
 constexpr int BM2 = 128;  // rows per CTA (256 per pair)
-constexpr int BK2 = 64;
-constexpr int A2_BYTES = BM2 * BK2 * 2;
+constexpr int BK2 = 64;   // one SWIZZLE_128B atom of K
+constexpr int KB2 = 2;    // k-blocks per pipeline stage: halves barrier round trips per FLOP
+constexpr int A2_ATOM = BM2 * BK2 * 2;
+constexpr int A2_BYTES = KB2 * A2_ATOM;
 
 template <int BN>
 struct Cfg2 {
   static constexpr int BH = BN / 2;  // W rows per CTA
-  static constexpr int B_BYTES = BH * BK2 * 2;
+  static constexpr int B_ATOM = BH * BK2 * 2;
+  static constexpr int B_BYTES = KB2 * B_ATOM;
   static constexpr int STAGE = A2_BYTES + B_BYTES;
   static constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
@@ -52,7 +55,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
   const int tile_n = blockIdx.x >> 1;
   const int n0 = tile_n * BN;
   const int m0 = blockIdx.y * (2 * BM2) + (int)rank * BM2;  // this CTA's rows
-  const int nk = (K + BK2 - 1) / BK2;
+  const int nk = (K + KB2 * BK2 - 1) / (KB2 * BK2);  // stages of KB2 k-blocks
 
   if (warp == 0 && lane == 0) {
     ptx::tma_prefetch(&tmA);
@@ -88,8 +91,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
           continue;
         }
         if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
-        ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES, kb * BK2, m0);
-        ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES, kb * BK2, n0 + (int)rank * C::BH);
+#pragma unroll
+        for (int h = 0; h < KB2; ++h) {
+          ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
+          ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
+                               n0 + (int)rank * C::BH);
+        }
       }
     }
   } else if (warp == 1) {
@@ -99,12 +106,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
         const int s = kb % C::STAGES;
         ptx::mbar_wait(&full[s], (kb / C::STAGES) & 1);
         ptx::tc_fence_after();
-        const uint32_t a_base = ptx::smem_u32(sA + s * A2_BYTES);
-        const uint32_t b_base = ptx::smem_u32(sB + s * C::B_BYTES);
 #pragma unroll
-        for (int k = 0; k < BK2 / 16; ++k)
-          if (!(ep.dbg & 1)) ptx::umma_bf16_2sm(tmem, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
-                             (kb | k) != 0);
+        for (int h = 0; h < KB2; ++h) {
+          const uint32_t a_base = ptx::smem_u32(sA + s * A2_BYTES + h * A2_ATOM);
+          const uint32_t b_base = ptx::smem_u32(sB + s * C::B_BYTES + h * C::B_ATOM);
+#pragma unroll
+          for (int k = 0; k < BK2 / 16; ++k)
+            if (!(ep.dbg & 1))
+              ptx::umma_bf16_2sm(tmem, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
+                                 (kb | h | k) != 0);
+        }
         ptx::umma_commit_2sm(&empty[s], 0x3);
       }
       ptx::umma_commit_2sm(tmem_full, 0x3);
