@@ -122,7 +122,7 @@ def dominant_kernel(wl, cfg):
     return None, None, None
 
 
-def time_node(torch, graph, node, args, out, stream, iters=20, replays=20):
+def time_node(torch, graph, node, args, out, stream, iters=50, replays=20):
     """Average device time of one launch of `node`'s kernel(s): `iters` launches captured in a CUDA
     graph (no host overhead), replayed `replays` times between CUDA events on `stream`."""
     graph.node_run(node, args, out, stream)

@@ -34,8 +34,11 @@ struct Cfg2 {
   static constexpr int SMEM = STAGES * STAGE + 1024 + 256 + BN * 4;
 };
 
-template <int BN, typename OutT>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
+// MC = 1: cluster of 4 CTAs = 2 pairs along N sharing the A rows; pair 0 loads A once and
+// multicasts it to pair 1 (halves A's L2->SMEM traffic).  MMA commits go to all 4 CTAs so a
+// stage is refilled only after both pairs consumed it (empty barrier count 2).
+template <int BN, typename OutT, int MC>
+__global__ void __launch_bounds__(192, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                  const TcEpilogue ep, int M, int N, int K) {
   using C = Cfg2<BN>;
@@ -51,8 +54,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
 
   const int warp = ptx::warp_id();
   const int lane = threadIdx.x & 31;
-  const uint32_t rank = ptx::cluster_ctarank();
-  const int tile_n = blockIdx.x >> 1;
+  const uint32_t crank = ptx::cluster_ctarank();
+  const uint32_t rank = crank & 1;          // rank within the CTA pair
+  const int pair = MC ? (int)(crank >> 1) : 0;
+  const int tile_n = MC ? (blockIdx.x >> 2) * 2 + pair : (blockIdx.x >> 1);
   const int n0 = tile_n * BN;
   const int m0 = blockIdx.y * (2 * BM2) + (int)rank * BM2;  // this CTA's rows
   const int nk = (K + KB2 * BK2 - 1) / (KB2 * BK2);  // stages of KB2 k-blocks
@@ -62,7 +67,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
     ptx::tma_prefetch(&tmW);
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
-      ptx::mbar_init(&empty[s], 1);
+      ptx::mbar_init(&empty[s], MC ? 2 : 1);
     }
     ptx::mbar_init(tmem_full, 1);
     ptx::fence_mbar_init();
@@ -80,8 +85,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
 
   if (warp == 0) {
     if (lane == 0) {
-      // full barriers live in the leader CTA; both CTAs' copies complete there
-      const uint32_t full_leader0 = ptx::mapa(ptx::smem_u32(&full[0]), 0);
+      // full barriers live in each pair's leader CTA; both CTAs' copies complete there
+      const uint32_t full_leader0 = ptx::mapa(ptx::smem_u32(&full[0]), crank & ~1u);
+      const uint16_t a_mask = (uint16_t)(0x5u << rank);  // CTA r of pair 0 and of pair 1
       for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % C::STAGES;
         if (kb >= C::STAGES) ptx::mbar_wait(&empty[s], ((kb / C::STAGES) - 1) & 1);
@@ -93,7 +99,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
         if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
 #pragma unroll
         for (int h = 0; h < KB2; ++h) {
-          ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
+          if (!MC)
+            ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
+          else if (pair == 0)
+            ptx::tma_load_2d_2sm_mc(&tmA, &full[s], sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0, a_mask);
           ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
                                n0 + (int)rank * C::BH);
         }
@@ -102,6 +111,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
   } else if (warp == 1) {
     if (rank == 0 && lane == 0) {
       constexpr uint32_t idesc = ptx::idesc_bf16(2 * BM2, BN);
+      const uint16_t empty_mask = MC ? (uint16_t)0xF : (uint16_t)0x3;
+      const uint16_t pair_mask = (uint16_t)(0x3u << (2 * pair));
       for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % C::STAGES;
         ptx::mbar_wait(&full[s], (kb / C::STAGES) & 1);
@@ -116,9 +127,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
               ptx::umma_bf16_2sm(tmem, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
                                  (kb | h | k) != 0);
         }
-        ptx::umma_commit_2sm(&empty[s], 0x3);
+        ptx::umma_commit_2sm(&empty[s], empty_mask);
       }
-      ptx::umma_commit_2sm(tmem_full, 0x3);
+      ptx::umma_commit_2sm(tmem_full, pair_mask);
     }
   } else {
     // epilogue warps 2..5: stage this tile's bias in smem while the mainloop runs
@@ -154,17 +165,33 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1)
   }
 }
 
-template <int BN, typename OutT>
+template <int BN, typename OutT, int MC>
 void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, int M, int N, int K, cudaStream_t st) {
   using C = Cfg2<BN>;
-  auto kern = gemm2_kernel<BN, OutT>;
+  auto kern = gemm2_kernel<BN, OutT, MC>;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
+    if (MC) CK(cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 0));
     attr = true;
   }
-  dim3 grid(2 * ((N + BN - 1) / BN), (M + 2 * BM2 - 1) / (2 * BM2));
-  launch_pdl(kern, grid, dim3(192), C::SMEM, st, a, w, ep, M, N, K);
+  const int tn = (N + BN - 1) / BN;
+  dim3 grid(MC ? 4 * ((tn + 1) / 2) : 2 * tn, (M + 2 * BM2 - 1) / (2 * BM2));
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = dim3(192);
+  cfg.dynamicSmemBytes = C::SMEM;
+  cfg.stream = st;
+  cudaLaunchAttribute attr2[2];
+  attr2[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr2[0].val.programmaticStreamSerializationAllowed = 1;
+  attr2[1].id = cudaLaunchAttributeClusterDimension;
+  attr2[1].val.clusterDim.x = MC ? 4 : 2;
+  attr2[1].val.clusterDim.y = 1;
+  attr2[1].val.clusterDim.z = 1;
+  cfg.attrs = attr2;
+  cfg.numAttrs = 2;
+  CK(cudaLaunchKernelEx(&cfg, kern, a, w, ep, M, N, K));
 }
 
 }  // namespace
@@ -184,11 +211,22 @@ int tc2_pick_bn(int M, int N, int K, int sms) {
 
 void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
                    int out_bf16, cudaStream_t st) {
+  // multicast pairs (opt-in, DUET_GEMM_MC=1): measured no gain at cluster size 4 (L2 dedups multicast
+  // only for wider clusters), kept for the wider-cluster experiments
+  static const int mc_env = getenv("DUET_GEMM_MC") ? atoi(getenv("DUET_GEMM_MC")) : 0;
+  const bool mc = mc_env && (N + bn - 1) / bn >= 2;
+#define DUET_L2(BNV)                                                                      \
+  if (mc)                                                                                 \
+    return out_bf16 ? launch2<BNV, __nv_bfloat16, 1>(ta, tw, ep, M, N, K, st)            \
+                    : launch2<BNV, float, 1>(ta, tw, ep, M, N, K, st);                    \
+  return out_bf16 ? launch2<BNV, __nv_bfloat16, 0>(ta, tw, ep, M, N, K, st)              \
+                  : launch2<BNV, float, 0>(ta, tw, ep, M, N, K, st);
   switch (bn) {
-    case 64: return out_bf16 ? launch2<64, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<64, float>(ta, tw, ep, M, N, K, st);
-    case 128: return out_bf16 ? launch2<128, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<128, float>(ta, tw, ep, M, N, K, st);
-    case 256: return out_bf16 ? launch2<256, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<256, float>(ta, tw, ep, M, N, K, st);
+    case 64: DUET_L2(64)
+    case 128: DUET_L2(128)
+    case 256: DUET_L2(256)
   }
+#undef DUET_L2
   fail(DUET_EUNSUPPORTED, "gemm_tc2: bn must be 64, 128 or 256");
 }
 

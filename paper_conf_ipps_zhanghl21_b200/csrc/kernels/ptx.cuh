@@ -287,6 +287,17 @@ __device__ __forceinline__ void tma_load_2d_2sm(const CUtensorMap* m, uint32_t b
       "l"((uint64_t)m), "r"(bar_cl), "r"(c0), "r"(c1)
       : "memory");
 }
+// 2-SM TMA with multicast: copies land at the same smem offset in every CTA of `mask`; each
+// destination's transaction bytes complete on its pair leader's barrier (peer bit cleared).
+__device__ __forceinline__ void tma_load_2d_2sm_mc(const CUtensorMap* m, uint64_t* bar, void* dst, int c0, int c1,
+                                                   uint16_t mask) {
+  const uint32_t b = smem_u32(bar) & 0xFEFFFFFFu;
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster "
+      "[%0], [%1, {%4, %5}], [%2], %3;" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)m), "r"(b), "h"(mask), "r"(c0), "r"(c1)
+      : "memory");
+}
 __device__ __forceinline__ void tmem_alloc_2sm(uint32_t* dst_smem, uint32_t ncols) {
   asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
                "r"(ncols)

@@ -624,8 +624,16 @@ struct ExecCache {
 
 void destroy_exec(ExecCache* e) { delete e; }
 
+struct HostCopy {
+  void* dst;
+  const void* src;
+  size_t bytes;
+  cudaMemcpyKind kind;
+};
+
 static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<cudaStream_t>& streams,
-                         const Ptrs& T, int64_t* launches) {
+                         const Ptrs& T, const std::vector<HostCopy>& h2d, const std::vector<HostCopy>& d2h,
+                         int64_t* launches) {
   const Partition& part = *S.p;
   ExecEntry E;
   cudaStream_t home = streams[0];
@@ -646,6 +654,8 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
   int64_t nk = 0;
   CK(cudaStreamBeginCapture(home, cudaStreamCaptureModeRelaxed));
   try {
+    // pinned-host inputs/outputs are memcpy nodes of the same graph: one launch per inference
+    for (auto& c : h2d) CK(cudaMemcpyAsync(c.dst, c.src, c.bytes, c.kind, home));
     CK(cudaEventRecord(fork, home));
     std::vector<char> forked(streams.size(), 0);
     std::vector<int> last_on(streams.size(), -1);
@@ -672,6 +682,7 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
     }
     for (size_t q = 0; q < streams.size(); ++q)
       if (last_on[q] >= 0 && streams[q] != home) CK(cudaStreamWaitEvent(home, done[last_on[q]], 0));
+    for (auto& c : d2h) CK(cudaMemcpyAsync(c.dst, c.src, c.bytes, c.kind, home));
   } catch (...) {
     cudaGraph_t junk = nullptr;
     cudaStreamEndCapture(home, &junk);
@@ -706,6 +717,7 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
   DeviceGuard dg(P->device);
   cudaStream_t home = streams[0];
   Ptrs T = P->buf;
+  std::vector<HostCopy> h2d, d2h;
   for (int i = 0; i < n_in; ++i) {
     const Node& nd = g->nodes[g->input_nodes[i]];
     check_tensor(nd, in[i], "input");
@@ -713,7 +725,7 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
       if (in[i].device != P->device) fail(DUET_EUNSUPPORTED, "input on another GPU");
       T[nd.id] = in[i].data;
     } else {
-      CK(cudaMemcpyAsync(P->buf[nd.id], in[i].data, (size_t)nd.nbytes(), cudaMemcpyHostToDevice, home));
+      h2d.push_back({P->buf[nd.id], in[i].data, (size_t)nd.nbytes(), cudaMemcpyHostToDevice});
     }
   }
   for (int i = 0; i < n_out; ++i) {
@@ -722,6 +734,8 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
     if (out[i].device >= 0) {
       if (out[i].device != P->device) fail(DUET_EUNSUPPORTED, "output on another GPU");
       T[nd.id] = out[i].data;
+    } else {
+      d2h.push_back({out[i].data, P->buf[nd.id], (size_t)nd.nbytes(), cudaMemcpyDeviceToHost});
     }
   }
   if (!S->exec || S->exec->prog.lock() != P) {
@@ -731,12 +745,14 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
   }
   std::vector<void*> key(T.begin(), T.end());
   for (auto st : streams) key.push_back((void*)st);
+  for (auto& c : h2d) key.push_back(const_cast<void*>(c.src));
+  for (auto& c : d2h) key.push_back(c.dst);
   ExecEntry* hit = nullptr;
   for (auto& e : S->exec->entries)
     if (e.key == key) hit = &e;
   if (!hit) {
     int64_t nk = 0;
-    ExecEntry E = capture(*P, *S, streams, T, &nk);
+    ExecEntry E = capture(*P, *S, streams, T, h2d, d2h, &nk);
     E.key = key;
     S->exec->launches = nk;
     if (S->exec->entries.size() >= 8) {
@@ -750,11 +766,6 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
     hit = &S->exec->entries.back();
   }
   CK(cudaGraphLaunch(hit->exec, home));
-  for (int i = 0; i < n_out; ++i) {
-    const Node& nd = g->nodes[g->outputs[i]];
-    if (out[i].device < 0)
-      CK(cudaMemcpyAsync(out[i].data, P->buf[nd.id], (size_t)nd.nbytes(), cudaMemcpyDeviceToHost, home));
-  }
 }
 
 int64_t schedule_launch_count(const Schedule* s) {
