@@ -266,6 +266,8 @@ def main():
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
     home = sess.home
 
+    torch.cuda.synchronize()  # inputs were generated on the default stream; duet_run uses `home`
+
     def step_duet():
         duet_s.run(sess.slots, inputs, outs)
 

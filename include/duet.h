@@ -202,8 +202,10 @@ duet_status duet_schedule_export(const duet_schedule_t* s, int32_t* sg_to_slot, 
 void duet_schedule_destroy(duet_schedule_t* s);
 
 /* ---- run (§IV-D) ---------------------------------------------------------------- */
-/* Enqueue one inference on slots[0].stream (asynchronous; no host sync).  inputs[] follow the
- * IR's input nodes in declaration order, outputs[] the IR's output list.  Device tensors are
+/* Enqueue one inference on slots[0].stream (asynchronous; no host sync).  The caller orders the
+ * home stream after the producers of the inputs (e.g. an event wait) and reads the outputs after
+ * the home stream reaches this point.  inputs[] follow the IR's input nodes in declaration order,
+ * outputs[] the IR's output nodes in declaration order.  Device tensors are
  * used in place; HOST tensors are copied H2D before / D2H after the graph on the home stream
  * (pinned memory keeps this asynchronous).  Slot streams other than the home stream only shape
  * the captured CUDA graph (one graph per distinct (slots, tensor pointers) — cached). */

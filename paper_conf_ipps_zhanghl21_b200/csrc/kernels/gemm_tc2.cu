@@ -182,9 +182,10 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, i
   cfg.blockDim = dim3(192);
   cfg.dynamicSmemBytes = C::SMEM;
   cfg.stream = st;
+  static const bool no_pdl = getenv("DUET_NO_PDL") != nullptr;
   cudaLaunchAttribute attr2[2];
   attr2[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr2[0].val.programmaticStreamSerializationAllowed = 1;
+  attr2[0].val.programmaticStreamSerializationAllowed = no_pdl ? 0 : 1;
   attr2[1].id = cudaLaunchAttributeClusterDimension;
   attr2[1].val.clusterDim.x = MC ? 4 : 2;
   attr2[1].val.clusterDim.y = 1;

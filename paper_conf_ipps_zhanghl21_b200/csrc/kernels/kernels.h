@@ -3,6 +3,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <string>
 #include <utility>
 
@@ -125,11 +126,12 @@ void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cuda
   cfg.blockDim = block;
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
+  static const bool no_pdl = getenv("DUET_NO_PDL") != nullptr;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = no_pdl ? 0 : 1;
   CK(cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...));
 }
 // blocks for a grid-stride kernel: enough for `work` items, capped at per_sm x SM count

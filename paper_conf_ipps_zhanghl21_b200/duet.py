@@ -170,7 +170,7 @@ class Graph:
         self._keep = {}
 
     def __del__(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:  # (module globals vanish at interpreter exit)
             _lib.duet_graph_destroy(self._h)
             self._h = None
 
@@ -205,7 +205,7 @@ class Partition:
         self._h, self.graph = h, graph
 
     def __del__(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:  # (module globals vanish at interpreter exit)
             _lib.duet_partition_destroy(self._h)
             self._h = None
 
@@ -260,7 +260,7 @@ class Profile:
         self._h, self.part = h, part
 
     def __del__(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:  # (module globals vanish at interpreter exit)
             _lib.duet_profile_destroy(self._h)
             self._h = None
 
@@ -290,7 +290,7 @@ class Schedule:
         self._h, self.prof = h, prof
 
     def __del__(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:  # (module globals vanish at interpreter exit)
             _lib.duet_schedule_destroy(self._h)
             self._h = None
 

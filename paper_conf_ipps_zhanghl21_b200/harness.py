@@ -50,6 +50,9 @@ class Session:
         return out
 
     def run(self, sched: duet.Schedule, inputs, outputs):
+        # duet_run enqueues on the home slot stream (non-blocking w.r.t. the legacy stream): order it
+        # after whatever produced the inputs / last used the outputs on the caller's current stream
+        self.home.wait_stream(torch.cuda.current_stream(self.device))
         sched.run(self.slots, inputs, outputs)
 
     @property

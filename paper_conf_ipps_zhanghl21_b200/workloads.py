@@ -115,12 +115,12 @@ class _Builder:
         bhh = self.param(f"{name}_bhh", "f32", (g * h,), ("uniform", bd))
         return self.node(name, kind, [x, Wih, Whh, bih, bhh], self.dt, (b, h))
 
-    def conv_bn(self, name, x, n, h, w, cin, cout, k, stride, pad, act):
+    def conv_bn(self, name, x, n, h, w, cin, cout, k, stride, pad, act, gamma=(0.5, 1.5)):
         ho = (h + 2 * pad - k) // stride + 1
         wo = (w + 2 * pad - k) // stride + 1
         std = math.sqrt(2.0 / (cin * k * k))  # Kaiming-normal (fan_in, ReLU gain)
         W = self.param(f"{name}_W", self.dt, (cout, k, k, cin), ("normal", std))
-        g = self.param(f"{name}_gamma", "f32", (cout,), ("uniform_range", 0.5, 1.5))
+        g = self.param(f"{name}_gamma", "f32", (cout,), ("uniform_range", *gamma))
         be = self.param(f"{name}_beta", "f32", (cout,), ("normal", 0.1))
         mu = self.param(f"{name}_mean", "f32", (cout,), ("normal", 0.1))
         var = self.param(f"{name}_var", "f32", (cout,), ("uniform_range", 0.5, 1.5))
@@ -139,7 +139,9 @@ class _Builder:
                 stride = 2 if (li > 0 and bi == 0) else 1
                 nm = f"{prefix}_l{li + 1}b{bi}"
                 y, h2, w2 = self.conv_bn(nm + "_c1", c, n, h, w, cin, cout, 3, stride, 1, "relu")
-                y, h2, w2 = self.conv_bn(nm + "_c2", y, n, h2, w2, cout, cout, 3, 1, 1, "none")
+                # residual-branch BN gamma ~ U(0.1, 0.3): keeps activations O(1) through the stack
+                # like a trained network (an untrained Kaiming ResNet doubles the variance per block)
+                y, h2, w2 = self.conv_bn(nm + "_c2", y, n, h2, w2, cout, cout, 3, 1, 1, "none", gamma=(0.1, 0.3))
                 if stride != 1 or cin != cout:
                     sc, _, _ = self.conv_bn(nm + "_ds", c, n, h, w, cin, cout, 1, stride, 0, "none")
                 else:

@@ -124,6 +124,28 @@ def test_host_buffers_e2e_equal_device():
     assert s.launch_count() >= 6
 
 
+@pytest.mark.parametrize("cfg,n_rows", [("c3", 6), ("c4", 2), ("c5", 6)])
+def test_full_size_sampled(cfg, n_rows):
+    """c3/c4/c5 at their BASELINE.json sizes (bench launch configuration: 2 slots, greedy-correction);
+    the oracle evaluates a few sampled batch rows (rows are independent) — every branch output."""
+    wl = W.build(cfg, branch_outputs=True)
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    outs = sess.outputs()
+    sess.run(sess.schedule(), inputs, outs)
+    torch.cuda.synchronize()
+    rows = np.random.default_rng(1).choice(wl.batch, n_rows, replace=False)
+    rows[0] = wl.batch - 1
+    oparams = {k: (lazy_rows(spec) if spec.numel > 10_000_000 else to_np(sess.params[k]))
+               for k, spec in wl.params.items()}
+    oin = {k: to_np(t)[rows] for k, t in zip(wl.inputs, inputs)}
+    want = OF.run(wl.ir, oparams, oin)
+    for (name, _, _), y in zip(wl.outputs, outs):
+        err = rel_err(y.float().cpu().numpy()[rows], want[name])
+        print(f"[parity] full {cfg} {name}: rel err {err:.3e}")
+        assert err <= TOL["bf16"], (cfg, name, err)
+
+
 def test_c2_full_size_sampled():
     """The bench workload (BASELINE.json:8 at full size) in the bench's launch configuration;
     the oracle evaluates 96 sampled rows (rows are independent), reading only the table rows they
