@@ -105,6 +105,8 @@ __global__ void fold_bn_kernel(const void* W, int bf16, const float* g, const fl
 // counters (no per-element division), write the row as 16-B stores
 __global__ void im2col_kernel(const __nv_bfloat16* __restrict__ x, __nv_bfloat16* __restrict__ cols, ConvShape s,
                               int ldk) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   const int K = s.kh * s.kw * s.C;
   const int M = s.N * s.Ho * s.Wo;
   const uint16_t* xs = reinterpret_cast<const uint16_t*>(x);
@@ -152,7 +154,8 @@ void im2col(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStre
   const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
   if (!M) return;
   if (M >= INT32_MAX || ldk % 8) fail(DUET_EUNSUPPORTED, "im2col: M < 2^31 and ldk % 8 == 0 required");
-  im2col_kernel<<<grid_for(M, 128, 16), 128, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)cols, s, (int)ldk);
+  launch_plain(im2col_kernel, dim3(grid_for(M, 128, 16)), dim3(128), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)cols, s,
+             (int)ldk);
   CK(cudaGetLastError());
 }
 

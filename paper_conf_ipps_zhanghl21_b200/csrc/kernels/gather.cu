@@ -32,6 +32,8 @@ __device__ __forceinline__ uint4 ld_stream16(const void* p) {
 }
 
 __global__ void hash_mod_kernel(const int64_t* __restrict__ raw, int32_t* __restrict__ ids, int64_t n, int64_t V) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     int64_t r = raw[i] % V;
     if (r < 0) r += V;
@@ -42,6 +44,8 @@ __global__ void hash_mod_kernel(const int64_t* __restrict__ raw, int32_t* __rest
 template <typename T>
 __global__ void gather_sum_kernel(const int32_t* __restrict__ ids, const T* __restrict__ tab,
                                   const float* __restrict__ b, float* __restrict__ y, int B, int F, int64_t R) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   const int warps = (blockDim.x >> 5);
   const int row = blockIdx.x * warps + (threadIdx.x >> 5);
   const int lane = threadIdx.x & 31;
@@ -60,6 +64,8 @@ template <int MODE>  // 0: gather_concat (row r = b*F + f), 1: embed_seq (row r 
 __global__ void gather_rows16_kernel(const int32_t* __restrict__ idx, const uint8_t* __restrict__ tab,
                                      uint8_t* __restrict__ out, int64_t rows, int vpr, int64_t row_bytes, int F,
                                      int64_t R, int B, int S) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   const int64_t total = rows * vpr;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -96,6 +102,8 @@ template <int MODE>
 __global__ void gather_rows_bytes_kernel(const int32_t* __restrict__ idx, const uint8_t* __restrict__ tab,
                                          uint8_t* __restrict__ out, int64_t rows, int64_t row_bytes, int F,
                                          int64_t R, int B, int S) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   const int64_t total = rows * row_bytes;
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < total; v += (int64_t)gridDim.x * blockDim.x) {
     int64_t r = v / row_bytes;
@@ -159,7 +167,7 @@ int grid_for(int64_t work, int threads, int per_sm) {
 
 void hash_mod(const int64_t* raw, int32_t* ids, int64_t n, int64_t V, cudaStream_t st) {
   if (n == 0) return;
-  hash_mod_kernel<<<grid_for(n, 256), 256, 0, st>>>(raw, ids, n, V);
+  launch_pdl(hash_mod_kernel, dim3(grid_for(n, 256)), dim3(256), 0, st, raw, ids, n, V);
   CK(cudaGetLastError());
 }
 
@@ -168,9 +176,9 @@ void gather_sum(const int32_t* ids, const void* T, int t_bf16, const float* b, f
   if (B == 0) return;
   int blocks = (B + 7) / 8;
   if (t_bf16)
-    gather_sum_kernel<__nv_bfloat16><<<blocks, 256, 0, st>>>(ids, (const __nv_bfloat16*)T, b, y, B, F, R);
+    launch_pdl(gather_sum_kernel<__nv_bfloat16>, dim3(blocks), dim3(256), 0, st, ids, (const __nv_bfloat16*)T, b, y, B, F, R);
   else
-    gather_sum_kernel<float><<<blocks, 256, 0, st>>>(ids, (const float*)T, b, y, B, F, R);
+    launch_pdl(gather_sum_kernel<float>, dim3(blocks), dim3(256), 0, st, ids, (const float*)T, b, y, B, F, R);
   CK(cudaGetLastError());
 }
 
@@ -184,15 +192,15 @@ static void gather_rows(int mode, const int32_t* idx, const void* tab, int esize
     int64_t total = rows * vpr;
     int g = grid_for((total + 3) / 4, 256, 16);
     if (mode == 0)
-      gather_rows16_kernel<0><<<g, 256, 0, st>>>(idx, (const uint8_t*)tab, (uint8_t*)out, rows, vpr, rb, F, R, B, S);
+      launch_pdl(gather_rows16_kernel<0>, dim3(g), dim3(256), 0, st, idx, (const uint8_t*)tab, (uint8_t*)out, rows, vpr, rb, F, R, B, S);
     else
-      gather_rows16_kernel<1><<<g, 256, 0, st>>>(idx, (const uint8_t*)tab, (uint8_t*)out, rows, vpr, rb, F, R, B, S);
+      launch_pdl(gather_rows16_kernel<1>, dim3(g), dim3(256), 0, st, idx, (const uint8_t*)tab, (uint8_t*)out, rows, vpr, rb, F, R, B, S);
   } else {
     int g = grid_for(rows * rb, 256);
     if (mode == 0)
-      gather_rows_bytes_kernel<0><<<g, 256, 0, st>>>(idx, (const uint8_t*)tab, (uint8_t*)out, rows, rb, F, R, B, S);
+      launch_pdl(gather_rows_bytes_kernel<0>, dim3(g), dim3(256), 0, st, idx, (const uint8_t*)tab, (uint8_t*)out, rows, rb, F, R, B, S);
     else
-      gather_rows_bytes_kernel<1><<<g, 256, 0, st>>>(idx, (const uint8_t*)tab, (uint8_t*)out, rows, rb, F, R, B, S);
+      launch_pdl(gather_rows_bytes_kernel<1>, dim3(g), dim3(256), 0, st, idx, (const uint8_t*)tab, (uint8_t*)out, rows, rb, F, R, B, S);
   }
   CK(cudaGetLastError());
 }

@@ -22,6 +22,8 @@ __device__ __forceinline__ void stx(void* p, int64_t i, float v, int bf16) {
 __device__ __forceinline__ int row_of_warp() { return blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); }
 
 __global__ void reduce_sum_kernel(const void* x, int bf16, const float* b, float* y, int B, int K) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   int row = row_of_warp(), lane = threadIdx.x & 31;
   if (row >= B) return;
   float s = 0.0f;
@@ -32,6 +34,8 @@ __global__ void reduce_sum_kernel(const void* x, int bf16, const float* b, float
 
 __global__ void dot_join_kernel(const float* s, const void* a, int bf16, const float* w, const float* b, float* y,
                                 int B, int K) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   int row = row_of_warp(), lane = threadIdx.x & 31;
   if (row >= B) return;
   float acc = 0.0f;
@@ -41,6 +45,8 @@ __global__ void dot_join_kernel(const float* s, const void* a, int bf16, const f
 }
 
 __global__ void cosine_join_kernel(const void* a, const void* b, int bf16, float* y, int B, int K) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   int row = row_of_warp(), lane = threadIdx.x & 31;
   if (row >= B) return;
   float ab = 0.0f, aa = 0.0f, bb = 0.0f;
@@ -67,6 +73,8 @@ struct HeadArgs {
 };
 
 __global__ void concat_head_kernel(HeadArgs h, const float* w, const float* b, float* y, int B, int act) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   int row = row_of_warp(), lane = threadIdx.x & 31;
   if (row >= B) return;
   float acc = 0.0f;
@@ -85,6 +93,8 @@ struct LogitArgs {
 };
 
 __global__ void logit_join_kernel(LogitArgs a, float* y, int B, int mean) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   int row = blockIdx.x * blockDim.x + threadIdx.x;
   if (row >= B) return;
   float s = 0.0f;
@@ -95,18 +105,24 @@ __global__ void logit_join_kernel(LogitArgs a, float* y, int B, int mean) {
 
 template <typename T>
 __global__ void add_act_kernel(const T* a, const T* b, T* y, int64_t n, int act) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     y[i] = from_f<T>(apply_act(to_f(a[i]) + to_f(b[i]), act));
 }
 
 template <typename T>
 __global__ void sigmoid_kernel(const T* x, T* y, int64_t n) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     y[i] = from_f<T>(sigmoidf_acc(to_f(x[i])));
 }
 
 template <typename T>
 __global__ void maxpool_kernel(const T* x, T* y, int N, int H, int W, int C, int k, int s, int p, int Ho, int Wo) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   int64_t total = (int64_t)N * Ho * Wo * C;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     int c = (int)(i % C);
@@ -132,6 +148,8 @@ __global__ void maxpool_kernel(const T* x, T* y, int N, int H, int W, int C, int
 // global average pool: one thread per (n, c), coalesced over c
 template <typename T>
 __global__ void avgpool_kernel(const T* x, T* y, int N, int HW, int C) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   int64_t total = (int64_t)N * C;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     int c = (int)(i % C);
@@ -148,6 +166,8 @@ int warp_rows_grid(int B) { return (B + 7) / 8; }
 // NHWC bf16 maxpool, 8 channels (16 B) per thread, 32-bit index math (C % 8 == 0)
 __global__ void maxpool8_kernel(const uint4* __restrict__ x, uint4* __restrict__ y, int N, int H, int W, int C8, int k,
                                 int s, int p, int Ho, int Wo) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   const int total = N * Ho * Wo * C8;
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += gridDim.x * blockDim.x) {
     int c8 = i % C8;
@@ -183,20 +203,20 @@ __global__ void maxpool8_kernel(const uint4* __restrict__ x, uint4* __restrict__
 
 void reduce_sum(const void* x, int x_bf16, const float* b, float* y, int B, int K, cudaStream_t st) {
   if (!B) return;
-  reduce_sum_kernel<<<warp_rows_grid(B), 256, 0, st>>>(x, x_bf16, b, y, B, K);
+  launch_pdl(reduce_sum_kernel, dim3(warp_rows_grid(B)), dim3(256), 0, st, x, x_bf16, b, y, B, K);
   CK(cudaGetLastError());
 }
 
 void dot_join(const float* s, const void* a, int a_bf16, const float* w, const float* b, float* y, int B, int K,
               cudaStream_t st) {
   if (!B) return;
-  dot_join_kernel<<<warp_rows_grid(B), 256, 0, st>>>(s, a, a_bf16, w, b, y, B, K);
+  launch_pdl(dot_join_kernel, dim3(warp_rows_grid(B)), dim3(256), 0, st, s, a, a_bf16, w, b, y, B, K);
   CK(cudaGetLastError());
 }
 
 void cosine_join(const void* a, const void* b, int bf16, float* y, int B, int K, cudaStream_t st) {
   if (!B) return;
-  cosine_join_kernel<<<warp_rows_grid(B), 256, 0, st>>>(a, b, bf16, y, B, K);
+  launch_pdl(cosine_join_kernel, dim3(warp_rows_grid(B)), dim3(256), 0, st, a, b, bf16, y, B, K);
   CK(cudaGetLastError());
 }
 
@@ -211,7 +231,7 @@ void concat_head(const void* const* parts, const int* Ks, const int* bf16s, int 
   }
   h.n = n;
   if (!B) return;
-  concat_head_kernel<<<warp_rows_grid(B), 256, 0, st>>>(h, w, b, y, B, act);
+  launch_pdl(concat_head_kernel, dim3(warp_rows_grid(B)), dim3(256), 0, st, h, w, b, y, B, act);
   CK(cudaGetLastError());
 }
 
@@ -221,26 +241,26 @@ void logit_join(const float* const* parts, int n, float* y, int B, int mean, cud
   for (int i = 0; i < n; ++i) a.p[i] = parts[i];
   a.n = n;
   if (!B) return;
-  logit_join_kernel<<<(B + 255) / 256, 256, 0, st>>>(a, y, B, mean);
+  launch_pdl(logit_join_kernel, dim3((B + 255) / 256), dim3(256), 0, st, a, y, B, mean);
   CK(cudaGetLastError());
 }
 
 void add_act(const void* a, const void* b, void* y, int bf16, int64_t n, int act, cudaStream_t st) {
   if (!n) return;
   if (bf16)
-    add_act_kernel<__nv_bfloat16><<<grid_for(n, 256), 256, 0, st>>>((const __nv_bfloat16*)a, (const __nv_bfloat16*)b,
+    launch_pdl(add_act_kernel<__nv_bfloat16>, dim3(grid_for(n, 256)), dim3(256), 0, st, (const __nv_bfloat16*)a, (const __nv_bfloat16*)b,
                                                                   (__nv_bfloat16*)y, n, act);
   else
-    add_act_kernel<float><<<grid_for(n, 256), 256, 0, st>>>((const float*)a, (const float*)b, (float*)y, n, act);
+    launch_pdl(add_act_kernel<float>, dim3(grid_for(n, 256)), dim3(256), 0, st, (const float*)a, (const float*)b, (float*)y, n, act);
   CK(cudaGetLastError());
 }
 
 void sigmoid_ew(const void* x, void* y, int bf16, int64_t n, cudaStream_t st) {
   if (!n) return;
   if (bf16)
-    sigmoid_kernel<__nv_bfloat16><<<grid_for(n, 256), 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, n);
+    launch_pdl(sigmoid_kernel<__nv_bfloat16>, dim3(grid_for(n, 256)), dim3(256), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)y, n);
   else
-    sigmoid_kernel<float><<<grid_for(n, 256), 256, 0, st>>>((const float*)x, (float*)y, n);
+    launch_pdl(sigmoid_kernel<float>, dim3(grid_for(n, 256)), dim3(256), 0, st, (const float*)x, (float*)y, n);
   CK(cudaGetLastError());
 }
 
@@ -250,16 +270,16 @@ void maxpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, 
   if (!total) return;
   if (bf16 && C % 8 == 0 && total / 8 < INT32_MAX && (int64_t)N * H * W * C / 8 < INT32_MAX &&
       ((uintptr_t)x % 16) == 0 && ((uintptr_t)y % 16) == 0) {
-    maxpool8_kernel<<<grid_for(total / 8, 256, 16), 256, 0, st>>>((const uint4*)x, (uint4*)y, N, H, W, C / 8, k, s, p,
-                                                                  Ho, Wo);
+    launch_plain(maxpool8_kernel, dim3(grid_for(total / 8, 256, 16)), dim3(256), 0, st, (const uint4*)x, (uint4*)y, N, H, W,
+               C / 8, k, s, p, Ho, Wo);
     CK(cudaGetLastError());
     return;
   }
   if (bf16)
-    maxpool_kernel<__nv_bfloat16><<<grid_for(total, 256), 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, N,
+    launch_plain(maxpool_kernel<__nv_bfloat16>, dim3(grid_for(total, 256)), dim3(256), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)y, N,
                                                                        H, W, C, k, s, p, Ho, Wo);
   else
-    maxpool_kernel<float><<<grid_for(total, 256), 256, 0, st>>>((const float*)x, (float*)y, N, H, W, C, k, s, p, Ho,
+    launch_plain(maxpool_kernel<float>, dim3(grid_for(total, 256)), dim3(256), 0, st, (const float*)x, (float*)y, N, H, W, C, k, s, p, Ho,
                                                                Wo);
   CK(cudaGetLastError());
 }
@@ -268,10 +288,10 @@ void avgpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, 
   int64_t total = (int64_t)N * C;
   if (!total) return;
   if (bf16)
-    avgpool_kernel<__nv_bfloat16><<<grid_for(total, 256), 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, N,
+    launch_plain(avgpool_kernel<__nv_bfloat16>, dim3(grid_for(total, 256)), dim3(256), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)y, N,
                                                                        H * W, C);
   else
-    avgpool_kernel<float><<<grid_for(total, 256), 256, 0, st>>>((const float*)x, (float*)y, N, H * W, C);
+    launch_plain(avgpool_kernel<float>, dim3(grid_for(total, 256)), dim3(256), 0, st, (const float*)x, (float*)y, N, H * W, C);
   CK(cudaGetLastError());
 }
 

@@ -134,6 +134,19 @@ void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cuda
   cfg.numAttrs = no_pdl ? 0 : 1;
   CK(cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...));
 }
+// Same, without the PDL attribute: full stream serialization (used for kernels adjacent to
+// persistent / cluster kernels in the CNN chain, where early dependent launch was observed to hang
+// back-to-back graph copies).
+template <typename... KArgs, typename... Args>
+void launch_plain(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cfg.numAttrs = 0;
+  CK(cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...));
+}
 // blocks for a grid-stride kernel: enough for `work` items, capped at per_sm x SM count
 int grid_for(int64_t work, int threads, int per_sm = 8);
 

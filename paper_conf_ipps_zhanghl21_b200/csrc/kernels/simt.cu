@@ -80,9 +80,13 @@ struct MlpArgs {
   int L;
 };
 
-// One CTA per block of up to 4 rows; activations ping-pong in shared memory (fp32).
-__global__ void mlp_small_kernel(const void* __restrict__ X, int bf16, MlpArgs a, void* __restrict__ Y, int y_bf16,
-                                 int M, int act, int last_act, int maxd) {
+// One CTA per block of up to 4 rows; activations ping-pong in shared memory (fp32).  32 warps;
+// each warp computes 2 outputs at a time with independent loads in flight (latency-bound at M = 1).
+__global__ void __launch_bounds__(1024) mlp_small_kernel(const void* __restrict__ X, int bf16, MlpArgs a,
+                                                         void* __restrict__ Y, int y_bf16, int M, int act, int last_act,
+                                                         int maxd) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
   extern __shared__ float sm[];
   const int R = 4;
   float* buf0 = sm;
@@ -100,17 +104,29 @@ __global__ void mlp_small_kernel(const void* __restrict__ X, int bf16, MlpArgs a
   for (int l = 0; l < a.L; ++l) {
     const int K = a.dims[l], N = a.dims[l + 1];
     const bool last = (l + 1 == a.L);
-    for (int o = warp; o < nr * N; o += nw) {
-      int r = o / N, n = o - r * N;
-      float s = 0.0f;
-      for (int k = lane; k < K; k += 32) s = fmaf(in[r * maxd + k], ldx(a.W[l], (int64_t)n * K + k, bf16), s);
-      s = warp_sum(s);
+    const int total = nr * N;
+    for (int o = warp * 2; o < total; o += nw * 2) {
+      const int o1 = o + 1 < total ? o + 1 : o;
+      const int ra = o / N, na = o - ra * N, rb = o1 / N, nb = o1 - rb * N;
+      float sa = 0.0f, sb = 0.0f;
+      for (int k = lane; k < K; k += 32) {
+        const float wa = ldx(a.W[l], (int64_t)na * K + k, bf16);
+        const float wb = ldx(a.W[l], (int64_t)nb * K + k, bf16);
+        sa = fmaf(in[ra * maxd + k], wa, sa);
+        sb = fmaf(in[rb * maxd + k], wb, sb);
+      }
+      sa = warp_sum(sa);
+      sb = warp_sum(sb);
       if (lane == 0) {
-        float v = apply_act(s + a.b[l][n], last ? last_act : act);
-        if (last)
-          stx(Y, (int64_t)(r0 + r) * N + n, v, y_bf16);
-        else
-          out[r * maxd + n] = bf16 ? __bfloat162float(__float2bfloat16_rn(v)) : v;  // stored-dtype rounding
+        const float va = apply_act(sa + a.b[l][na], last ? last_act : act);
+        const float vb = apply_act(sb + a.b[l][nb], last ? last_act : act);
+        if (last) {
+          stx(Y, (int64_t)(r0 + ra) * N + na, va, y_bf16);
+          if (o1 != o) stx(Y, (int64_t)(r0 + rb) * N + nb, vb, y_bf16);
+        } else {
+          out[ra * maxd + na] = bf16 ? __bfloat162float(__float2bfloat16_rn(va)) : va;  // stored-dtype rounding
+          if (o1 != o) out[rb * maxd + nb] = bf16 ? __bfloat162float(__float2bfloat16_rn(vb)) : vb;
+        }
       }
     }
     __syncthreads();
@@ -209,7 +225,7 @@ void mlp_small(const void* X, int bf16, const void* const* Ws, const float* cons
   size_t smem = (size_t)2 * 4 * maxd * sizeof(float);
   if (smem > 200 * 1024) fail(DUET_EUNSUPPORTED, "mlp: layer too wide for the fused small-M kernel");
   if (smem > 48 * 1024) CK(cudaFuncSetAttribute(mlp_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  mlp_small_kernel<<<(M + 3) / 4, 256, smem, st>>>(X, bf16, a, Y, y_bf16, M, act, last_act, maxd);
+  launch_pdl(mlp_small_kernel, dim3((M + 3) / 4), dim3(1024), smem, st, X, bf16, a, Y, y_bf16, M, act, last_act, maxd);
   CK(cudaGetLastError());
 }
 
