@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--profile-samples", type=int, default=100)
+    ap.add_argument("--sched", default="measured", choices=["measured", "model"],
+                    help="Step 3's `measure latency`: device measurement (default) or the C3 model")
     return ap.parse_args()
 
 
@@ -261,7 +263,9 @@ def main():
                    profile=dict(warmup=5, samples=args.profile_samples, reps=10, calibrate_comm=True))
     inputs = list(materialize(wl.inputs, dev).values())
     outs = sess.outputs()
-    duet_s = sess.schedule(duet.GREEDY_CORRECTION)
+    torch.cuda.synchronize()
+    model_s = sess.schedule(duet.GREEDY_CORRECTION)
+    duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=30) if args.sched == "measured" else model_s
     serial_s = sess.schedule(duet.SERIAL)
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
     home = sess.home
@@ -276,6 +280,10 @@ def main():
 
     # serial 1-stream reference of the same kernels (BASELINE.json:2)
     t_serial = time_steps(torch, step_serial, home, args.steps, args.warmup, flush)
+    t_model = None
+    if duet_s is not model_s and duet_s.export()["slot_of"] != model_s.export()["slot_of"]:
+        t_model = time_steps(torch, lambda: model_s.run(sess.slots, inputs, outs), home, args.steps, args.warmup,
+                             flush)
 
     # --- timed region (DUET) ---
     MR.barrier()
@@ -356,9 +364,13 @@ def main():
         "p999_ms": round(percentile(t_duet, 99.9), 5),
         "serial_p50_ms": round(p50_serial, 5),
         "speedup_vs_serial": round(p50_serial / p50, 4),
-        "schedule": {"slot_of": sched["slot_of"], "fell_back": sched["fell_back"],
+        "schedule": {"step3": args.sched, "slot_of": sched["slot_of"], "fell_back": sched["fell_back"],
                      "model_makespan_ns": sched["makespan"], "profile_t_ns": prof["t_ns"][:, 0].tolist(),
-                     "comm_alpha_same_ns": prof["comm"][0][0]},
+                     "comm_alpha_same_ns": prof["comm"][0][0],
+                     "measured_ns": getattr(duet_s, "measured_ns", None),
+                     "evaluations": getattr(duet_s, "evaluations", None),
+                     "model_mode_slot_of": model_s.export()["slot_of"],
+                     "model_mode_p50_ms": round(statistics.median(t_model), 5) if t_model else None},
         "e2e": {"value": round(world * wl.batch * args.steps / (e2e_ms / 1e3), 1), "unit": "samples/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "p50_ms": round(statistics.median(t_e2e), 5)},

@@ -73,7 +73,7 @@
 extern "C" {
 #endif
 
-#define DUET_ABI_VERSION 1
+#define DUET_ABI_VERSION 2
 #define DUET_HOST (-1)
 #define DUET_MAX_DIMS 8
 
@@ -142,11 +142,23 @@ typedef struct {
 typedef struct {
   int mode;              /* 0 greedy-correction, 1 greedy only (Steps 1-2),
                             2 serial on the home slot (operators-in-sequence),
-                            3 fixed assignment (tests / experiments)                        */
+                            3 fixed assignment (tests / experiments),
+                            the Fig. 13 baselines:
+                            4 random, 5 round-robin (slot = id mod D), 6 random + correction */
   int correction_rounds; /* x of "x round of swaps ... without decreasing"; 1 */
   int allow_fallback;    /* 1: best single slot if not slower            */
   const int32_t* fixed_slot_of; /* mode 3: slot per subgraph (length n_sg)                  */
+  uint32_t seed;         /* modes 4, 6: slot of s = h(seed, s) mod D, h = lowbias32 of
+                            (seed * 0x9E3779B1 + s) mod 2^32 (R-29)               */
 } duet_sched_opts;
+
+/* Measured-mode options (duet_schedule_measured). */
+typedef struct {
+  int samples;          /* timed replays per candidate assignment; latency = lower median; 20  */
+  int warmup;           /* untimed replays per candidate before timing; 3                      */
+  int64_t measured_ns;  /* OUT: measured latency of the returned assignment                     */
+  int32_t evaluations;  /* OUT: distinct assignments captured and timed                         */
+} duet_measure_opts;
 
 /* Thread-local message of the last failing call on this thread (valid until the next call). */
 const char* duet_last_error(void);
@@ -195,6 +207,18 @@ void duet_profile_destroy(duet_profile_t* pr);
 /* ---- schedule (PAPER.md:81, Algorithm 1; fallback PAPER.md:71, :90) ------------- */
 duet_status duet_schedule(const duet_partition_t* p, const duet_profile_t* pr, const duet_sched_opts* o,
                           duet_schedule_t** out);
+/* Measured mode (Algorithm 1's "measure latency"): the same
+ * Steps 1-2 (or random start) from the profile, then Step 3 and the fallback compare candidate
+ * assignments by their latency MEASURED on the device: each distinct assignment is captured as
+ * the duet_run executor graph over `slots` (device staging buffers filled with synthetic data,
+ * no host copies), replayed mo->warmup times, then mo->samples times between CUDA events on
+ * slots[0].stream; latency = lower median, int64 ns, memoised per assignment.  Synchronous
+ * (blocks the host).  Not deterministic: two calls may return different assignments.  Modes
+ * 1..5 have no Step 3 and only measure the fallback.  Requires bound parameters and slots on
+ * the parameters' GPU.  mo may be NULL (defaults; no OUT fields). */
+duet_status duet_schedule_measured(const duet_partition_t* p, const duet_profile_t* pr,
+                                   const duet_sched_opts* o, const duet_slot* slots, int n_slots,
+                                   duet_measure_opts* mo, duet_schedule_t** out);
 /* Any pointer may be NULL. sg_to_slot[n_sg]; order[n_sg] = global issue order pi (per-slot
  * order = pi filtered by slot); model makespan in ns. */
 duet_status duet_schedule_export(const duet_schedule_t* s, int32_t* sg_to_slot, int32_t* order,

@@ -255,9 +255,21 @@ def correct(m: Model, a, p, rounds: int = 1):
     return a
 
 
+def lowbias32(x: int) -> int:
+    """32-bit integer hash (the seeded random placement of the Fig. 13 baselines, R-29)."""
+    x &= 0xFFFFFFFF
+    x ^= x >> 16
+    x = (x * 0x7FEB352D) & 0xFFFFFFFF
+    x ^= x >> 15
+    x = (x * 0x846CA68B) & 0xFFFFFFFF
+    x ^= x >> 16
+    return x
+
+
 def schedule(part: Partition, T, slot_gpu, comm: Comm, mode: int = 0, correction_rounds: int = 1,
-             allow_fallback: bool = True, fixed=None) -> Schedule:
-    """mode 0 greedy-correction, 1 greedy only, 2 serial (home slot 0), 3 fixed."""
+             allow_fallback: bool = True, fixed=None, seed: int = 0) -> Schedule:
+    """mode 0 greedy-correction, 1 greedy only, 2 serial (home slot 0), 3 fixed; Fig. 13
+    baselines: 4 random, 5 round-robin, 6 random + correction."""
     m = Model(part, T, slot_gpu, comm)
     n = part.n_sg
     fell = 0
@@ -266,8 +278,13 @@ def schedule(part: Partition, T, slot_gpu, comm: Comm, mode: int = 0, correction
     elif mode == 3:
         a = [int(x) for x in fixed]
     else:
-        a = greedy(m)
-        if mode == 0:
+        if mode in (4, 6):
+            a = [lowbias32((seed * 0x9E3779B1 + s) & 0xFFFFFFFF) % m.D for s in range(n)]
+        elif mode == 5:
+            a = [s % m.D for s in range(n)]
+        else:
+            a = greedy(m)
+        if mode in (0, 6):
             for p in range(part.n_phase):
                 if part.phase_kind[p] == MULTI:
                     a = correct(m, a, p, correction_rounds)

@@ -212,6 +212,20 @@ duet_status duet_schedule(const duet_partition_t* p, const duet_profile_t* pr, c
   });
 }
 
+duet_status duet_schedule_measured(const duet_partition_t* p, const duet_profile_t* pr, const duet_sched_opts* o,
+                                   const duet_slot* slots, int n_slots, duet_measure_opts* mo, duet_schedule_t** out) {
+  if (out) *out = nullptr;
+  return guard([&] {
+    need(p, "partition");
+    need(pr, "profile");
+    need(slots, "slots");
+    need(out, "out");
+    std::unique_ptr<duet_schedule_t> h(new duet_schedule_t());
+    h->s.reset(schedule_measured(p->p.get(), pr->pr.get(), o, slots, n_slots, mo));
+    *out = h.release();
+  });
+}
+
 duet_status duet_schedule_export(const duet_schedule_t* s, int32_t* sg_to_slot, int32_t* order,
                                  int64_t* model_makespan_ns, int32_t* fell_back) {
   return guard([&] {

@@ -6,6 +6,7 @@
 #include <memory>
 #include <set>
 #include <string>
+#include <functional>
 #include <vector>
 
 #include "duet.h"
@@ -108,11 +109,21 @@ struct Schedule {
   std::vector<int> order;
   int64_t makespan = 0;
   int fell_back = 0;
+  int64_t measured_ns = -1;         // measured mode: device latency of slot_of (else -1)
   std::shared_ptr<ExecCache> exec;  // captured CUDA graphs (runtime.cu)
   ~Schedule();
 };
 
+// latency of a complete assignment (slot per subgraph), int64 ns
+using Latency = std::function<int64_t(const std::vector<int>&)>;
+
 Schedule* make_schedule(const Partition* p, const Profile* pr, const duet_sched_opts* o);
+// Same algorithm; Step 3's and the fallback's `measure latency` = `measured` when non-null.
+Schedule* make_schedule_with(const Partition* p, const Profile* pr, const duet_sched_opts* o,
+                             const Latency* measured);
+// Measured mode: times each candidate assignment on the device.
+Schedule* schedule_measured(const Partition* p, const Profile* pr, const duet_sched_opts* o,
+                            const duet_slot* slots, int n_slots, duet_measure_opts* mo);
 
 // ---- runtime (runtime.cu) ----
 Profile* profile_on_device(const Partition* p, const duet_slot* slots, int n_slots,

@@ -86,6 +86,10 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
     }
     ptx::fence_mbar_init();
   }
+  // wait for the previous kernel BEFORE taking tensor memory: a PDL-dependent CTA that holds TMEM
+  // while it waits can starve a co-resident kernel of another stream (observed as a hang with
+  // two slots)
+  ptx::pdl_wait();
   if (warp == 1) {
     ptx::tmem_alloc(tmem_slot, 2 * C::TMEM_COLS);
     ptx::tmem_relinquish();
@@ -94,7 +98,6 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
-  ptx::pdl_wait();
   ptx::pdl_trigger();
 
   if (warp == 0) {
@@ -223,7 +226,7 @@ void launch_conv_tma(const CUtensorMap& tx, const CUtensorMap& tw, const ConvArg
   int dev = 0;
   cudaGetDevice(&dev);
   const int grid = (int)std::min<int64_t>(tiles, num_sms(dev));
-  launch_pdl(kern, dim3(grid), dim3(192), C::SMEM, st, tx, tw, a);
+  launch_pdl_if(pdl_on(true), kern, dim3(grid), dim3(192), C::SMEM, st, tx, tw, a);
 }
 
 

@@ -72,6 +72,10 @@ __global__ void __launch_bounds__(192, 1)
     ptx::mbar_init(tmem_full, 1);
     ptx::fence_mbar_init();
   }
+  // wait for the previous kernel BEFORE taking tensor memory: a PDL-dependent CTA that holds TMEM
+  // while it waits can starve a co-resident kernel of another stream (observed as a hang with
+  // two slots)
+  ptx::pdl_wait();
   if (warp == 1) {
     ptx::tmem_alloc(tmem_slot, Cfg::TMEM_COLS);
     ptx::tmem_relinquish();
@@ -79,8 +83,7 @@ __global__ void __launch_bounds__(192, 1)
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
-  ptx::pdl_wait();     // A / gx / c_state / h_prev come from the previous kernel in the stream
+  const uint32_t tmem = *tmem_slot;     // A / gx / c_state / h_prev come from the previous kernel in the stream
   ptx::pdl_trigger();
 
   if (warp == 0) {
@@ -265,7 +268,7 @@ void launch_tc(const CUtensorMap& a, const CUtensorMap& w, const CUtensorMap& x,
     attr_done = true;
   }
   dim3 grid((N + BN - 1) / BN, (M + BM - 1) / BM);
-  launch_pdl(kern, grid, dim3(192), Cfg::SMEM, st, a, w, x, ep, M, N, K);
+  launch_pdl_if(pdl_on(true), kern, grid, dim3(192), Cfg::SMEM, st, a, w, x, ep, M, N, K);
 }
 
 // Fused recurrent weights: row r' = tile*BN + g*U + j' <-> (gate block g, unit j = tile*U + j');

@@ -72,6 +72,10 @@ __global__ void __launch_bounds__(192, 1)
     ptx::mbar_init(tmem_full, 1);
     ptx::fence_mbar_init();
   }
+  // wait for the previous kernel BEFORE taking tensor memory: a PDL-dependent CTA that holds TMEM
+  // while it waits can starve a co-resident kernel of another stream (observed as a hang with
+  // two slots)
+  ptx::pdl_wait();
   if (warp == 1) {
     ptx::tmem_alloc_2sm(tmem_slot, C::TMEM_COLS);
     ptx::tmem_relinquish_2sm();
@@ -80,7 +84,6 @@ __global__ void __launch_bounds__(192, 1)
   ptx::cluster_sync();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
-  ptx::pdl_wait();
   ptx::pdl_trigger();
 
   if (warp == 0) {
@@ -182,7 +185,7 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, i
   cfg.blockDim = dim3(192);
   cfg.dynamicSmemBytes = C::SMEM;
   cfg.stream = st;
-  static const bool no_pdl = getenv("DUET_NO_PDL") != nullptr;
+  const bool no_pdl = !pdl_on(true);
   cudaLaunchAttribute attr2[2];
   attr2[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr2[0].val.programmaticStreamSerializationAllowed = no_pdl ? 0 : 1;

@@ -119,20 +119,31 @@ int num_sms(int device);
 
 // Launch with the programmatic-stream-serialization attribute (PDL): the kernel must execute
 // griddepcontrol.wait before touching data produced by the preceding kernel in the stream.
+// PDL switches: DUET_NO_PDL (any value) disables it everywhere, DUET_PDL_TC=0 only for the
+// tcgen05 kernels (experiments).
+inline bool pdl_on(bool tc) {
+  static const bool off = getenv("DUET_NO_PDL") != nullptr;
+  static const bool tc_off = getenv("DUET_PDL_TC") && atoi(getenv("DUET_PDL_TC")) == 0;
+  return !off && !(tc && tc_off);
+}
 template <typename... KArgs, typename... Args>
-void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+void launch_pdl_if(bool on, void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                   Args&&... args) {
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = grid;
   cfg.blockDim = block;
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  static const bool no_pdl = getenv("DUET_NO_PDL") != nullptr;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = no_pdl ? 0 : 1;
+  cfg.numAttrs = on ? 1 : 0;
   CK(cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...));
+}
+template <typename... KArgs, typename... Args>
+void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+  launch_pdl_if(pdl_on(false), kern, grid, block, smem, st, std::forward<Args>(args)...);
 }
 // Same, without the PDL attribute: full stream serialization (used for kernels adjacent to
 // persistent / cluster kernels in the CNN chain, where early dependent launch was observed to hang

@@ -9,6 +9,7 @@
 //    (the sync queue), and a replay is a single cudaGraphLaunch on the home stream.
 //  * Profiler — PAPER.md:80 (§IV-B) / :87 (500 runs): each subgraph is captured alone and timed
 //    with CUDA events (samples of R replays; lower median, int64 ns).
+#include <chrono>
 #include <algorithm>
 #include <cstring>
 #include <functional>
@@ -692,9 +693,17 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
     throw;
   }
   CK(cudaStreamEndCapture(home, &E.graph));
+  static const bool log = getenv("DUET_MEASURE_LOG") != nullptr;
+  auto t_inst = std::chrono::steady_clock::now();
   // per-node priorities: kernels captured from a higher-priority slot stream keep it inside the
   // graph, so a latency-bound branch gets SMs first when a co-running branch's CTAs retire
   CK(cudaGraphInstantiate(&E.exec, E.graph, cudaGraphInstantiateFlagUseNodePriority));
+  if (log) {
+    size_t nn = 0;
+    cudaGraphGetNodes(E.graph, nullptr, &nn);
+    fprintf(stderr, "[capture] %zu graph nodes, instantiate %.1f ms\n", nn,
+            std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_inst).count());
+  }
   *launches = nk;
   return E;
 }
@@ -766,6 +775,97 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
     hit = &S->exec->entries.back();
   }
   CK(cudaGraphLaunch(hit->exec, home));
+}
+
+// ------------------------------------------------------------------------------------------------
+// Measured correction: Algorithm 1's `measure latency` on the device
+// ------------------------------------------------------------------------------------------------
+namespace {
+void fill_inputs(const Program& P, cudaStream_t st);
+int64_t lower_median(std::vector<double> v);
+}  // namespace
+
+Schedule* schedule_measured(const Partition* p, const Profile* pr, const duet_sched_opts* o, const duet_slot* slots,
+                            int n_slots, duet_measure_opts* mo) {
+  Graph* g = const_cast<Graph*>(p->g);
+  auto P = ensure_program(g);
+  if (n_slots != pr->n_slots) fail(DUET_EINVAL, "n_slots differs from the profile's slot count");
+  duet_measure_opts opts{20, 3, 0, 0};
+  if (mo) opts.samples = mo->samples, opts.warmup = mo->warmup;
+  if (opts.samples < 1 || opts.warmup < 0) fail(DUET_EINVAL, "bad measure options");
+  std::vector<cudaStream_t> streams;
+  for (int d = 0; d < n_slots; ++d) {
+    if (slots[d].gpu != P->device) fail(DUET_EUNSUPPORTED, "measured mode: every slot must be on the graph's GPU");
+    if (!slots[d].stream) fail(DUET_EINVAL, "slot stream is NULL (the legacy default stream cannot be captured)");
+    streams.push_back((cudaStream_t)slots[d].stream);
+  }
+  DeviceGuard dg(P->device);
+  cudaStream_t home = streams[0];
+  fill_inputs(*P, home);
+  for (int s = 0; s < p->n_sg(); ++s) launch_subgraph(*P, *p, s, P->buf, home);  // real data everywhere
+  CK(cudaStreamSynchronize(home));
+  std::vector<cudaEvent_t> ev(opts.samples + 1);
+  for (auto& e : ev) CK(cudaEventCreate(&e));
+  std::map<std::vector<int>, int64_t> memo;
+  static const bool log = getenv("DUET_MEASURE_LOG") != nullptr;
+  const Latency lat = [&](const std::vector<int>& a) -> int64_t {
+    auto it = memo.find(a);
+    if (it != memo.end()) return it->second;
+    auto h0 = std::chrono::steady_clock::now();
+    Schedule S;
+    S.p = p;
+    S.pr = pr;
+    S.slot_of = a;
+    for (int s = 0; s < p->n_sg(); ++s) S.order.push_back(s);
+    int64_t nk = 0;
+    ExecEntry E = capture(*P, S, streams, P->buf, {}, {}, &nk);
+    auto h1 = std::chrono::steady_clock::now();
+    std::vector<double> ns;
+    try {
+      for (int w = 0; w < opts.warmup; ++w) CK(cudaGraphLaunch(E.exec, home));
+      CK(cudaEventRecord(ev[0], home));
+      for (int k = 0; k < opts.samples; ++k) {
+        CK(cudaGraphLaunch(E.exec, home));
+        CK(cudaEventRecord(ev[k + 1], home));
+      }
+      CK(cudaStreamSynchronize(home));
+      for (int k = 0; k < opts.samples; ++k) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, ev[k], ev[k + 1]));
+        ns.push_back(ms * 1e6);
+      }
+    } catch (...) {
+      cudaGraphExecDestroy(E.exec);
+      cudaGraphDestroy(E.graph);
+      for (auto e : E.events) cudaEventDestroy(e);
+      throw;
+    }
+    cudaGraphExecDestroy(E.exec);
+    cudaGraphDestroy(E.graph);
+    for (auto e : E.events) cudaEventDestroy(e);
+    int64_t t = lower_median(ns);
+    memo[a] = t;
+    if (log) {
+      auto h2 = std::chrono::steady_clock::now();
+      fprintf(stderr, "[measure] #%zu capture+instantiate %.1f ms, timing %.1f ms, latency %lld ns, %lld kernels\n",
+              memo.size(), std::chrono::duration<double, std::milli>(h1 - h0).count(),
+              std::chrono::duration<double, std::milli>(h2 - h1).count(), (long long)t, (long long)nk);
+    }
+    return t;
+  };
+  Schedule* S = nullptr;
+  try {
+    S = make_schedule_with(p, pr, o, &lat);
+  } catch (...) {
+    for (auto e : ev) cudaEventDestroy(e);
+    throw;
+  }
+  for (auto e : ev) cudaEventDestroy(e);
+  if (mo) {
+    mo->measured_ns = S->measured_ns;
+    mo->evaluations = (int32_t)memo.size();
+  }
+  return S;
 }
 
 int64_t schedule_launch_count(const Schedule* s) {

@@ -210,8 +210,10 @@ std::vector<int> greedy(const Model& m) {
   return a;
 }
 
-void correct(const Model& m, std::vector<int>& a, int ph, int rounds) {
-  int64_t t_old = m.makespan(a);
+// `lat` is Algorithm 1's `measure latency`: the C3 model (model mode) or a device measurement of
+// the whole assignment (measured mode); tie-breaks are the same in both.
+void correct(const Model& m, std::vector<int>& a, int ph, int rounds, const Latency& lat) {
+  int64_t t_old = lat(a);
   const auto& P = m.phases[ph];
   int idle = 0;
   while (true) {
@@ -226,7 +228,7 @@ void correct(const Model& m, std::vector<int>& a, int ph, int rounds) {
           if (d == a[i]) continue;
           b = a;
           b[i] = d;
-          auto key = std::make_tuple(m.makespan(b), 0, i, d);
+          auto key = std::make_tuple(lat(b), 0, i, d);
           if (!have || key < best) best = key, have = true;
         }
       for (size_t x = 0; x < U.size(); ++x)
@@ -235,7 +237,7 @@ void correct(const Model& m, std::vector<int>& a, int ph, int rounds) {
           if (a[i] == a[j]) continue;
           b = a;
           std::swap(b[i], b[j]);
-          auto key = std::make_tuple(m.makespan(b), 1, i, j);
+          auto key = std::make_tuple(lat(b), 1, i, j);
           if (!have || key < best) best = key, have = true;
         }
       if (!have) break;
@@ -259,16 +261,27 @@ void correct(const Model& m, std::vector<int>& a, int ph, int rounds) {
   }
 }
 
+uint32_t lowbias32(uint32_t x) {
+  x ^= x >> 16;
+  x *= 0x7feb352du;
+  x ^= x >> 15;
+  x *= 0x846ca68bu;
+  x ^= x >> 16;
+  return x;
+}
+
 }  // namespace
 
-Schedule* make_schedule(const Partition* p, const Profile* pr, const duet_sched_opts* o) {
+Schedule* make_schedule_with(const Partition* p, const Profile* pr, const duet_sched_opts* o, const Latency* measured) {
   if (pr->p != p) fail(DUET_EINVAL, "profile belongs to another partition");
-  duet_sched_opts opts{0, 1, 1, nullptr};
+  duet_sched_opts opts{0, 1, 1, nullptr, 0};
   if (o) opts = *o;
-  if (opts.mode < 0 || opts.mode > 3) fail(DUET_EINVAL, "mode must be 0..3");
+  if (opts.mode < 0 || opts.mode > 6) fail(DUET_EINVAL, "mode must be 0..6");
   if (opts.correction_rounds < 1) fail(DUET_EINVAL, "correction_rounds must be >= 1");
   Model m(p, pr);
   if (m.D < 1) fail(DUET_EINVAL, "no slots");
+  const Latency model = [&](const std::vector<int>& b) { return m.makespan(b); };
+  const Latency& lat = measured ? *measured : model;
   std::unique_ptr<Schedule> S(new Schedule());
   S->p = p;
   S->pr = pr;
@@ -283,16 +296,22 @@ Schedule* make_schedule(const Partition* p, const Profile* pr, const duet_sched_
       a.push_back(d);
     }
   } else {
-    a = greedy(m);
-    if (opts.mode == 0)
+    if (opts.mode == 4 || opts.mode == 6) {
+      for (int s = 0; s < m.n; ++s) a.push_back((int)(lowbias32(opts.seed * 0x9E3779B1u + (uint32_t)s) % (uint32_t)m.D));
+    } else if (opts.mode == 5) {
+      for (int s = 0; s < m.n; ++s) a.push_back(s % m.D);
+    } else {
+      a = greedy(m);
+    }
+    if (opts.mode == 0 || opts.mode == 6)
       for (int ph = 0; ph < (int)m.phases.size(); ++ph)
-        if (p->phase_kind[ph] == kMulti) correct(m, a, ph, opts.correction_rounds);
+        if (p->phase_kind[ph] == kMulti) correct(m, a, ph, opts.correction_rounds, lat);
     if (opts.allow_fallback) {
-      int64_t m_gc = m.makespan(a);
+      int64_t m_gc = lat(a);
       int64_t best = -1;
       int bd = 0;
       for (int d = 0; d < m.D; ++d) {
-        int64_t v = m.makespan(std::vector<int>(m.n, d));
+        int64_t v = lat(std::vector<int>(m.n, d));
         if (best < 0 || v < best) best = v, bd = d;
       }
       if (best <= m_gc) {
@@ -304,7 +323,12 @@ Schedule* make_schedule(const Partition* p, const Profile* pr, const duet_sched_
   S->slot_of = a;
   for (int s = 0; s < m.n; ++s) S->order.push_back(s);
   S->makespan = m.makespan(a);
+  if (measured) S->measured_ns = lat(a);
   return S.release();
+}
+
+Schedule* make_schedule(const Partition* p, const Profile* pr, const duet_sched_opts* o) {
+  return make_schedule_with(p, pr, o, nullptr);
 }
 
 }  // namespace duet

@@ -24,7 +24,7 @@ _lib = C.CDLL(LIB_PATH)
 MAX_DIMS = 8
 HOST = -1
 F32, BF16, I32, I64 = 0, 1, 2, 3
-GREEDY_CORRECTION, GREEDY_ONLY, SERIAL, FIXED = 0, 1, 2, 3
+GREEDY_CORRECTION, GREEDY_ONLY, SERIAL, FIXED, RANDOM, ROUND_ROBIN, RANDOM_CORRECTION = 0, 1, 2, 3, 4, 5, 6
 STATUS = {0: "OK", -1: "EINVAL", -2: "EPARSE", -3: "ECYCLE", -4: "ESHAPE", -5: "EDTYPE", -6: "EUNBOUND",
           -7: "ECUDA", -8: "ENCCL", -9: "ENOMEM", -10: "EUNSUPPORTED", -11: "ESTATE"}
 
@@ -62,9 +62,13 @@ class ProfileOpts(C.Structure):
                 ("calibrate_comm", C.c_int)]
 
 
+class MeasureOpts(C.Structure):
+    _fields_ = [("samples", C.c_int), ("warmup", C.c_int), ("measured_ns", C.c_int64), ("evaluations", C.c_int32)]
+
+
 class SchedOpts(C.Structure):
     _fields_ = [("mode", C.c_int), ("correction_rounds", C.c_int), ("allow_fallback", C.c_int),
-                ("fixed_slot_of", C.POINTER(C.c_int32))]
+                ("fixed_slot_of", C.POINTER(C.c_int32)), ("seed", C.c_uint32)]
 
 
 _P = C.c_void_p
@@ -87,6 +91,8 @@ _sig = {
                                       C.POINTER(C.c_int32)]),
     "duet_profile_destroy": (None, [_P]),
     "duet_schedule": (C.c_int, [_P, _P, C.POINTER(SchedOpts), C.POINTER(_P)]),
+    "duet_schedule_measured": (C.c_int, [_P, _P, C.POINTER(SchedOpts), C.POINTER(Slot), C.c_int,
+                                         C.POINTER(MeasureOpts), C.POINTER(_P)]),
     "duet_schedule_export": (C.c_int, [_P, C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.POINTER(C.c_int64),
                                        C.POINTER(C.c_int32)]),
     "duet_schedule_destroy": (None, [_P]),
@@ -275,14 +281,30 @@ class Profile:
                 "comm": ((cm.same_gpu.alpha_ns, cm.same_gpu.ps_per_byte),
                          (cm.cross_gpu.alpha_ns, cm.cross_gpu.ps_per_byte))}
 
-    def schedule(self, mode=GREEDY_CORRECTION, correction_rounds=1, allow_fallback=True, fixed=None) -> "Schedule":
+    def schedule(self, mode=GREEDY_CORRECTION, correction_rounds=1, allow_fallback=True, fixed=None,
+                 seed=0) -> "Schedule":
         fx = None
         if fixed is not None:
             fx = np.ascontiguousarray(fixed, dtype=np.int32)
-        o = SchedOpts(mode, correction_rounds, int(allow_fallback), _np_ptr(fx, C.c_int32) if fx is not None else None)
+        o = SchedOpts(mode, correction_rounds, int(allow_fallback), _np_ptr(fx, C.c_int32) if fx is not None else None,
+                      seed)
         h = _P()
         _check(_lib.duet_schedule(self.part._h, self._h, C.byref(o), C.byref(h)))
         return Schedule(h, self)
+
+    def schedule_measured(self, slots, mode=GREEDY_CORRECTION, correction_rounds=1, allow_fallback=True,
+                          seed=0, samples=20, warmup=3) -> "Schedule":
+        """Measured-mode Step 3 (duet_schedule_measured): candidates timed on the device over
+        `slots`.  The returned Schedule carries .measured_ns and .evaluations."""
+        o = SchedOpts(mode, correction_rounds, int(allow_fallback), None, seed)
+        mo = MeasureOpts(samples, warmup, 0, 0)
+        sa = make_slots(slots)
+        h = _P()
+        _check(_lib.duet_schedule_measured(self.part._h, self._h, C.byref(o), sa, len(slots), C.byref(mo),
+                                           C.byref(h)))
+        s = Schedule(h, self)
+        s.measured_ns, s.evaluations = mo.measured_ns, mo.evaluations
+        return s
 
 
 class Schedule:

@@ -35,10 +35,16 @@ class Session:
             self.prof = self.part.profile(self.slots, **(profile or {}))
         self.schedules = {}
 
-    def schedule(self, mode=duet.GREEDY_CORRECTION, **kw) -> duet.Schedule:
-        key = (mode, tuple(sorted(kw.items())))
+    def schedule(self, mode=duet.GREEDY_CORRECTION, measured=False, **kw) -> duet.Schedule:
+        """measured=True: Step 3 / fallback compare assignments by device-measured latency over
+        this session's slots (duet_schedule_measured); else by the profile's makespan model."""
+        key = (mode, measured, tuple(sorted(kw.items())))
         if key not in self.schedules:
-            self.schedules[key] = self.prof.schedule(mode=mode, **kw)
+            if measured:
+                torch.cuda.current_stream(self.device).synchronize()
+                self.schedules[key] = self.prof.schedule_measured(self.slots, mode=mode, **kw)
+            else:
+                self.schedules[key] = self.prof.schedule(mode=mode, **kw)
         return self.schedules[key]
 
     def outputs(self, device=True):

@@ -26,7 +26,7 @@ def test_exports_every_declared_symbol():
     for name in declared:
         assert hasattr(lib, name), name
     assert set(duet.EXPORTED) == declared
-    assert duet.abi_version() == 1
+    assert duet.abi_version() == 2
 
 
 @pytest.mark.parametrize("ir,code", [
@@ -105,11 +105,12 @@ def test_partition_and_schedule_bit_exact_fuzz(seed):
     part = duet.Graph(ir).partition(gran)
     prof = part.profile_from_table(slot_gpu, T, comm)
     oc = Comm(Link(*comm[0]), Link(*comm[1]))
-    for mode in (0, 1, 2):
-        for rounds in ((1, 2) if mode == 0 else (1,)):
+    for mode in (0, 1, 2, 4, 5, 6):
+        for rounds in ((1, 2) if mode in (0, 6) else (1,)):
             for fb in (True, False):
-                s = prof.schedule(mode=mode, correction_rounds=rounds, allow_fallback=fb).export()
-                os_ = o_schedule(o, T, slot_gpu, oc, mode=mode, correction_rounds=rounds, allow_fallback=fb)
+                s = prof.schedule(mode=mode, correction_rounds=rounds, allow_fallback=fb, seed=seed).export()
+                os_ = o_schedule(o, T, slot_gpu, oc, mode=mode, correction_rounds=rounds, allow_fallback=fb,
+                                 seed=seed)
                 assert s["slot_of"] == os_.slot_of, (mode, rounds, fb)
                 assert s["makespan"] == os_.makespan
                 assert s["fell_back"] == os_.fell_back

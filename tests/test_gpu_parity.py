@@ -226,3 +226,29 @@ def test_rnn_node(kind, S, B, E, H, dt):
     err = rel_err(y.float().cpu().numpy(), want)
     print(f"[parity] {kind} S{S} B{B} E{E} H{H} {dt}: rel err {err:.3e}")
     assert err <= TOL[dt], err
+
+
+@pytest.mark.parametrize("cfg,mode", [("c5", duet.GREEDY_CORRECTION), ("c5", duet.RANDOM_CORRECTION),
+                                      ("c3", duet.GREEDY_CORRECTION)])
+def test_measured_correction(cfg, mode):
+    """Step 3 with device-measured latency returns a valid assignment whose
+    outputs equal the serial schedule's bit for bit and still meet the oracle bar."""
+    wl = W.build(cfg, small=True, dt="bf16")
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    s = sess.schedule(mode, measured=True, samples=5, warmup=1, seed=3)
+    e = s.export()
+    assert len(e["slot_of"]) == sess.part.n_sg and all(0 <= d < 2 for d in e["slot_of"])
+    assert s.measured_ns > 0 and s.evaluations >= 1
+    if mode == duet.RANDOM_CORRECTION and not e["fell_back"]:
+        assert s.evaluations >= 2
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    want = _oracle_outputs(wl, sess.params, dict(zip(wl.inputs, inputs)))
+    got = {}
+    for key, sch in (("measured", s), ("serial", sess.schedule(duet.SERIAL))):
+        outs = sess.outputs()
+        sess.run(sch, inputs, outs)
+        torch.cuda.synchronize()
+        got[key] = [o.float().cpu().numpy() for o in outs]
+    for (name, _, _), y, z in zip(wl.outputs, got["measured"], got["serial"]):
+        np.testing.assert_array_equal(y, z)
+        assert rel_err(y, want[name]) <= TOL["bf16"]

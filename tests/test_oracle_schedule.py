@@ -233,3 +233,23 @@ def test_gc_near_optimal_on_paper_like_fixtures():
             total += 1
             worst = max(worst, s.makespan / opt)
     assert hits / total >= 0.8 and worst < 1.25, (hits, total, worst)
+
+
+def test_fig13_baselines_definitions():
+    """PAPER.md:88 Fig. 13 schemes: round-robin alternates by id; random is the seeded hash; the
+    correction step never makes a random start worse; greedy+correction <= its greedy start."""
+    from oracle.schedule import lowbias32
+    assert lowbias32(0) == 0 and lowbias32(1) != 1
+    p = partition(branches_ir(6, join=True))
+    T = [[(i + 2) * 1000, (7 - i) * 1000] for i in range(7)]
+    rr = schedule(p, T, [0, 1], ZERO, mode=5, allow_fallback=False)
+    assert rr.slot_of == [i % 2 for i in range(7)]
+    for seed in range(10):
+        rnd = schedule(p, T, [0, 1], ZERO, mode=4, allow_fallback=False, seed=seed)
+        assert rnd.slot_of == [lowbias32((seed * 0x9E3779B1 + s) & 0xFFFFFFFF) % 2 for s in range(7)]
+        rc = schedule(p, T, [0, 1], ZERO, mode=6, allow_fallback=False, seed=seed)
+        assert rc.makespan <= rnd.makespan
+    g = schedule(p, T, [0, 1], ZERO, mode=1, allow_fallback=False)
+    gc = schedule(p, T, [0, 1], ZERO, mode=0, allow_fallback=False)
+    assert gc.makespan <= g.makespan
+    assert gc.makespan >= brute_force(p, T, [0, 1], ZERO)[0]
