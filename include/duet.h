@@ -230,8 +230,12 @@ void duet_schedule_destroy(duet_schedule_t* s);
  * home stream after the producers of the inputs (e.g. an event wait) and reads the outputs after
  * the home stream reaches this point.  inputs[] follow the IR's input nodes in declaration order,
  * outputs[] the IR's output nodes in declaration order.  Device tensors are
- * used in place; HOST tensors are copied H2D before / D2H after the graph on the home stream
- * (pinned memory keeps this asynchronous).  Slot streams other than the home stream only shape
+ * used in place.  HOST tensors must be pinned (page-locked; else DUET_EINVAL).  A host input
+ * whose only consumer reads it once, coalesced (hash_mod, the ids of gather_sum / gather_concat),
+ * is read by that kernel directly over PCIe (zero-copy); a host output no node consumes, produced
+ * by a join / reduce_sum / gather_sum, is stored directly into host memory; other host tensors
+ * are copied H2D before / D2H after the graph on the home stream (DUET_ZERO_COPY=0: always copy).
+ * Host buffers must stay untouched until the home stream passes this call.  Slot streams other than the home stream only shape
  * the captured CUDA graph (one graph per distinct (slots, tensor pointers) — cached). */
 duet_status duet_run(duet_schedule_t* s, const duet_slot* slots, int n_slots, const duet_tensor* inputs,
                      int n_in, duet_tensor* outputs, int n_out);

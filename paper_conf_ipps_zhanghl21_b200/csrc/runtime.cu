@@ -708,6 +708,58 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
   return E;
 }
 
+// ---- zero-copy host I/O (duet_run with pinned HOST tensors) ----------------------------------
+// A pinned host buffer is device-addressable (UVA).  An input whose single consumer reads it once,
+// coalesced (hashing, the id reads of the gathers), is read by that kernel over PCIe: no copy
+// engine round trip, and the transfer overlaps the kernel's own work.  An output nobody in the
+// graph reads, produced by a plain-store kernel (the joins), is stored straight into host memory.
+// Everything else (pageable memory, several consumers, strided / re-read access such as token
+// ids or conv images) keeps the memcpy nodes.  DUET_ZERO_COPY=0 disables both.
+static bool zero_copy_enabled() {
+  static const bool on = !(getenv("DUET_ZERO_COPY") && atoi(getenv("DUET_ZERO_COPY")) == 0);
+  return on;
+}
+
+static void* mapped_host_ptr(const void* p) {
+  cudaPointerAttributes a{};
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  if (a.type != cudaMemoryTypeHost || !a.devicePointer) return nullptr;
+  return a.devicePointer;
+}
+
+static void* direct_input_ptr(const Graph& g, const Node& in, const void* host) {
+  if (!zero_copy_enabled()) return nullptr;
+  const Node* consumer = nullptr;
+  int uses = 0;
+  for (const Node& c : g.nodes)
+    for (int a : c.arg_nodes)
+      if (a == in.id) ++uses, consumer = &c;
+  for (int o : g.outputs)
+    if (o == in.id) return nullptr;
+  if (uses != 1) return nullptr;
+  const std::string& op = consumer->op;
+  if (op != "hash_mod" && op != "gather_sum" && op != "gather_concat") return nullptr;
+  return mapped_host_ptr(host);
+}
+
+static void* direct_output_ptr(const Graph& g, const Node& out, void* host) {
+  if (!zero_copy_enabled()) return nullptr;
+  for (const Node& c : g.nodes)
+    for (int a : c.arg_nodes)
+      if (a == out.id) return nullptr;
+  int listed = 0;
+  for (int o : g.outputs) listed += o == out.id;
+  if (listed != 1) return nullptr;
+  static const char* ok[] = {"dot_join", "cosine_join", "concat_head", "sum_join", "mean_join", "reduce_sum", "gather_sum"};
+  bool found = false;
+  for (auto* k : ok) found |= out.op == k;
+  if (!found) return nullptr;
+  return mapped_host_ptr(host);
+}
+
 void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_tensor* in, int n_in, duet_tensor* out,
                   int n_out) {
   const Graph* gc = S->p->g;
@@ -733,6 +785,10 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
     if (in[i].device >= 0) {
       if (in[i].device != P->device) fail(DUET_EUNSUPPORTED, "input on another GPU");
       T[nd.id] = in[i].data;
+    } else if (!mapped_host_ptr(in[i].data)) {
+      fail(DUET_EINVAL, "input " + nd.name + ": host tensors must be pinned (page-locked) memory");
+    } else if (void* dp = direct_input_ptr(*g, nd, in[i].data)) {
+      T[nd.id] = dp;  // zero-copy: its only consumer streams it once over PCIe
     } else {
       h2d.push_back({P->buf[nd.id], in[i].data, (size_t)nd.nbytes(), cudaMemcpyHostToDevice});
     }
@@ -743,6 +799,10 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
     if (out[i].device >= 0) {
       if (out[i].device != P->device) fail(DUET_EUNSUPPORTED, "output on another GPU");
       T[nd.id] = out[i].data;
+    } else if (!mapped_host_ptr(out[i].data)) {
+      fail(DUET_EINVAL, "output " + nd.name + ": host tensors must be pinned (page-locked) memory");
+    } else if (void* dp = direct_output_ptr(*g, nd, out[i].data)) {
+      T[nd.id] = dp;  // zero-copy: the producing kernel stores straight into pinned host memory
     } else {
       d2h.push_back({out[i].data, P->buf[nd.id], (size_t)nd.nbytes(), cudaMemcpyDeviceToHost});
     }
