@@ -334,6 +334,21 @@ CUtensorMap make_tmap_bf16_2d(const void* base, int64_t rows, int64_t cols, int 
   return m;
 }
 
+bool make_tmap_store_2d(CUtensorMap* m, void* base, int eb, int64_t rows, int64_t cols, int64_t ld, int span_bytes) {
+  if (((uintptr_t)base & 15) || (ld * eb) % 16 || cols * eb < span_bytes || rows < 32) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(ld * eb)};
+  cuuint32_t box[2] = {(cuuint32_t)(span_bytes / eb), 32};
+  cuuint32_t estr[2] = {1, 1};
+  const CUtensorMapSwizzle sw = span_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                : span_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                   : CU_TENSOR_MAP_SWIZZLE_32B;
+  CUresult r = get_encode()(m, eb == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, base,
+                            dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+                            CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
 int tc_pick_bn(int M, int N, int num_sms) {
   // Smallest-waste tile width that still fills the SMs: prefer the widest BN whose tile count
   // reaches the SM count; else the narrowest (most CTAs).

@@ -15,9 +15,22 @@
 
 namespace duet {
 
+// Phase timestamps per CTA for the micro-benchmarks (ep.dbg & 32): %globaltimer ns at
+// 0 entry, 1 after prologue, 2 first TMA issued, 3 first stage landed (MMA thread),
+// 4 last MMA commit issued, 5 accumulator ready (epilogue), 6 epilogue stores done, 7 exit.
+__device__ unsigned long long g_tc2_trace[8 * 4096];
+
 namespace {
 
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
 constexpr int BM2 = 128;  // rows per CTA (256 per pair)
+constexpr int kEpiThreads2 = 256;           // 8 epilogue warps
+constexpr int kThreads2 = 64 + kEpiThreads2;  // + TMA producer warp + MMA warp
 constexpr int BK2 = 64;   // one SWIZZLE_128B atom of K
 constexpr int KB2 = 2;    // k-blocks per pipeline stage: halves barrier round trips per FLOP
 constexpr int A2_ATOM = BM2 * BK2 * 2;
@@ -38,9 +51,9 @@ struct Cfg2 {
 // multicasts it to pair 1 (halves A's L2->SMEM traffic).  MMA commits go to all 4 CTAs so a
 // stage is refilled only after both pairs consumed it (empty barrier count 2).
 template <int BN, typename OutT, int MC>
-__global__ void __launch_bounds__(192, 1)
+__global__ void __launch_bounds__(kThreads2, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
-                 const TcEpilogue ep, int M, int N, int K) {
+                 const __grid_constant__ CUtensorMap tmO, const TcEpilogue ep, int M, int N, int K) {
   using C = Cfg2<BN>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -54,6 +67,9 @@ __global__ void __launch_bounds__(192, 1)
 
   const int warp = ptx::warp_id();
   const int lane = threadIdx.x & 31;
+  const bool tr = (ep.dbg & 32) != 0;
+  unsigned long long* trace = g_tc2_trace + 8 * ((blockIdx.y * gridDim.x + blockIdx.x) & 4095);
+  if (tr && threadIdx.x == 0) trace[0] = gtimer();
   const uint32_t crank = ptx::cluster_ctarank();
   const uint32_t rank = crank & 1;          // rank within the CTA pair
   const int pair = MC ? (int)(crank >> 1) : 0;
@@ -61,6 +77,7 @@ __global__ void __launch_bounds__(192, 1)
   const int n0 = tile_n * BN;
   const int m0 = blockIdx.y * (2 * BM2) + (int)rank * BM2;  // this CTA's rows
   const int nk = (K + KB2 * BK2 - 1) / (KB2 * BK2);  // stages of KB2 k-blocks
+  const int npre = nk < C::STAGES ? nk : C::STAGES;  // stages whose W tiles load before the PDL wait
 
   if (warp == 0 && lane == 0) {
     ptx::tma_prefetch(&tmA);
@@ -72,6 +89,22 @@ __global__ void __launch_bounds__(192, 1)
     ptx::mbar_init(tmem_full, 1);
     ptx::fence_mbar_init();
   }
+  // barrier init visible to the peer CTA before any TMA completes on the leader's barriers
+  ptx::cluster_sync();
+  const uint32_t full_leader0 = ptx::mapa(ptx::smem_u32(&full[0]), crank & ~1u);
+  if (warp == 0 && lane == 0 && !(ep.dbg & 2)) {
+    // weights are graph parameters, never written by the previous kernel: their first stages
+    // stream in while the previous kernel drains (programmatic dependent launch)
+    for (int kb = 0; kb < npre; ++kb) {
+      const uint32_t fb = full_leader0 + kb * 8;
+      if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
+      if (tr && kb == 0) trace[2] = gtimer();
+#pragma unroll
+      for (int h = 0; h < KB2; ++h)
+        ptx::tma_load_2d_2sm(&tmW, fb, sB + kb * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
+                             n0 + (int)rank * C::BH);
+    }
+  }
   // wait for the previous kernel BEFORE taking tensor memory: a PDL-dependent CTA that holds TMEM
   // while it waits can starve a co-resident kernel of another stream (observed as a hang with
   // two slots)
@@ -81,33 +114,37 @@ __global__ void __launch_bounds__(192, 1)
     ptx::tmem_relinquish_2sm();
   }
   ptx::tc_fence_before();
-  ptx::cluster_sync();
+  // A loads (below) follow this CTA's alloc, so the leader's first full barrier implies both CTAs'
+  // TMEM is allocated before the first MMA.  With multicast, pair 1 receives A from pair 0, so
+  // the whole cluster synchronises instead.
+  if constexpr (MC) ptx::cluster_sync(); else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  if (tr && threadIdx.x == 0) trace[1] = gtimer();
   ptx::pdl_trigger();
 
   if (warp == 0) {
     if (lane == 0) {
-      // full barriers live in each pair's leader CTA; both CTAs' copies complete there
-      const uint32_t full_leader0 = ptx::mapa(ptx::smem_u32(&full[0]), crank & ~1u);
       const uint16_t a_mask = (uint16_t)(0x5u << rank);  // CTA r of pair 0 and of pair 1
       for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % C::STAGES;
+        const bool pre = kb < npre && !(ep.dbg & 2);
         if (kb >= C::STAGES) ptx::mbar_wait(&empty[s], ((kb / C::STAGES) - 1) & 1);
         const uint32_t fb = full_leader0 + s * 8;
         if (ep.dbg & 2) {
           if (rank == 0) ptx::mbar_arrive(&full[s]);
           continue;
         }
-        if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
+        if (!pre && rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
 #pragma unroll
         for (int h = 0; h < KB2; ++h) {
           if (!MC)
             ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
           else if (pair == 0)
             ptx::tma_load_2d_2sm_mc(&tmA, &full[s], sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0, a_mask);
-          ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
-                               n0 + (int)rank * C::BH);
+          if (!pre)
+            ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
+                                 n0 + (int)rank * C::BH);
         }
       }
     }
@@ -120,6 +157,7 @@ __global__ void __launch_bounds__(192, 1)
         const int s = kb % C::STAGES;
         ptx::mbar_wait(&full[s], (kb / C::STAGES) & 1);
         ptx::tc_fence_after();
+        if (tr && kb == 0) trace[3] = gtimer();
 #pragma unroll
         for (int h = 0; h < KB2; ++h) {
           const uint32_t a_base = ptx::smem_u32(sA + s * A2_BYTES + h * A2_ATOM);
@@ -133,35 +171,105 @@ __global__ void __launch_bounds__(192, 1)
         ptx::umma_commit_2sm(&empty[s], empty_mask);
       }
       ptx::umma_commit_2sm(tmem_full, pair_mask);
+      if (tr) trace[4] = gtimer();
     }
   } else {
-    // epilogue warps 2..5: stage this tile's bias in smem while the mainloop runs
-    const int et = threadIdx.x - 64;
-    for (int c = et; c < BN; c += 128) s_bias[c] = (ep.bias && n0 + c < N) ? ep.bias[n0 + c] : 0.0f;
-    asm volatile("bar.sync 1, 128;" ::: "memory");
+    // epilogue warps 2..9: warp w reads TMEM lanes 32 (w % 4) .. +32 (hardware lane-quarter
+    // rule); the two warps of a quarter split the columns.  Bias of this tile -> smem first
+    // (overlaps the mainloop).
+    for (int c = threadIdx.x - 64; c < BN; c += kEpiThreads2) s_bias[c] = (ep.bias && n0 + c < N) ? ep.bias[n0 + c] : 0.0f;
+    asm volatile("bar.sync 1, %0;" ::"n"(kEpiThreads2) : "memory");
     const int q = warp & 3;
+    const int half = (warp - 2) >> 2;
     const int row = m0 + q * 32 + lane;
     ptx::mbar_wait(tmem_full, 0);
     ptx::tc_fence_after();
+    if (tr && warp == 2 && lane == 0) trace[5] = gtimer();
     const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
-    OutT* out = reinterpret_cast<OutT*>(ep.out) + (size_t)row * ep.ldo;
     const int act = ep.act;
+    constexpr int EB = (int)sizeof(OutT);
+    // columns per TMEM round trip = one swizzle span (<= 128 B) of output
+    constexpr int CW = (BN / 2) * EB < 128 ? BN / 2 : 128 / EB;
+    if (ep.tma_store && !(ep.dbg & 8)) {
+      // Stage the warp's 32 x CW sub-tile in swizzled smem (the A stages are idle once the
+      // accumulator is complete) and let TMA write whole lines: a direct st.global from this
+      // layout touches 32 rows per instruction.
+      constexpr int SPAN = CW * EB;  // bytes per staged row: 128, 64 or 32
+      constexpr int SW_SHIFT = SPAN == 128 ? 0 : SPAN == 64 ? 1 : 2;  // row bits feeding the XOR
+      constexpr int SW_MASK = SPAN / 16 - 1;
+      uint8_t* stage_base = sA + (warp - 2) * (2 * 32 * SPAN);
+      int buf = 0;
 #pragma unroll 1
-    for (int c = 0; c < BN / 16; ++c) {
-      if (ep.dbg & 8) break;
-      float v[16];
-      ptx::tmem_ld16(tq + c * 16, v);
-      if (ep.dbg & 16) continue;
-      const int col0 = n0 + c * 16;
-      if (row < M && col0 < N) {
+      for (int c0 = half * (BN / 2); c0 < (half + 1) * (BN / 2); c0 += CW, buf ^= 1) {
+        float v[CW];
+        if constexpr (CW == 64) {
+          ptx::tmem_ld64(tq + c0, v);
+        } else {
 #pragma unroll
-        for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i] + s_bias[c * 16 + i], act);
-        store_row16_any(out + col0, v, N - col0);
+          for (int j = 0; j < CW / 16; ++j) ptx::tmem_ld16(tq + c0 + 16 * j, v + 16 * j);
+        }
+#pragma unroll
+        for (int i = 0; i < CW; ++i) v[i] = apply_act(v[i] + s_bias[c0 + i], act);
+        uint8_t* st_row = stage_base + buf * (32 * SPAN) + lane * SPAN;
+        if (lane == 0) ptx::bulk_wait_read<1>();  // this buffer's previous store has read smem
+        __syncwarp();
+#pragma unroll
+        for (int u = 0; u < SPAN / 16; ++u) {
+          uint4 pk;
+          if constexpr (EB == 2) {
+            uint32_t w[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+              __nv_bfloat162 h2 = __floats2bfloat162_rn(v[u * 8 + 2 * t], v[u * 8 + 2 * t + 1]);
+              w[t] = *reinterpret_cast<uint32_t*>(&h2);
+            }
+            pk = make_uint4(w[0], w[1], w[2], w[3]);
+          } else {
+            pk = make_uint4(__float_as_uint(v[u * 4]), __float_as_uint(v[u * 4 + 1]), __float_as_uint(v[u * 4 + 2]),
+                            __float_as_uint(v[u * 4 + 3]));
+          }
+          const int slot = u ^ ((lane >> SW_SHIFT) & SW_MASK);
+          *reinterpret_cast<uint4*>(st_row + slot * 16) = pk;
+        }
+        ptx::fence_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          ptx::tma_store_2d(&tmO, stage_base + buf * (32 * SPAN), n0 + c0, m0 + q * 32);
+          ptx::bulk_commit();
+        }
+      }
+      if (lane == 0) ptx::bulk_wait_all();
+    } else {
+      OutT* out = reinterpret_cast<OutT*>(ep.out) + (size_t)row * ep.ldo;
+#pragma unroll 1
+      for (int c0 = half * (BN / 2); c0 < (half + 1) * (BN / 2); c0 += CW) {
+        if (ep.dbg & 8) break;
+        float v[CW];
+        if constexpr (CW == 64) {
+          ptx::tmem_ld64(tq + c0, v);
+        } else {
+#pragma unroll
+          for (int j = 0; j < CW / 16; ++j) ptx::tmem_ld16(tq + c0 + 16 * j, v + 16 * j);
+        }
+        if (ep.dbg & 16) continue;
+        if (row < M) {
+#pragma unroll
+          for (int j = 0; j < CW / 16; ++j) {
+            const int col0 = n0 + c0 + 16 * j;
+            if (col0 < N) {
+#pragma unroll
+              for (int i = 0; i < 16; ++i) v[16 * j + i] = apply_act(v[16 * j + i] + s_bias[c0 + 16 * j + i], act);
+              store_row16_any(out + col0, v + 16 * j, N - col0);
+            }
+          }
+        }
       }
     }
+    if (tr && warp == 2 && lane == 0) trace[6] = gtimer();
   }
   ptx::tc_fence_before();
   ptx::cluster_sync();
+  if (tr && threadIdx.x == 0) trace[7] = gtimer();
   if (warp == 1) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc_2sm(tmem, C::TMEM_COLS);
@@ -169,8 +277,16 @@ __global__ void __launch_bounds__(192, 1)
 }
 
 template <int BN, typename OutT, int MC>
-void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, int M, int N, int K, cudaStream_t st) {
+void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep_in, int M, int N, int K, cudaStream_t st) {
   using C = Cfg2<BN>;
+  static const bool no_tma_store = getenv("DUET_TMA_STORE") && atoi(getenv("DUET_TMA_STORE")) == 0;
+  TcEpilogue ep = ep_in;
+  CUtensorMap to{};
+  constexpr int EB = (int)sizeof(OutT);
+  constexpr int SPAN = (BN / 2) * EB < 128 ? (BN / 2) * EB : 128;
+  static_assert(2 * 32 * SPAN * 8 <= C::STAGES * A2_BYTES, "TMA-store staging must fit in the A stages");
+  ep.tma_store = !no_tma_store && !(ep.dbg & 8) && SPAN >= 32 &&
+                 make_tmap_store_2d(&to, ep.out, EB, M, N, ep.ldo, SPAN);
   auto kern = gemm2_kernel<BN, OutT, MC>;
   static bool attr = false;
   if (!attr) {
@@ -182,7 +298,7 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, i
   dim3 grid(MC ? 4 * ((tn + 1) / 2) : 2 * tn, (M + 2 * BM2 - 1) / (2 * BM2));
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = grid;
-  cfg.blockDim = dim3(192);
+  cfg.blockDim = dim3(kThreads2);
   cfg.dynamicSmemBytes = C::SMEM;
   cfg.stream = st;
   const bool no_pdl = !pdl_on(true);
@@ -195,7 +311,7 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep, i
   attr2[1].val.clusterDim.z = 1;
   cfg.attrs = attr2;
   cfg.numAttrs = 2;
-  CK(cudaLaunchKernelEx(&cfg, kern, a, w, ep, M, N, K));
+  CK(cudaLaunchKernelEx(&cfg, kern, a, w, to, ep, M, N, K));
 }
 
 }  // namespace
@@ -235,3 +351,9 @@ void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, i
 }
 
 }  // namespace duet
+
+// debug hook for tools/gemm_trace.py (not part of the C ABI in include/duet.h)
+extern "C" int duet_debug_tc2_trace(unsigned long long* host, int n) {
+  if (n > 8 * 4096) n = 8 * 4096;
+  return (int)cudaMemcpyFromSymbol(host, duet::g_tc2_trace, (size_t)n * sizeof(unsigned long long));
+}

@@ -37,11 +37,16 @@ struct TcEpilogue {
   int H = 0;
   int kx = 0;                  // k-blocks read from the X map (x_t) before switching to A (h)
   int x_row0 = 0;              // row offset of x_t in the X map ([S*B, E] time-major)
+  int tma_store = 0;  // EPI_BIAS_ACT: 1 = output tile leaves through TMA stores (map passed separately)
   int dbg = 0;  // micro-benchmark switches: 1 = skip UMMA, 2 = skip TMA, 4 = epilogue backoff
 };
 
 // ---- tcgen05 GEMM (gemm_tc.cu) ----
 CUtensorMap make_tmap_bf16_2d(const void* base, int64_t rows, int64_t cols, int box_rows);
+// Output map for TMA-store epilogues: [rows, cols] with row pitch ld elements of `eb` bytes; box =
+// span_bytes / eb columns x 32 rows, swizzle matching span_bytes (128, 64 or 32).  Returns false
+// (map untouched) when the TMA alignment rules are not met.
+bool make_tmap_store_2d(CUtensorMap* m, void* base, int eb, int64_t rows, int64_t cols, int64_t ld, int span_bytes);
 int tc_pick_bn(int M, int N, int num_sms);
 void gemm_tc(const void* A, const void* W, int M, int N, int K, int bn, const TcEpilogue& ep, int epi,
              int out_bf16, cudaStream_t st);
