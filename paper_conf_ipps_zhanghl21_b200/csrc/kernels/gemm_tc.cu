@@ -334,6 +334,8 @@ CUtensorMap make_tmap_bf16_2d(const void* base, int64_t rows, int64_t cols, int 
   return m;
 }
 
+PFN_cuTensorMapEncodeTiled_v12000 tmap_encode_tiled() { return get_encode(); }
+
 bool make_tmap_store_2d(CUtensorMap* m, void* base, int eb, int64_t rows, int64_t cols, int64_t ld, int span_bytes) {
   if (((uintptr_t)base & 15) || (ld * eb) % 16 || cols * eb < span_bytes || rows < 32) return false;
   cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};

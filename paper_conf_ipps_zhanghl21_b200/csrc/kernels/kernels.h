@@ -43,6 +43,10 @@ struct TcEpilogue {
 
 // ---- tcgen05 GEMM (gemm_tc.cu) ----
 CUtensorMap make_tmap_bf16_2d(const void* base, int64_t rows, int64_t cols, int box_rows);
+}  // namespace duet
+#include <cudaTypedefs.h>
+namespace duet {
+PFN_cuTensorMapEncodeTiled_v12000 tmap_encode_tiled();
 // Output map for TMA-store epilogues: [rows, cols] with row pitch ld elements of `eb` bytes; box =
 // span_bytes / eb columns x 32 rows, swizzle matching span_bytes (128, 64 or 32).  Returns false
 // (map untouched) when the TMA alignment rules are not met.
@@ -119,6 +123,13 @@ bool conv_tma_ok(const ConvShape& s);
 // Explicit im2col (layers with C % 64 != 0): cols[m, k] = x[n, ho*s-p+r, wo*s-p+q, c], k = (r, q, c),
 // rows padded to ldk (zeros), bf16.
 void im2col(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStream_t st);
+
+// Direct small-channel conv (conv_stem.cu): im2col in shared memory, tcgen05, persistent.
+bool conv_stem_ok(const ConvShape& s);
+void conv_stem_pack(const void* wf, int64_t ldw, void* wk, const ConvShape& s, cudaStream_t st);  // wk [Co, 192]
+CUtensorMap conv_stem_wmap(const void* wk, int Co);
+void conv_stem(const CUtensorMap& tw, const void* x, const float* bias, void* y, const ConvShape& s, int act,
+               cudaStream_t st);
 
 int num_sms(int device);
 

@@ -393,9 +393,11 @@ void build_op(Program& P, const Node& n, Op& op) {
     }
     // bf16 paths: C % 64 == 0 -> persistent TMA-im2col implicit GEMM; otherwise (the 3-channel
     // stem) explicit im2col [M, ldk] + the CTA-pair GEMM with the folded BN as its bias.
+    static const bool no_stem = getenv("DUET_CONV_STEM") && atoi(getenv("DUET_CONV_STEM")) == 0;
     const bool tma = bf && s.Co % 16 == 0 && conv_tma_ok(s);
-    const bool cols = bf && !tma && s.Co >= 16 && s.Co % 8 == 0 && res < 0;
-    const int64_t ldw = (tma || cols) ? (per_co + 7) / 8 * 8 : per_co;
+    const bool stem = bf && !tma && res < 0 && !no_stem && conv_stem_ok(s);
+    const bool cols = bf && !tma && !stem && s.Co >= 16 && s.Co % 8 == 0 && res < 0;
+    const int64_t ldw = (tma || cols || stem) ? (per_co + 7) / 8 * 8 : per_co;
     void* Wf = P.alloc((int64_t)s.Co * ldw * dtype_bytes(w.dtype));
     float* bias = (float*)P.alloc((int64_t)s.Co * 4);
     fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
@@ -407,6 +409,12 @@ void build_op(Program& P, const Node& n, Op& op) {
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         conv_tc(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, K, act, bn, st);
       };
+      op.n_kernels = 1;
+    } else if (stem) {
+      void* Wk = P.alloc((int64_t)s.Co * 192 * 2);
+      conv_stem_pack(Wf, ldw, Wk, s, 0);
+      CUtensorMap tw = conv_stem_wmap(Wk, s.Co);
+      op.launch = [=](const Ptrs& T, cudaStream_t st) { conv_stem(tw, T[in], bias, T[dst], s, act, st); };
       op.n_kernels = 1;
     } else if (cols) {
       const int64_t M = (int64_t)s.N * s.Ho * s.Wo;

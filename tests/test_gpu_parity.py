@@ -178,7 +178,11 @@ def test_c2_full_size_sampled():
 
 
 @pytest.mark.parametrize("N,H,W,C,Co,k,stride,pad", [
-    (2, 23, 19, 3, 64, 7, 2, 3),      # stem: scalar im2col path (C % 64 != 0), K padded to 8
+    (2, 23, 19, 3, 64, 7, 2, 3),      # W*C % 8 != 0: explicit im2col + pair GEMM, K padded to 8
+    (1, 224, 224, 3, 64, 7, 2, 3),    # ResNet stem at full size: smem-im2col kernel (conv_stem.cu)
+    (2, 64, 64, 3, 64, 7, 2, 3),      # stem kernel, one TMA box per input row
+    (3, 40, 24, 3, 32, 7, 2, 3),      # stem kernel, Wo = 12, Co = 32, rows outside the image
+    (2, 30, 16, 4, 48, 5, 2, 2),      # stem kernel with no dummy element (pad*C even), Co = 48
     (3, 14, 14, 64, 64, 3, 1, 1),     # 3x3, vector path, ragged M tile
     (2, 15, 13, 128, 256, 3, 2, 1),   # stride 2, Co = 256
     (2, 9, 9, 64, 128, 1, 2, 0),      # 1x1 downsample
