@@ -181,22 +181,25 @@ __global__ void __launch_bounds__(THREADS, 1)
     }
   } else if (warp == NB) {
     // ---------------- MMA issuer ----------------
-    if (lane == 0 && my_tiles > 0) {
+    // the whole warp walks the loop (uniform descriptors); elect.sync issues each UMMA
+    if (my_tiles > 0) {
       constexpr uint32_t idesc = ptx::idesc_bf16(ROWS, CO);
       ptx::mbar_wait(w_full, 0);
+      const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
+      const uint64_t dw0 = ptx::desc_sw128(ptx::smem_u32(sW));
       for (int i = 0; i < my_tiles; ++i) {
         const int b = i & 1;
         ptx::mbar_wait(&a_full[b], (i >> 1) & 1);
         if (i >= 2) ptx::mbar_wait(&t_empty[b], ((i >> 1) - 1) & 1);
         ptx::tc_fence_after();
-        const uint32_t a0 = ptx::smem_u32(sA + b * A_BYTES), w0 = ptx::smem_u32(sW);
+        const uint64_t da = da0 + (uint64_t)((b * A_BYTES) >> 4);
         for (int k = 0; k < ((g.dbg & 2) ? 0 : g.ksteps); ++k) {
           const int atom = k >> 2, kk = k & 3;
-          ptx::umma_bf16(tmem + b * CO, ptx::desc_sw128(a0 + atom * A_ATOM_BYTES + kk * 32),
-                         ptx::desc_sw128(w0 + atom * CO * 128 + kk * 32), idesc, k != 0);
+          ptx::umma_bf16_elect(tmem + b * CO, da + (uint64_t)((atom * A_ATOM_BYTES + kk * 32) >> 4),
+                               dw0 + (uint64_t)((atom * CO * 128 + kk * 32) >> 4), idesc, k != 0);
         }
-        ptx::umma_commit(&a_empty[b]);
-        ptx::umma_commit(&t_full[b]);
+        ptx::umma_commit_elect(&a_empty[b]);
+        ptx::umma_commit_elect(&t_full[b]);
       }
     }
   } else {

@@ -130,33 +130,33 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
-      constexpr uint32_t idesc = ptx::idesc_bf16(CBM, BN);
-      int64_t g = 0;
-      int j = 0;
-      for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++j) {
-        const int acc = j & 1;
-        const int use_acc = j >> 1;
-        if (use_acc >= 1) ptx::mbar_wait(&tmem_empty[acc], (use_acc - 1) & 1);
+    // the whole warp walks the loop (uniform descriptors); elect.sync issues each UMMA
+    constexpr uint32_t idesc = ptx::idesc_bf16(CBM, BN);
+    const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
+    const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
+    int64_t g = 0;
+    int j = 0;
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++j) {
+      const int acc = j & 1;
+      const int use_acc = j >> 1;
+      if (use_acc >= 1) ptx::mbar_wait(&tmem_empty[acc], (use_acc - 1) & 1);
+      ptx::tc_fence_after();
+      const uint32_t d = tmem + acc * C::TMEM_COLS;
+      for (int it = 0; it < nk; ++it, ++g) {
+        const int st = (int)(g % C::STAGES);
+        ptx::mbar_wait(&full[st], (uint32_t)((g / C::STAGES) & 1));
         ptx::tc_fence_after();
-        const uint32_t d = tmem + acc * C::TMEM_COLS;
-        for (int it = 0; it < nk; ++it, ++g) {
-          const int st = (int)(g % C::STAGES);
-          ptx::mbar_wait(&full[st], (uint32_t)((g / C::STAGES) & 1));
-          ptx::tc_fence_after();
 #pragma unroll
-          for (int h = 0; h < KB; ++h) {
-            const uint32_t a_base = ptx::smem_u32(sA + st * CA_BYTES + h * (CBM * CBK * 2));
-            const uint32_t b_base = ptx::smem_u32(sB + st * C::B_BYTES + h * C::B_ATOM);
+        for (int h = 0; h < KB; ++h) {
+          // descriptor start address is bits [0, 14) in 16-byte units: offsets add directly
+          const uint64_t da = da0 + (uint64_t)((st * CA_BYTES + h * (CBM * CBK * 2)) >> 4);
+          const uint64_t db = db0 + (uint64_t)((st * C::B_BYTES + h * C::B_ATOM) >> 4);
 #pragma unroll
-            for (int k = 0; k < CBK / 16; ++k)
-              ptx::umma_bf16(d, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
-                             (it | h | k) != 0);
-          }
-          ptx::umma_commit(&empty[st]);
+          for (int k = 0; k < CBK / 16; ++k) ptx::umma_bf16_elect(d, da + 2 * k, db + 2 * k, idesc, (it | h | k) != 0);
         }
-        ptx::umma_commit(&tmem_full[acc]);
+        ptx::umma_commit_elect(&empty[st]);
       }
+      ptx::umma_commit_elect(&tmem_full[acc]);
     }
   } else {
     const int et = threadIdx.x - 64;

@@ -104,24 +104,25 @@ __global__ void __launch_bounds__(192, 1)
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
-      constexpr uint32_t idesc = ptx::idesc_bf16(BM, BN);
-      for (int kb = 0; kb < nk; ++kb) {
-        const int s = kb % Cfg::STAGES;
-        ptx::mbar_wait(&full[s], (kb / Cfg::STAGES) & 1);
-        ptx::tc_fence_after();
-        const uint32_t a_base = ptx::smem_u32(sA + s * A_STAGE_BYTES);
-        const uint32_t b_base = ptx::smem_u32(sB + s * Cfg::B_STAGE_BYTES);
+    // the whole warp walks the k loop (uniform descriptors); elect.sync issues each UMMA
+    constexpr uint32_t idesc = ptx::idesc_bf16(BM, BN);
+    const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
+    const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
+    for (int kb = 0; kb < nk; ++kb) {
+      const int s = kb % Cfg::STAGES;
+      ptx::mbar_wait(&full[s], (kb / Cfg::STAGES) & 1);
+      ptx::tc_fence_after();
+      // descriptor start address is bits [0, 14) in 16-byte units: offsets add directly
+      const uint64_t da = da0 + (uint64_t)((s * A_STAGE_BYTES) >> 4);
+      const uint64_t db = db0 + (uint64_t)((s * Cfg::B_STAGE_BYTES) >> 4);
 #pragma unroll
-        for (int k = 0; k < BK / 16; ++k) {
-          if (ep.dbg & 1) break;
-          ptx::umma_bf16(tmem, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
-                         (kb | k) != 0);
-        }
-        ptx::umma_commit(&empty[s]);
+      for (int k = 0; k < BK / 16; ++k) {
+        if (ep.dbg & 1) break;
+        ptx::umma_bf16_elect(tmem, da + 2 * k, db + 2 * k, idesc, (kb | k) != 0);
       }
-      ptx::umma_commit(tmem_full);
+      ptx::umma_commit_elect(&empty[s]);
     }
+    ptx::umma_commit_elect(tmem_full);
   } else {
     // ---------------- epilogue warps 2..5 ----------------
     const int q = warp & 3;  // TMEM lane quarter this warp may access

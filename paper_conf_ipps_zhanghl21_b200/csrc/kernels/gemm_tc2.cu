@@ -47,10 +47,11 @@ struct Cfg2 {
   static constexpr int SMEM = STAGES * STAGE + 1024 + 256 + BN * 4;
 };
 
-// MC = 1: cluster of 4 CTAs = 2 pairs along N sharing the A rows; pair 0 loads A once and
-// multicasts it to pair 1 (halves A's L2->SMEM traffic).  MMA commits go to all 4 CTAs so a
-// stage is refilled only after both pairs consumed it (empty barrier count 2).
-template <int BN, typename OutT, int MC>
+// NP > 1: cluster of 2*NP CTAs = NP pairs along N sharing the A rows.  Each A k-block is split
+// into NP row slices of 128/NP rows; pair p's CTA r loads slice p of its rows and multicasts it
+// to CTA r of every pair, so the cluster reads A from L2 once instead of NP times.  MMA commits go
+// to all 2*NP CTAs so a stage is refilled only after every pair consumed it (empty count NP).
+template <int BN, typename OutT, int NP>
 __global__ void __launch_bounds__(kThreads2, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                  const __grid_constant__ CUtensorMap tmO, const TcEpilogue ep, int M, int N, int K) {
@@ -70,10 +71,12 @@ __global__ void __launch_bounds__(kThreads2, 1)
   const bool tr = (ep.dbg & 32) != 0;
   unsigned long long* trace = g_tc2_trace + 8 * ((blockIdx.y * gridDim.x + blockIdx.x) & 4095);
   if (tr && threadIdx.x == 0) trace[0] = gtimer();
+  constexpr bool MC = NP > 1;
+  constexpr int SLICE = BM2 / NP;  // A rows per multicast slice
   const uint32_t crank = ptx::cluster_ctarank();
   const uint32_t rank = crank & 1;          // rank within the CTA pair
   const int pair = MC ? (int)(crank >> 1) : 0;
-  const int tile_n = MC ? (blockIdx.x >> 2) * 2 + pair : (blockIdx.x >> 1);
+  const int tile_n = (int)(blockIdx.x / (2 * NP)) * NP + pair;
   const int n0 = tile_n * BN;
   const int m0 = blockIdx.y * (2 * BM2) + (int)rank * BM2;  // this CTA's rows
   const int nk = (K + KB2 * BK2 - 1) / (KB2 * BK2);  // stages of KB2 k-blocks
@@ -84,7 +87,7 @@ __global__ void __launch_bounds__(kThreads2, 1)
     ptx::tma_prefetch(&tmW);
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
-      ptx::mbar_init(&empty[s], MC ? 2 : 1);
+      ptx::mbar_init(&empty[s], NP);
     }
     ptx::mbar_init(tmem_full, 1);
     ptx::fence_mbar_init();
@@ -115,8 +118,8 @@ __global__ void __launch_bounds__(kThreads2, 1)
   }
   ptx::tc_fence_before();
   // A loads (below) follow this CTA's alloc, so the leader's first full barrier implies both CTAs'
-  // TMEM is allocated before the first MMA.  With multicast, pair 1 receives A from pair 0, so
-  // the whole cluster synchronises instead.
+  // TMEM is allocated before the first MMA.  With multicast, a pair receives A slices from the
+  // other pairs, so the whole cluster synchronises instead.
   if constexpr (MC) ptx::cluster_sync(); else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
@@ -125,7 +128,7 @@ __global__ void __launch_bounds__(kThreads2, 1)
 
   if (warp == 0) {
     if (lane == 0) {
-      const uint16_t a_mask = (uint16_t)(0x5u << rank);  // CTA r of pair 0 and of pair 1
+      const uint16_t a_mask = (uint16_t)((NP == 4 ? 0x55u : NP == 2 ? 0x5u : 0x1u) << rank);  // CTA r of every pair
       for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % C::STAGES;
         const bool pre = kb < npre && !(ep.dbg & 2);
@@ -140,8 +143,9 @@ __global__ void __launch_bounds__(kThreads2, 1)
         for (int h = 0; h < KB2; ++h) {
           if (!MC)
             ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
-          else if (pair == 0)
-            ptx::tma_load_2d_2sm_mc(&tmA, &full[s], sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0, a_mask);
+          else
+            ptx::tma_load_2d_2sm_mc(&tmA, &full[s], sA + s * A2_BYTES + h * A2_ATOM + pair * SLICE * 128,
+                                    (kb * KB2 + h) * BK2, m0 + pair * SLICE, a_mask);
           if (!pre)
             ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
                                  n0 + (int)rank * C::BH);
@@ -149,29 +153,32 @@ __global__ void __launch_bounds__(kThreads2, 1)
       }
     }
   } else if (warp == 1) {
-    if (rank == 0 && lane == 0) {
+    if (rank == 0) {
+      // the whole warp walks the k loop (uniform descriptors); elect.sync issues each UMMA
       constexpr uint32_t idesc = ptx::idesc_bf16(2 * BM2, BN);
-      const uint16_t empty_mask = MC ? (uint16_t)0xF : (uint16_t)0x3;
+      const uint16_t empty_mask = (uint16_t)((1u << (2 * NP)) - 1);
       const uint16_t pair_mask = (uint16_t)(0x3u << (2 * pair));
+      const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
+      const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
       for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % C::STAGES;
         ptx::mbar_wait(&full[s], (kb / C::STAGES) & 1);
         ptx::tc_fence_after();
-        if (tr && kb == 0) trace[3] = gtimer();
+        if (tr && kb == 0 && lane == 0) trace[3] = gtimer();
 #pragma unroll
         for (int h = 0; h < KB2; ++h) {
-          const uint32_t a_base = ptx::smem_u32(sA + s * A2_BYTES + h * A2_ATOM);
-          const uint32_t b_base = ptx::smem_u32(sB + s * C::B_BYTES + h * C::B_ATOM);
+          // descriptor start address is bits [0, 14) in 16-byte units: offsets add directly
+          const uint64_t da = da0 + (uint64_t)((s * A2_BYTES + h * A2_ATOM) >> 4);
+          const uint64_t db = db0 + (uint64_t)((s * C::B_BYTES + h * C::B_ATOM) >> 4);
 #pragma unroll
           for (int k = 0; k < BK2 / 16; ++k)
             if (!(ep.dbg & 1))
-              ptx::umma_bf16_2sm(tmem, ptx::desc_sw128(a_base + k * 32), ptx::desc_sw128(b_base + k * 32), idesc,
-                                 (kb | h | k) != 0);
+              ptx::umma_bf16_2sm_elect(tmem, da + 2 * k, db + 2 * k, idesc, (kb | h | k) != 0);
         }
-        ptx::umma_commit_2sm(&empty[s], empty_mask);
+        ptx::umma_commit_2sm_elect(&empty[s], empty_mask);
       }
-      ptx::umma_commit_2sm(tmem_full, pair_mask);
-      if (tr) trace[4] = gtimer();
+      ptx::umma_commit_2sm_elect(tmem_full, pair_mask);
+      if (tr && lane == 0) trace[4] = gtimer();
     }
   } else {
     // epilogue warps 2..9: warp w reads TMEM lanes 32 (w % 4) .. +32 (hardware lane-quarter
@@ -276,7 +283,7 @@ __global__ void __launch_bounds__(kThreads2, 1)
   }
 }
 
-template <int BN, typename OutT, int MC>
+template <int BN, typename OutT, int NP>
 void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep_in, int M, int N, int K, cudaStream_t st) {
   using C = Cfg2<BN>;
   static const bool no_tma_store = getenv("DUET_TMA_STORE") && atoi(getenv("DUET_TMA_STORE")) == 0;
@@ -287,15 +294,14 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep_in
   static_assert(2 * 32 * SPAN * 8 <= C::STAGES * A2_BYTES, "TMA-store staging must fit in the A stages");
   ep.tma_store = !no_tma_store && !(ep.dbg & 8) && SPAN >= 32 &&
                  make_tmap_store_2d(&to, ep.out, EB, M, N, ep.ldo, SPAN);
-  auto kern = gemm2_kernel<BN, OutT, MC>;
+  auto kern = gemm2_kernel<BN, OutT, NP>;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
-    if (MC) CK(cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 0));
     attr = true;
   }
   const int tn = (N + BN - 1) / BN;
-  dim3 grid(MC ? 4 * ((tn + 1) / 2) : 2 * tn, (M + 2 * BM2 - 1) / (2 * BM2));
+  dim3 grid(2 * NP * ((tn + NP - 1) / NP), (M + 2 * BM2 - 1) / (2 * BM2));
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = grid;
   cfg.blockDim = dim3(kThreads2);
@@ -306,7 +312,7 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep_in
   attr2[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr2[0].val.programmaticStreamSerializationAllowed = no_pdl ? 0 : 1;
   attr2[1].id = cudaLaunchAttributeClusterDimension;
-  attr2[1].val.clusterDim.x = MC ? 4 : 2;
+  attr2[1].val.clusterDim.x = 2 * NP;
   attr2[1].val.clusterDim.y = 1;
   attr2[1].val.clusterDim.z = 1;
   cfg.attrs = attr2;
@@ -329,18 +335,29 @@ int tc2_pick_bn(int M, int N, int K, int sms) {
   return 64;
 }
 
-void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
-                   int out_bf16, cudaStream_t st) {
-  // multicast pairs (opt-in, DUET_GEMM_MC=1): measured no gain at cluster size 4 (L2 dedups multicast
-  // only for wider clusters), kept for the wider-cluster experiments
-  static const int mc_env = getenv("DUET_GEMM_MC") ? atoi(getenv("DUET_GEMM_MC")) : 0;
-  const bool mc = mc_env && (N + bn - 1) / bn >= 2;
+int tc2_pick_np(int M, int N, int bn) {
+  // pairs per cluster sharing A by multicast (1, 2 or 4); DUET_GEMM_MC overrides
+  (void)M;
+  static const int env = getenv("DUET_GEMM_MC") ? atoi(getenv("DUET_GEMM_MC")) : -1;
+  const int tn = (N + bn - 1) / bn;
+  int np = env >= 0 ? env : 1;
+  if (np != 1 && np != 2 && np != 4) np = 1;
+  while (np > 1 && tn % np) np >>= 1;
+  return np;
+}
+
+void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, int np,
+                   const TcEpilogue& ep, int out_bf16, cudaStream_t st) {
+  // `ta` must have been encoded with box rows 128 / np (A multicast slices)
 #define DUET_L2(BNV)                                                                      \
-  if (mc)                                                                                 \
-    return out_bf16 ? launch2<BNV, __nv_bfloat16, 1>(ta, tw, ep, M, N, K, st)            \
-                    : launch2<BNV, float, 1>(ta, tw, ep, M, N, K, st);                    \
-  return out_bf16 ? launch2<BNV, __nv_bfloat16, 0>(ta, tw, ep, M, N, K, st)              \
-                  : launch2<BNV, float, 0>(ta, tw, ep, M, N, K, st);
+  if (np == 4)                                                                            \
+    return out_bf16 ? launch2<BNV, __nv_bfloat16, 4>(ta, tw, ep, M, N, K, st)            \
+                    : launch2<BNV, float, 4>(ta, tw, ep, M, N, K, st);                    \
+  if (np == 2)                                                                            \
+    return out_bf16 ? launch2<BNV, __nv_bfloat16, 2>(ta, tw, ep, M, N, K, st)            \
+                    : launch2<BNV, float, 2>(ta, tw, ep, M, N, K, st);                    \
+  return out_bf16 ? launch2<BNV, __nv_bfloat16, 1>(ta, tw, ep, M, N, K, st)              \
+                  : launch2<BNV, float, 1>(ta, tw, ep, M, N, K, st);
   switch (bn) {
     case 64: DUET_L2(64)
     case 128: DUET_L2(128)

@@ -63,8 +63,10 @@ void rnn_pack(int kind, const void* Wih, const void* Whh, const float* bih, cons
 
 // CTA-pair GEMM (gemm_tc2.cu): 256 x bn tiles, bn in {64,128,256}; W map box rows = bn / 2.
 int tc2_pick_bn(int M, int N, int K, int num_sms);
-void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
-                   int out_bf16, cudaStream_t st);
+// pairs per cluster that share the A tile by TMA multicast (A map box rows = 128 / np)
+int tc2_pick_np(int M, int N, int bn);
+void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, int np,
+                   const TcEpilogue& ep, int out_bf16, cudaStream_t st);
 
 // ---- SIMT fallbacks / small kernels (simt.cu) ----
 // Y[M,N] = act(X[M,K] W[N,K]^T + b) ; X/W dtype per flags; fp32 accumulate.

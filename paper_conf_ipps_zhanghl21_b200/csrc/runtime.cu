@@ -205,18 +205,19 @@ void build_op(Program& P, const Node& n, Op& op) {
     if (xb && wb && K % 8 == 0 && N >= 16 && pair) {
       const char* bn_env = getenv("DUET_GEMM_BN");
       const int bn = bn_env ? atoi(bn_env) : tc2_pick_bn(M, N, K, sms);
+      const int np = tc2_pick_np(M, N, bn);
       const char* dbg_env = getenv("DUET_GEMM_DBG");
       const int dbg2 = dbg_env ? atoi(dbg_env) : 0;
       CUtensorMap tw = make_tmap_bf16_2d(W, N, K, bn / 2);
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
-        CUtensorMap ta = make_tmap_bf16_2d(T[in], M, K, 128);
+        CUtensorMap ta = make_tmap_bf16_2d(T[in], M, K, 128 / np);
         TcEpilogue ep;
         ep.bias = b;
         ep.out = T[me];
         ep.ldo = N;
         ep.act = act;
         ep.dbg = dbg2;
-        gemm_tc2_maps(ta, tw, M, N, K, bn, ep, yb, st);
+        gemm_tc2_maps(ta, tw, M, N, K, bn, np, ep, yb, st);
       };
     } else if (xb && wb && K % 8 == 0 && N >= 16) {
       const char* dbg_env = getenv("DUET_GEMM_DBG");
@@ -429,7 +430,7 @@ void build_op(Program& P, const Node& n, Op& op) {
         ep.out = T[dst];
         ep.ldo = s.Co;
         ep.act = act;
-        gemm_tc2_maps(ta, tw, (int)M, s.Co, (int)ldw, bn, ep, 1, st);
+        gemm_tc2_maps(ta, tw, (int)M, s.Co, (int)ldw, bn, 1, ep, 1, st);
       };
       op.n_kernels = 2;
     } else {

@@ -4,7 +4,7 @@ import ctypes
 import os
 import sys
 
-os.environ["DUET_GEMM_DBG"] = "32"
+os.environ["DUET_GEMM_DBG"] = str(32 | int(os.environ.get("DBG", "0")))
 if len(sys.argv) > 4:
     os.environ["DUET_GEMM_BN"] = sys.argv[4]
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -31,7 +31,13 @@ lib.duet_debug_tc2_trace(buf, 8 * 4096)
 a = np.frombuffer(buf, dtype=np.uint64).reshape(4096, 8).astype(np.int64)
 ctas = a[a[:, 0] > 0]
 t0 = ctas[:, 0].min()
-print(f"M={M} N={N} K={K}: {len(ctas)} CTAs; times in ns relative to the first CTA entry")
+try:
+    import pynvml
+    pynvml.nvmlInit()
+    clk = pynvml.nvmlDeviceGetClockInfo(pynvml.nvmlDeviceGetHandleByIndex(0), pynvml.NVML_CLOCK_SM)
+except Exception:
+    clk = -1
+print(f"M={M} N={N} K={K}: {len(ctas)} CTAs; sm clock {clk} MHz; times in ns relative to the first CTA entry")
 print(f"{'phase':16s} {'min':>8s} {'median':>8s} {'max':>8s}")
 for i, n in enumerate(names):
     v = ctas[:, i]
