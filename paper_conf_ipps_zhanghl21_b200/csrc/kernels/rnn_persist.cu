@@ -1,0 +1,393 @@
+// Persistent fused LSTM / GRU recurrence for latency-bound batches.
+//
+// One launch runs all S time steps.  CTA (n, m) owns gate-block tile n (U = BN/4 hidden units,
+// all four gate blocks, the same packed weights as the per-step kernel in gemm_tc.cu) for batch
+// rows [128 m, +128).  Per step t:
+//
+//   acc[t&1]  = x_t W_x^T              (kx k-blocks; independent of h, so they are loaded and
+//                                       multiplied while step t-1's epilogue and barrier run)
+//   acc[t&1] += h_{t-1} W_h^T          (kh k-blocks, loaded by TMA after the grid barrier)
+//   epilogue: gates -> c_t (LSTM, fp32 in registers for the whole sequence), h_t -> bf16 global
+//   grid barrier: every CTA's slice of h_t is written (one release-add per epilogue warp per step)
+//
+// Versus one kernel per step this removes the launch / prologue / TMEM allocation of every step
+// and the x-projection from the critical path; the cell state never leaves the SM.  The TMEM
+// accumulator is double-buffered (2 x BN columns) so step t+1's x part overlaps step t's epilogue.
+// Co-residency of the grid (required by the barrier) is guaranteed by a cooperative launch; the
+// runtime uses this kernel only when the grid fits in half of the SMs (two recurrent branches on
+// two stream slots must co-reside).
+//
+// Warp roles: warp 0 TMA producer, warp 1 TMEM allocator + MMA issuer (warp-convergent, elect.sync),
+// warps 2..9 epilogue (warp w reads TMEM lane quarter w % 4; the two warps of a quarter split the
+// units of the tile).
+#include "../common.h"
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace duet {
+
+// per-CTA, per-step %globaltimer stamps when RnnPersistArgs::dbg & 1 (tools/rnn_trace.py):
+// [cta][t][0] h_{t-1} barrier passed (producer), [1] first x stage landed (MMA warp),
+// [2] accumulator ready (epilogue), [3] h_t stored + released (epilogue), [4] first h stage landed
+// (MMA warp), [5] last UMMA of the step issued
+__device__ unsigned long long g_rp_trace[128 * 64 * 16];
+
+namespace {
+
+__device__ __forceinline__ unsigned long long rp_gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+constexpr int RBM = 128;
+constexpr int RBK = 64;
+constexpr int R_A_BYTES = RBM * RBK * 2;
+constexpr int kREpiWarps = 8;
+constexpr int kRThreads = 64 + 32 * kREpiWarps + 32;  // + W producer warp (last)
+constexpr int kWWarp = 2 + kREpiWarps;
+
+template <int BN>
+struct RCfg {
+  static constexpr int U = BN / 4;   // hidden units per tile
+  static constexpr int UH = U / 2;   // units per epilogue thread
+  static constexpr int B_BYTES = BN * RBK * 2;
+  static constexpr int TMEM_COLS = 2 * BN <= 128 ? 128 : 256;
+  static constexpr int EXTRA = 1024 + 512 + BN * 4;  // alignment slack + barriers + bias
+};
+// Shared-memory plan: [A ring: stages x 16 KB][W: resident (kx + kh blocks) or a ring of `stages`
+// blocks][barriers][bias].  W is resident when it fits next to a ring of >= 6 A stages.
+constexpr int kRSmemBudget = 227 * 1024;
+inline int rp_plan(int bn, int nkw, bool* wres) {
+  const int bb = bn * RBK * 2, extra = 1024 + 512 + bn * 4;
+  const int res_stages = (kRSmemBudget - extra - nkw * bb) / R_A_BYTES;
+  if (res_stages >= 6) {
+    *wres = true;
+    return res_stages > 10 ? 10 : res_stages;
+  }
+  *wres = false;
+  const int st = (192 * 1024) / (R_A_BYTES + bb);
+  return st > 10 ? 10 : st;
+}
+
+// (measured: a relaxed polling loop + one fence.acq_rel.gpu passes the barrier ~0.3 us later than
+// polling with ld.acquire)
+__device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void red_release_gpu_add(unsigned* p, unsigned v) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_global() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
+__device__ __forceinline__ float tanh_approx(float x) {
+  float y;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+// bf16 path only (tolerance 2e-2): tanh.approx.f32 has ~2^-11 relative error,
+// below the bf16 rounding of h_t itself
+// sigma(x) = 0.5 tanh(x / 2) + 0.5: one MUFU op instead of ex2 + rcp (the epilogue is MUFU-bound:
+// 2048 cells x 5 transcendental per CTA per step)
+__device__ __forceinline__ float rsig(float x) { return fmaf(0.5f, tanh_approx(0.5f * x), 0.5f); }
+__device__ __forceinline__ float rtanh(float x) { return tanh_approx(x); }
+
+// mbarrier wait with the hardware suspend of try_wait: ten warps wait at different times here, and
+// a spinning test_wait loop steals issue slots from the epilogue warps on the same SM sub-partition
+__device__ __forceinline__ void wait_sleep(uint64_t* bar, uint32_t parity) {
+  const uint32_t addr = ptx::smem_u32(bar);
+  while (!ptx::mbar_try_wait(addr, parity)) {
+  }
+}
+
+template <int N>
+__device__ __forceinline__ void tmem_ld_n(uint32_t taddr, float* v) {
+  if constexpr (N == 16) ptx::tmem_ld16(taddr, v);
+  else ptx::tmem_ld8(taddr, v);
+}
+
+template <int BN, int KIND, bool WRES>
+__global__ void __launch_bounds__(kRThreads, 1)
+    rnn_persist_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmH0,
+                       const __grid_constant__ CUtensorMap tmH1, const __grid_constant__ CUtensorMap tmW,
+                       const RnnPersistArgs a) {
+  using C = RCfg<BN>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int STAGES = a.stages;
+  const int nkw = a.kx + a.kh;  // packed weight k-blocks
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + STAGES * R_A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + (WRES ? nkw : STAGES) * C::B_BYTES);
+  uint64_t* empty = full + 10;
+  uint64_t* tfull = empty + 10;
+  uint64_t* tempty = tfull + 2;
+  uint64_t* w_full = tempty + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(w_full + 1);
+  float* s_bias = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(full) + 512);
+
+  const int warp = ptx::warp_id();
+  const int lane = threadIdx.x & 31;
+  const int n0 = blockIdx.x * BN;
+  const int m0 = blockIdx.y * RBM;
+  const int S = a.S, kx = a.kx, kh = a.kh;
+  const int cta = blockIdx.y * gridDim.x + blockIdx.x;
+  unsigned long long* trace = (a.dbg & 1) && cta < 128 ? g_rp_trace + (size_t)cta * 64 * 16 : nullptr;
+
+  if (threadIdx.x == 0) {
+    ptx::tma_prefetch(&tmX);
+    ptx::tma_prefetch(&tmH0);
+    ptx::tma_prefetch(&tmH1);
+    ptx::tma_prefetch(&tmW);
+    for (int s = 0; s < STAGES; ++s) {
+      ptx::mbar_init(&full[s], WRES ? 1 : 2);  // A producer (+ W producer), each with its tx bytes
+      ptx::mbar_init(&empty[s], 1);
+    }
+    ptx::mbar_init(w_full, 1);
+    for (int b = 0; b < 2; ++b) {
+      ptx::mbar_init(&tfull[b], 1);
+      ptx::mbar_init(&tempty[b], kREpiWarps);
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) {
+    ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
+    ptx::tmem_relinquish();
+  }
+  for (int c = (int)threadIdx.x - 64; c >= 0 && c < BN; c += 32 * kREpiWarps) s_bias[c] = a.bias[n0 + c];
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    // ---------------- TMA producer ----------------
+    int g = 0;
+    for (int t = 0; t < S; ++t) {
+      const int nkb = kx + (t > 0 ? kh : 0);  // h_{-1} = 0: step 0 has only the x part
+      const CUtensorMap* th = ((t - 1) & 1) ? &tmH1 : &tmH0;
+      for (int j = 0; j < nkb; ++j, ++g) {
+        const int s = g % STAGES;
+        if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
+        if (j == kx) {
+          // h_{t-1}: wait until every CTA has released its slice (grid barrier), then order the
+          // generic-proxy writes it observed before this thread's async-proxy (TMA) reads
+          if (lane == 0) {
+            const unsigned target = (unsigned)t * (unsigned)a.n_cta * kREpiWarps;
+            while (ld_acquire_gpu(a.counter) < target) {
+            }
+            fence_proxy_async_global();
+            if (trace && t < 64) trace[t * 16 + 0] = rp_gtimer();
+          }
+          __syncwarp();
+        }
+        if (lane == 0) {
+          ptx::mbar_arrive_expect_tx(&full[s], R_A_BYTES);
+          if (j < kx)
+            ptx::tma_load_2d(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
+          else
+            ptx::tma_load_2d(th, &full[s], sA + s * R_A_BYTES, (j - kx) * RBK, m0);
+        }
+        __syncwarp();
+      }
+    }
+  } else if (warp == kWWarp) {
+    // ---------------- W producer: weights never depend on h ----------------
+    if constexpr (WRES) {
+      // resident: every packed weight block of this tile, loaded once for the whole sequence
+      if (lane == 0) {
+        ptx::mbar_arrive_expect_tx(w_full, (uint32_t)(nkw * C::B_BYTES));
+        for (int j = 0; j < nkw; ++j) ptx::tma_load_2d(&tmW, w_full, sB + j * C::B_BYTES, j * RBK, n0);
+      }
+    } else {
+      // streamed ahead of the barrier in the A ring's stage order
+      int g = 0;
+      for (int t = 0; t < S; ++t) {
+        const int nkb = kx + (t > 0 ? kh : 0);
+        for (int j = 0; j < nkb; ++j, ++g) {
+          const int s = g % STAGES;
+          if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
+          if (lane == 0) {
+            ptx::mbar_arrive_expect_tx(&full[s], C::B_BYTES);
+            // packed weight columns: [x part (kx blocks) | h part (kh blocks)] -> column block j
+            ptx::tma_load_2d(&tmW, &full[s], sB + s * C::B_BYTES, j * RBK, n0);
+          }
+          __syncwarp();
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ---------------- MMA issuer (whole warp, elect.sync issues) ----------------
+    constexpr uint32_t idesc = ptx::idesc_bf16(RBM, BN);
+    const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
+    const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
+    if constexpr (WRES) wait_sleep(w_full, 0);
+    int g = 0;
+    for (int t = 0; t < S; ++t) {
+      const int buf = t & 1;
+      if (t >= 2) wait_sleep(&tempty[buf], ((t >> 1) - 1) & 1);
+      ptx::tc_fence_after();
+      const uint32_t d = tmem + (uint32_t)(buf * BN);
+      const int nkb = kx + (t > 0 ? kh : 0);
+      for (int j = 0; j < nkb; ++j, ++g) {
+        const int s = g % STAGES;
+        wait_sleep(&full[s], (g / STAGES) & 1);
+        ptx::tc_fence_after();
+        if (trace && t < 64 && lane == 0) {
+          if (j == 0) trace[t * 16 + 1] = rp_gtimer();
+          if (j == kx) trace[t * 16 + 4] = rp_gtimer();  // first h stage landed
+        }
+        const uint64_t da = da0 + (uint64_t)((s * R_A_BYTES) >> 4);
+        const uint64_t db = db0 + (uint64_t)(((WRES ? j : s) * C::B_BYTES) >> 4);
+        if (!(a.dbg & 16))
+#pragma unroll
+          for (int k = 0; k < RBK / 16; ++k) ptx::umma_bf16_elect(d, da + 2 * k, db + 2 * k, idesc, (j | k) != 0);
+        ptx::umma_commit_elect(&empty[s]);
+      }
+      ptx::umma_commit_elect(&tfull[buf]);
+      if (trace && t < 64 && lane == 0) trace[t * 16 + 5] = rp_gtimer();  // last UMMA issued
+    }
+  } else {
+    // ---------------- epilogue: gates, cell, h_t ----------------
+    constexpr int U = C::U, UH = C::UH;
+    const int q = warp & 3;
+    const int half = (warp - 2) >> 2;
+    const int row = m0 + q * 32 + lane;
+    const int H = a.H;
+    const int unit0 = blockIdx.x * U + half * UH;
+    const int nv = min(UH, H - unit0);  // multiple of 8 (H % 8 == 0)
+    const bool live = row < a.B && nv > 0;
+    float bias[4][UH];  // this thread's gate biases, in registers for the whole sequence
+#pragma unroll
+    for (int g = 0; g < 4; ++g)
+#pragma unroll
+      for (int i = 0; i < UH; ++i) bias[g][i] = s_bias[g * U + half * UH + i];
+    float state[UH];  // LSTM: c_{t-1}; GRU: h_{t-1} (fp32)
+#pragma unroll
+    for (int i = 0; i < UH; ++i) state[i] = 0.0f;
+    for (int t = 0; t < S; ++t) {
+      const int buf = t & 1;
+      wait_sleep(&tfull[buf], (t >> 1) & 1);
+      ptx::tc_fence_after();
+      if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 2] = rp_gtimer();
+      const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
+      float acc[4][UH];
+#pragma unroll
+      for (int g = 0; g < 4; ++g) tmem_ld_n<UH>(tq + g * U + half * UH, acc[g]);
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&tempty[buf]);  // accumulator buffer free for step t+2
+      if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 6] = rp_gtimer();  // TMEM read
+      float h[UH];
+#pragma unroll
+      for (int i = 0; i < UH; ++i) {
+        const float a0 = acc[0][i] + bias[0][i], a1 = acc[1][i] + bias[1][i];
+        const float a2 = acc[2][i] + bias[2][i], a3 = acc[3][i] + bias[3][i];
+        if constexpr (KIND == EPI_LSTM) {
+          const float ig = rsig(a0), fg = rsig(a1), gg = rtanh(a2), og = rsig(a3);
+          state[i] = fg * state[i] + ig * gg;
+          h[i] = og * rtanh(state[i]);
+        } else {
+          const float r = rsig(a0), z = rsig(a1);
+          const float n = rtanh(a2 + r * a3);  // (W_in x + b_in) + r * (W_hn h + b_hn)
+          h[i] = (1.0f - z) * n + z * state[i];
+          state[i] = h[i];
+        }
+      }
+      __nv_bfloat16* dst = (t == S - 1 ? a.out : a.hbuf[buf]) + (size_t)row * H + unit0;
+      if (live) {
+#pragma unroll
+        for (int v = 0; v < UH / 8; ++v) {
+          if (v * 8 < nv) {
+            uint32_t w[4];
+#pragma unroll
+            for (int p = 0; p < 4; ++p) {
+              __nv_bfloat162 b2 = __floats2bfloat162_rn(h[v * 8 + 2 * p], h[v * 8 + 2 * p + 1]);
+              w[p] = *reinterpret_cast<uint32_t*>(&b2);
+            }
+            reinterpret_cast<uint4*>(dst)[v] = make_uint4(w[0], w[1], w[2], w[3]);
+          }
+        }
+      }
+      if (trace && t < 64 && lane == 0) trace[t * 16 + 6 + warp] = rp_gtimer();  // [8..15] math + stores
+      if (t < S - 1) {
+        // each warp releases its own slice of h_t (no CTA-wide barrier): the generic-proxy stores
+        // are ordered before the release-add by __syncwarp; the consumer acquires the counter and
+        // issues fence.proxy.async before its TMA reads
+        if (!(a.dbg & 2)) fence_proxy_async_global();
+        __syncwarp();
+        if (lane == 0) red_release_gpu_add(a.counter, 1u);
+        if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 3] = rp_gtimer();
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem, C::TMEM_COLS);
+  }
+}
+
+template <int BN, int KIND, bool WRES>
+void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1, const CUtensorMap& tw,
+               const RnnPersistArgs& a, dim3 grid, cudaStream_t st) {
+  using C = RCfg<BN>;
+  auto kern = rnn_persist_kernel<BN, KIND, WRES>;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kRSmemBudget));
+    attr = true;
+  }
+  const int smem = a.stages * R_A_BYTES + (WRES ? a.kx + a.kh : a.stages) * C::B_BYTES + C::EXTRA;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = dim3(kRThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  CK(cudaLaunchKernelEx(&cfg, kern, tx, th0, th1, tw, a));
+}
+
+template <int BN, int KIND>
+void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1, const CUtensorMap& tw,
+                   RnnPersistArgs a, dim3 grid, cudaStream_t st) {
+  static const int wres_env = getenv("DUET_RNN_WRES") ? atoi(getenv("DUET_RNN_WRES")) : 1;
+  bool wres = false;
+  a.stages = rp_plan(BN, a.kx + a.kh, &wres);
+  if (wres && !wres_env) {  // streamed W (comparisons)
+    wres = false;
+    a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
+    if (a.stages > 10) a.stages = 10;
+  }
+  if (wres) return launch_rp<BN, KIND, true>(tx, th0, th1, tw, a, grid, st);
+  launch_rp<BN, KIND, false>(tx, th0, th1, tw, a, grid, st);
+}
+
+}  // namespace
+
+void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1,
+                 const CUtensorMap& tw, const RnnPersistArgs& a, int tiles_n, int tiles_m, cudaStream_t st) {
+  const dim3 grid(tiles_n, tiles_m);
+  if (kind == EPI_LSTM && bn == 64) return launch_rp_any<64, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
+  if (kind == EPI_LSTM && bn == 128) return launch_rp_any<128, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
+  if (kind == EPI_GRU && bn == 64) return launch_rp_any<64, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
+  if (kind == EPI_GRU && bn == 128) return launch_rp_any<128, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
+  fail(DUET_EUNSUPPORTED, "rnn_persist: bn must be 64 or 128");
+}
+
+}  // namespace duet
+
+// debug hook for tools/rnn_trace.py (not part of the C ABI in include/duet.h)
+extern "C" int duet_debug_rp_trace(unsigned long long* host, int n) {
+  if (n > 128 * 64 * 16) n = 128 * 64 * 16;
+  return (int)cudaMemcpyFromSymbol(host, duet::g_rp_trace, (size_t)n * sizeof(unsigned long long));
+}

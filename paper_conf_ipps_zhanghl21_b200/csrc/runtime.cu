@@ -311,7 +311,57 @@ void build_op(Program& P, const Node& n, Op& op) {
     const int es = dtype_bytes(x.dtype);
     void* hb[2] = {P.alloc((int64_t)B * H * es), P.alloc((int64_t)B * H * es)};
     float* cst = (float*)P.alloc((int64_t)B * H * 4);
-    if (tc) {
+    // persistent recurrence (kernels/rnn_persist.cu) when the grid fits in half of the SMs (two
+    // recurrent branches on two slots co-reside); DUET_RNN_PERSIST=0 forces the per-step kernels
+    static const int rp_env = getenv("DUET_RNN_PERSIST") ? atoi(getenv("DUET_RNN_PERSIST")) : 1;
+    static const int rp_bn_env = getenv("DUET_RNN_BN") ? atoi(getenv("DUET_RNN_BN")) : 0;
+    int rp_bn = 0;
+    if (tc && rp_env) {
+      const int mt = (B + 127) / 128;
+      for (int cand : {64, 128}) {
+        if (rp_bn_env && cand != rp_bn_env) continue;
+        if (mt * ((H + cand / 4 - 1) / (cand / 4)) <= sms / 2) {
+          rp_bn = cand;
+          break;
+        }
+      }
+    }
+    if (rp_bn) {
+      const int bn = rp_bn;
+      const int U = bn / 4;
+      const int tiles = (H + U - 1) / U;
+      const int mt = (B + 127) / 128;
+      const int Np = tiles * bn;
+      const int Ep = (E + 63) / 64 * 64;
+      const int Kc = Ep + H;
+      void* Wcat = P.alloc((int64_t)Np * Kc * 2);
+      float* bias = (float*)P.alloc((int64_t)Np * 4);
+      unsigned* counter = (unsigned*)P.alloc(256);
+      rnn_pack(kind, Wih, Whh, bih, bhh, Wcat, bias, E, Ep, H, U, bn, tiles, 0);
+      CK(cudaDeviceSynchronize());
+      CUtensorMap t_w = make_tmap_bf16_2d(Wcat, Np, Kc, bn);
+      CUtensorMap t_h0 = make_tmap_bf16_2d(hb[0], B, H, 128), t_h1 = make_tmap_bf16_2d(hb[1], B, H, 128);
+      RnnPersistArgs ra;
+      ra.bias = bias;
+      ra.hbuf[0] = (__nv_bfloat16*)hb[0];
+      ra.hbuf[1] = (__nv_bfloat16*)hb[1];
+      ra.counter = counter;
+      ra.S = S;
+      ra.B = B;
+      ra.H = H;
+      ra.kx = Ep / 64;
+      ra.kh = (H + 63) / 64;
+      ra.n_cta = tiles * mt;
+      ra.dbg = getenv("DUET_RNN_DBG") ? atoi(getenv("DUET_RNN_DBG")) : 0;
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        CK(cudaMemsetAsync(counter, 0, sizeof(unsigned), st));
+        CUtensorMap tx = make_tmap_bf16_2d(T[in], (int64_t)S * B, E, 128);
+        RnnPersistArgs r = ra;
+        r.out = (__nv_bfloat16*)T[me];
+        rnn_persist(kind, bn, tx, t_h0, t_h1, t_w, r, tiles, mt, st);
+      };
+      op.n_kernels = 1;
+    } else if (tc) {
       // fused step (kernels/gemm_tc.cu EPI_LSTM/EPI_GRU): K = [x_t (E, padded to Ep) | h_{t-1} (H)],
       // 4 gate blocks per tile; no G_x buffer and no separate input-projection GEMM
       const int bn = rnn_step_bn(kind, B, H, sms);
