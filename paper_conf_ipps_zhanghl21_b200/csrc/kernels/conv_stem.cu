@@ -4,8 +4,9 @@
 // TMA's 16-byte minimum, and the explicit im2col buffer (M x 152 bf16 = 244 MB at batch 64) made the
 // stem HBM-bound at ~0.5 ms.  Here the im2col happens in shared memory instead:
 //
-//   tile   = one output row (n, ho): Wo <= 128 pixels = the UMMA M rows (rows >= Wo stay zero)
-//   patch  = the kh input rows that tile reads: nbx TMA boxes of [kh rows x 256 elements] whose
+//   tile   = rp consecutive output rows of one image (rp = 128 / Wo: one row at 224x224, eight at
+//            32x32): rp * Wo <= 128 pixels = the UMMA M rows (the rest stay zero)
+//   patch  = the (rp-1)*stride + kh input rows that tile reads: nbx TMA boxes of [rows x 256 elements] whose
 //            starts are STEP = 256 - 24 elements apart, so every pixel's 24-element window lies
 //            inside one box (3 requests per tile for the stem; TMA's per-request cost, not bytes,
 //            bounded a row-per-request version).  Out-of-image rows / columns, including the
@@ -53,6 +54,9 @@ struct StemGeom {
   int rowb;    // bytes per box row = BOXW * 2
   int bw, nbx; // box width (BOXW) and boxes per tile
   int ksteps;  // UMMA K steps (16) covering kh * SEG
+  int rp;      // output rows per tile
+  int bh;      // patch box rows = (rp - 1) * stride + kh
+  int tpi;     // tiles per image = ceil(Ho / rp)
   int np;      // patch buffers in flight (prefetch depth; HBM latency is the bound with 2)
   int act;
   int dbg;     // micro-benchmark switches (DUET_STEM_DBG): 1 skip build, 2 skip MMA, 4 skip stores,
@@ -79,7 +83,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint8_t* sA = smem;                                  // 2 x A_BYTES
   uint8_t* sW = sA + 2 * A_BYTES;                      // ATOMS x CO x 128 B
   uint8_t* sP = sW + ATOMS * CO * 128;                 // np x nbx x kh x rowb
-  const int bbytes = g.kh * g.rowb;                    // one box
+  const int bbytes = g.bh * g.rowb;                    // one box
   const int pbytes = g.nbx * bbytes;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sP + g.np * pbytes);
   uint64_t* patch_full = bars;          // [np] TMA tx
@@ -93,7 +97,7 @@ __global__ void __launch_bounds__(THREADS, 1)
 
   const int warp = ptx::warp_id();
   const int lane = threadIdx.x & 31;
-  const int tiles = g.N * g.Ho;
+  const int tiles = g.N * g.tpi;
   const int my_tiles = blockIdx.x < tiles ? (tiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
   const uint32_t patch_tx = (uint32_t)pbytes;
 
@@ -132,7 +136,7 @@ __global__ void __launch_bounds__(THREADS, 1)
 
   auto issue_patch = [&](int i) {  // TMA of local tile i's input rows into patch buffer i % np
     const int tile = blockIdx.x + i * gridDim.x;
-    const int n = tile / g.Ho, ho = tile % g.Ho;
+    const int n = tile / g.tpi, ho = (tile % g.tpi) * g.rp;
     const int pb = i % g.np;
     uint8_t* dst = sP + pb * pbytes;
     if (g.dbg & 8) {
@@ -147,18 +151,20 @@ __global__ void __launch_bounds__(THREADS, 1)
   if (warp < NB) {
     // ---------------- builders: patch -> A (im2col in shared memory) ----------------
     const int m = threadIdx.x & (ROWS - 1);  // output pixel (UMMA row) of this thread
+    const int rr = m / g.Wo, wo = m % g.Wo;   // output row within the tile, column
     const int kh_half = (g.kh + 1) / 2;
     const int r0 = threadIdx.x < ROWS ? 0 : kh_half, r1 = threadIdx.x < ROWS ? kh_half : g.kh;
     if (threadIdx.x == 0)
       for (int i = 0; i < g.np && i < my_tiles; ++i) issue_patch(i);
-    // this pixel's window: box b, element offset o (even: 4-byte aligned words)
-    const int off = g.stride * g.C * m + g.L - g.pad * g.C - g.d;
-    const int src0 = (off / STEP) * bbytes + (off % STEP) * 2;
+    // this pixel's window: box b, element offset o (even: 4-byte aligned words), box row rr*stride
+    const int off = g.stride * g.C * wo + g.L - g.pad * g.C - g.d;
+    const int src0 = (off / STEP) * bbytes + (off % STEP) * 2 + rr * g.stride * g.rowb;
+    const bool live_px = m < g.rp * g.Wo;
     for (int i = 0; i < my_tiles; ++i) {
       const int p = i & 1, pb = i % g.np;
       ptx::mbar_wait(&patch_full[pb], (i / g.np) & 1);
       if (i >= 2) ptx::mbar_wait(&a_empty[p], ((i >> 1) - 1) & 1);
-      if (m < g.Wo && !(g.dbg & 1)) {
+      if (live_px && !(g.dbg & 1)) {
         const uint8_t* prow = sP + pb * pbytes + src0;
         uint8_t* arow = sA + p * A_BYTES + m * 128;
 #pragma unroll 4
@@ -223,8 +229,10 @@ __global__ void __launch_bounds__(THREADS, 1)
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&t_empty[b]);
-      if (m < g.Wo && !(g.dbg & 4)) {
-        __nv_bfloat16* out = y + ((int64_t)tile * g.Wo + m) * CO;
+      const int n = tile / g.tpi, ho0 = (tile % g.tpi) * g.rp;
+      if (m < g.rp * g.Wo && ho0 + m / g.Wo < g.Ho && !(g.dbg & 4)) {
+        // the tile's rows are consecutive in NHWC: pixel m of the tile is pixel m after (n, ho0, 0)
+        __nv_bfloat16* out = y + (((int64_t)n * g.Ho + ho0) * g.Wo + m) * CO;
 #pragma unroll
         for (int c = 0; c < CO; c += 16) {
           float t[16];
@@ -244,7 +252,10 @@ __global__ void __launch_bounds__(THREADS, 1)
 }
 
 StemGeom geom(const ConvShape& s, int act) {
-  StemGeom g{s.N, s.H, s.W, s.C, s.Co, s.kh, s.kw, s.stride, s.pad, s.Ho, s.Wo, 0, 0, 0, 0, 0, 0, 2, act, 0};
+  StemGeom g{s.N, s.H, s.W, s.C, s.Co, s.kh, s.kw, s.stride, s.pad, s.Ho, s.Wo, 0, 0, 0, 0, 0, 0, 0, 0, 0, 2, act, 0};
+  g.rp = std::max(1, std::min(ROWS / std::max(1, s.Wo), s.Ho));
+  g.bh = (g.rp - 1) * s.stride + s.kh;
+  g.tpi = (s.Ho + g.rp - 1) / g.rp;
   g.dbg = getenv("DUET_STEM_DBG") ? atoi(getenv("DUET_STEM_DBG")) : 0;
   g.d = (s.pad * s.C) & 1;
   g.L = (s.pad * s.C + g.d + 7) / 8 * 8;
@@ -256,14 +267,14 @@ StemGeom geom(const ConvShape& s, int act) {
   g.nbx = (s.stride * s.C * (s.Wo - 1) + g.L - s.pad * s.C - g.d) / STEP + 1;
   g.ksteps = (s.kh * SEG + 15) / 16;
   const size_t fixed = 1024 + 2 * A_BYTES + (size_t)ATOMS * s.Co * 128 + (NPMAX + 9) * 8 + (size_t)s.Co * 4;
-  const size_t pb = (size_t)g.nbx * s.kh * g.rowb;
+  const size_t pb = (size_t)g.nbx * g.bh * g.rowb;
   g.np = (int)std::min<size_t>(NPMAX, (227 * 1024 - fixed) / pb);
   if (g.np < 2) g.np = 2;  // (conv_stem_ok rejects shapes that do not fit two)
   return g;
 }
 
 size_t stem_smem(const StemGeom& g) {
-  return 1024 + 2 * A_BYTES + (size_t)ATOMS * g.Co * 128 + (size_t)g.np * g.nbx * g.kh * g.rowb + (NPMAX + 9) * 8 +
+  return 1024 + 2 * A_BYTES + (size_t)ATOMS * g.Co * 128 + (size_t)g.np * g.nbx * g.bh * g.rowb + (NPMAX + 9) * 8 +
          (size_t)g.Co * 4;
 }
 
@@ -271,6 +282,7 @@ size_t stem_smem(const StemGeom& g) {
 
 bool conv_stem_ok(const ConvShape& s) {
   if (s.kh > KPAD / SEG || s.Wo > ROWS || s.Co % 16 || s.Co < 16 || s.Co > 128) return false;
+  if ((std::min(ROWS / std::max(1, s.Wo), s.Ho) - 1) * s.stride + s.kh > 256) return false;  // TMA box rows
   if ((s.pad * s.C) % 2 + s.kw * s.C > SEG) return false;      // window fits a segment
   if ((s.stride * s.C) % 2) return false;                        // 4-byte aligned windows
   if ((s.W * s.C) % 8) return false;                             // TMA row pitch (16 B)
@@ -293,14 +305,14 @@ void conv_stem(const CUtensorMap& tw, const void* x, const float* bias, void* y,
   CUtensorMap tx;
   cuuint64_t dims[3] = {(cuuint64_t)s.W * s.C, (cuuint64_t)s.H, (cuuint64_t)s.N};
   cuuint64_t strides[2] = {(cuuint64_t)s.W * s.C * 2, (cuuint64_t)s.H * s.W * s.C * 2};
-  cuuint32_t box[3] = {(cuuint32_t)BOXW, (cuuint32_t)s.kh, 1};
+  cuuint32_t box[3] = {(cuuint32_t)BOXW, (cuuint32_t)g.bh, 1};
   cuuint32_t estr[3] = {1, 1, 1};
   CUresult r = tmap_encode_tiled()(&tx, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(x), dims, strides, box,
                                    estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) fail(DUET_ECUDA, "conv_stem: image tensor map (" + std::to_string((int)r) + ")");
   const size_t smem = stem_smem(g);
-  const int tiles = s.N * s.Ho;
+  const int tiles = s.N * g.tpi;
   int dev = 0;
   CK(cudaGetDevice(&dev));
   const int grid = std::min(tiles, num_sms(dev));

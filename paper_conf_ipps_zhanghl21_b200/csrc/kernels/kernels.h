@@ -62,21 +62,24 @@ void gemm_tc_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, in
 void rnn_pack(int kind, const void* Wih, const void* Whh, const float* bih, const float* bhh, void* Wcat, float* bias,
               int E, int Ep, int H, int U, int BN, int tiles, cudaStream_t st);
 
-// Persistent fused recurrence (rnn_persist.cu): all S steps in one cooperative launch, grid =
-// (tiles_n, tiles_m) CTAs of 128 rows x bn packed gate columns (the rnn_pack layout with U = bn/4).
+// Persistent fused recurrence (rnn_persist.cu): all S steps in one cooperative launch of `grid`
+// CTAs over tiles_n x tiles_m tiles of 128 rows x bn packed gate columns (the rnn_pack layout with
+// U = bn/4); grid < tiles -> each CTA owns several tiles (state kept in global memory).
 struct RnnPersistArgs {
   const float* bias = nullptr;        // [tiles_n * bn] packed gate bias
   __nv_bfloat16* hbuf[2] = {nullptr, nullptr};  // [B, H] ping-pong h_t (t even -> 0, odd -> 1)
   __nv_bfloat16* out = nullptr;       // [B, H] h_S
   unsigned* counter = nullptr;        // grid-barrier counter, zeroed before each launch
-  int S = 0, B = 0, H = 0, kx = 0, kh = 0, n_cta = 0;
+  float* c_state = nullptr;           // LSTM cell state [B, H] fp32 (several tiles per CTA only)
+  int S = 0, B = 0, H = 0, kx = 0, kh = 0;
+  int tiles_n = 0, tiles_m = 0;       // tile grid: n (gate-block tiles of bn columns) fastest
   int dbg = 0;                        // 1 = per-step timestamps (g_rp_trace)
   int stages = 0;                     // A-ring depth (set by the launcher)
 };
 // tx: [S*B, E] (box 128 rows), th0/th1: hbuf[0/1] [B, H] (box 128 rows), tw: packed weights
 // [tiles_n*bn, kx*64 + H] (box bn rows).
 void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1,
-                 const CUtensorMap& tw, const RnnPersistArgs& a, int tiles_n, int tiles_m, cudaStream_t st);
+                 const CUtensorMap& tw, const RnnPersistArgs& a, int grid, cudaStream_t st);
 
 // CTA-pair GEMM (gemm_tc2.cu): 256 x bn tiles, bn in {64,128,256}; W map box rows = bn / 2.
 int tc2_pick_bn(int M, int N, int K, int num_sms);

@@ -104,13 +104,38 @@ __device__ __forceinline__ void wait_sleep(uint64_t* bar, uint32_t parity) {
   }
 }
 
+// one LSTM / GRU cell from its four gate pre-activations; `st` = c (LSTM) or h_{t-1} (GRU), updated
+template <int KIND>
+__device__ __forceinline__ float cell(float a0, float a1, float a2, float a3, float& st) {
+  if constexpr (KIND == EPI_LSTM) {
+    const float ig = rsig(a0), fg = rsig(a1), gg = rtanh(a2), og = rsig(a3);
+    st = fg * st + ig * gg;
+    return og * rtanh(st);
+  } else {
+    const float r = rsig(a0), z = rsig(a1);
+    const float n = rtanh(a2 + r * a3);  // (W_in x + b_in) + r * (W_hn h + b_hn)
+    const float h = (1.0f - z) * n + z * st;
+    st = h;
+    return h;
+  }
+}
+__device__ __forceinline__ void store_bf16x8(__nv_bfloat16* dst, const float* h) {
+  uint32_t w[4];
+#pragma unroll
+  for (int p = 0; p < 4; ++p) {
+    __nv_bfloat162 b2 = __floats2bfloat162_rn(h[2 * p], h[2 * p + 1]);
+    w[p] = *reinterpret_cast<uint32_t*>(&b2);
+  }
+  *reinterpret_cast<uint4*>(dst) = make_uint4(w[0], w[1], w[2], w[3]);
+}
+
 template <int N>
 __device__ __forceinline__ void tmem_ld_n(uint32_t taddr, float* v) {
   if constexpr (N == 16) ptx::tmem_ld16(taddr, v);
   else ptx::tmem_ld8(taddr, v);
 }
 
-template <int BN, int KIND, bool WRES>
+template <int BN, int KIND, bool WRES, bool MULTI>
 __global__ void __launch_bounds__(kRThreads, 1)
     rnn_persist_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmH0,
                        const __grid_constant__ CUtensorMap tmH1, const __grid_constant__ CUtensorMap tmW,
@@ -132,11 +157,15 @@ __global__ void __launch_bounds__(kRThreads, 1)
 
   const int warp = ptx::warp_id();
   const int lane = threadIdx.x & 31;
-  const int n0 = blockIdx.x * BN;
-  const int m0 = blockIdx.y * RBM;
   const int S = a.S, kx = a.kx, kh = a.kh;
-  const int cta = blockIdx.y * gridDim.x + blockIdx.x;
-  unsigned long long* trace = (a.dbg & 1) && cta < 128 ? g_rp_trace + (size_t)cta * 64 * 16 : nullptr;
+  // static tile assignment: tile = blockIdx.x + i * gridDim.x (n-tile fastest); one tile per CTA
+  // unless MULTI
+  const int n_tiles = a.tiles_n * a.tiles_m;
+  const int my_tiles = MULTI ? (n_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 1;
+  auto tile_n0 = [&](int i) { return ((int)(blockIdx.x + i * gridDim.x) % a.tiles_n) * BN; };
+  auto tile_m0 = [&](int i) { return ((int)(blockIdx.x + i * gridDim.x) / a.tiles_n) * RBM; };
+  const int cta = blockIdx.x;
+  unsigned long long* trace = (a.dbg & 1) && !MULTI && cta < 128 ? g_rp_trace + (size_t)cta * 64 * 16 : nullptr;
 
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tmX);
@@ -158,41 +187,46 @@ __global__ void __launch_bounds__(kRThreads, 1)
     ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
     ptx::tmem_relinquish();
   }
-  for (int c = (int)threadIdx.x - 64; c >= 0 && c < BN; c += 32 * kREpiWarps) s_bias[c] = a.bias[n0 + c];
+  if (!MULTI)
+    for (int c = (int)threadIdx.x - 64; c >= 0 && c < BN; c += 32 * kREpiWarps) s_bias[c] = a.bias[tile_n0(0) + c];
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
   if (warp == 0) {
-    // ---------------- TMA producer ----------------
+    // ---------------- A producer: x_t blocks, [grid barrier], h_{t-1} blocks per (step, tile) ------
     int g = 0;
     for (int t = 0; t < S; ++t) {
       const int nkb = kx + (t > 0 ? kh : 0);  // h_{-1} = 0: step 0 has only the x part
       const CUtensorMap* th = ((t - 1) & 1) ? &tmH1 : &tmH0;
-      for (int j = 0; j < nkb; ++j, ++g) {
-        const int s = g % STAGES;
-        if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
-        if (j == kx) {
-          // h_{t-1}: wait until every CTA has released its slice (grid barrier), then order the
-          // generic-proxy writes it observed before this thread's async-proxy (TMA) reads
-          if (lane == 0) {
-            const unsigned target = (unsigned)t * (unsigned)a.n_cta * kREpiWarps;
-            while (ld_acquire_gpu(a.counter) < target) {
+      for (int i = 0; i < my_tiles; ++i) {
+        const int m0 = tile_m0(i);
+        for (int j = 0; j < nkb; ++j, ++g) {
+          const int s = g % STAGES;
+          if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
+          if (j == kx && i == 0) {
+            // h_{t-1}: wait until every epilogue warp of every tile has released its slice (grid
+            // barrier), then order the generic-proxy writes it observed before this thread's
+            // async-proxy (TMA) reads
+            if (lane == 0) {
+              const unsigned target = (unsigned)t * (unsigned)n_tiles * kREpiWarps;
+              while (ld_acquire_gpu(a.counter) < target) {
+              }
+              fence_proxy_async_global();
+              if (trace && t < 64) trace[t * 16 + 0] = rp_gtimer();
             }
-            fence_proxy_async_global();
-            if (trace && t < 64) trace[t * 16 + 0] = rp_gtimer();
+            __syncwarp();
+          }
+          if (lane == 0) {
+            ptx::mbar_arrive_expect_tx(&full[s], R_A_BYTES);
+            if (j < kx)
+              ptx::tma_load_2d(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
+            else
+              ptx::tma_load_2d(th, &full[s], sA + s * R_A_BYTES, (j - kx) * RBK, m0);
           }
           __syncwarp();
         }
-        if (lane == 0) {
-          ptx::mbar_arrive_expect_tx(&full[s], R_A_BYTES);
-          if (j < kx)
-            ptx::tma_load_2d(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
-          else
-            ptx::tma_load_2d(th, &full[s], sA + s * R_A_BYTES, (j - kx) * RBK, m0);
-        }
-        __syncwarp();
       }
     }
   } else if (warp == kWWarp) {
@@ -201,22 +235,25 @@ __global__ void __launch_bounds__(kRThreads, 1)
       // resident: every packed weight block of this tile, loaded once for the whole sequence
       if (lane == 0) {
         ptx::mbar_arrive_expect_tx(w_full, (uint32_t)(nkw * C::B_BYTES));
-        for (int j = 0; j < nkw; ++j) ptx::tma_load_2d(&tmW, w_full, sB + j * C::B_BYTES, j * RBK, n0);
+        for (int j = 0; j < nkw; ++j) ptx::tma_load_2d(&tmW, w_full, sB + j * C::B_BYTES, j * RBK, tile_n0(0));
       }
     } else {
       // streamed ahead of the barrier in the A ring's stage order
       int g = 0;
       for (int t = 0; t < S; ++t) {
         const int nkb = kx + (t > 0 ? kh : 0);
-        for (int j = 0; j < nkb; ++j, ++g) {
-          const int s = g % STAGES;
-          if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
-          if (lane == 0) {
-            ptx::mbar_arrive_expect_tx(&full[s], C::B_BYTES);
-            // packed weight columns: [x part (kx blocks) | h part (kh blocks)] -> column block j
-            ptx::tma_load_2d(&tmW, &full[s], sB + s * C::B_BYTES, j * RBK, n0);
+        for (int i = 0; i < my_tiles; ++i) {
+          const int n0 = tile_n0(i);
+          for (int j = 0; j < nkb; ++j, ++g) {
+            const int s = g % STAGES;
+            if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
+            if (lane == 0) {
+              ptx::mbar_arrive_expect_tx(&full[s], C::B_BYTES);
+              // packed weight columns: [x part (kx blocks) | h part (kh blocks)] -> column block j
+              ptx::tma_load_2d(&tmW, &full[s], sB + s * C::B_BYTES, j * RBK, n0);
+            }
+            __syncwarp();
           }
-          __syncwarp();
         }
       }
     }
@@ -226,102 +263,156 @@ __global__ void __launch_bounds__(kRThreads, 1)
     const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
     const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
     if constexpr (WRES) wait_sleep(w_full, 0);
-    int g = 0;
+    int g = 0, u = 0;  // u: work unit (step, tile) counter -> accumulator buffer u & 1
     for (int t = 0; t < S; ++t) {
-      const int buf = t & 1;
-      if (t >= 2) wait_sleep(&tempty[buf], ((t >> 1) - 1) & 1);
-      ptx::tc_fence_after();
-      const uint32_t d = tmem + (uint32_t)(buf * BN);
       const int nkb = kx + (t > 0 ? kh : 0);
-      for (int j = 0; j < nkb; ++j, ++g) {
-        const int s = g % STAGES;
-        wait_sleep(&full[s], (g / STAGES) & 1);
+      for (int i = 0; i < my_tiles; ++i, ++u) {
+        const int buf = u & 1;
+        if (u >= 2) wait_sleep(&tempty[buf], ((u >> 1) - 1) & 1);
         ptx::tc_fence_after();
-        if (trace && t < 64 && lane == 0) {
-          if (j == 0) trace[t * 16 + 1] = rp_gtimer();
-          if (j == kx) trace[t * 16 + 4] = rp_gtimer();  // first h stage landed
-        }
-        const uint64_t da = da0 + (uint64_t)((s * R_A_BYTES) >> 4);
-        const uint64_t db = db0 + (uint64_t)(((WRES ? j : s) * C::B_BYTES) >> 4);
-        if (!(a.dbg & 16))
+        const uint32_t d = tmem + (uint32_t)(buf * BN);
+        for (int j = 0; j < nkb; ++j, ++g) {
+          const int s = g % STAGES;
+          wait_sleep(&full[s], (g / STAGES) & 1);
+          ptx::tc_fence_after();
+          if (trace && t < 64 && lane == 0) {
+            if (j == 0) trace[t * 16 + 1] = rp_gtimer();
+            if (j == kx) trace[t * 16 + 4] = rp_gtimer();  // first h stage landed
+          }
+          const uint64_t da = da0 + (uint64_t)((s * R_A_BYTES) >> 4);
+          const uint64_t db = db0 + (uint64_t)(((WRES ? j : s) * C::B_BYTES) >> 4);
+          if (!(a.dbg & 16))
 #pragma unroll
-          for (int k = 0; k < RBK / 16; ++k) ptx::umma_bf16_elect(d, da + 2 * k, db + 2 * k, idesc, (j | k) != 0);
-        ptx::umma_commit_elect(&empty[s]);
+            for (int k = 0; k < RBK / 16; ++k) ptx::umma_bf16_elect(d, da + 2 * k, db + 2 * k, idesc, (j | k) != 0);
+          ptx::umma_commit_elect(&empty[s]);
+        }
+        ptx::umma_commit_elect(&tfull[buf]);
+        if (trace && t < 64 && lane == 0) trace[t * 16 + 5] = rp_gtimer();  // last UMMA issued
       }
-      ptx::umma_commit_elect(&tfull[buf]);
-      if (trace && t < 64 && lane == 0) trace[t * 16 + 5] = rp_gtimer();  // last UMMA issued
     }
   } else {
     // ---------------- epilogue: gates, cell, h_t ----------------
     constexpr int U = C::U, UH = C::UH;
     const int q = warp & 3;
     const int half = (warp - 2) >> 2;
-    const int row = m0 + q * 32 + lane;
     const int H = a.H;
-    const int unit0 = blockIdx.x * U + half * UH;
-    const int nv = min(UH, H - unit0);  // multiple of 8 (H % 8 == 0)
-    const bool live = row < a.B && nv > 0;
-    float bias[4][UH];  // this thread's gate biases, in registers for the whole sequence
+    if constexpr (!MULTI) {
+      // one tile for the whole sequence: bias and the recurrent state (LSTM c, GRU h in fp32) stay
+      // in registers
+      const int row = tile_m0(0) + q * 32 + lane;
+      const int unit0 = (tile_n0(0) / BN) * U + half * UH;
+      const int nv = min(UH, H - unit0);  // multiple of 8 (H % 8 == 0)
+      const bool live = row < a.B && nv > 0;
+      float bias[4][UH];
 #pragma unroll
-    for (int g = 0; g < 4; ++g)
+      for (int g = 0; g < 4; ++g)
 #pragma unroll
-      for (int i = 0; i < UH; ++i) bias[g][i] = s_bias[g * U + half * UH + i];
-    float state[UH];  // LSTM: c_{t-1}; GRU: h_{t-1} (fp32)
+        for (int i = 0; i < UH; ++i) bias[g][i] = s_bias[g * U + half * UH + i];
+      float state[UH];  // LSTM: c_{t-1}; GRU: h_{t-1} (fp32)
 #pragma unroll
-    for (int i = 0; i < UH; ++i) state[i] = 0.0f;
-    for (int t = 0; t < S; ++t) {
-      const int buf = t & 1;
-      wait_sleep(&tfull[buf], (t >> 1) & 1);
-      ptx::tc_fence_after();
-      if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 2] = rp_gtimer();
-      const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
-      float acc[4][UH];
+      for (int i = 0; i < UH; ++i) state[i] = 0.0f;
+      for (int t = 0; t < S; ++t) {
+        const int buf = t & 1;
+        wait_sleep(&tfull[buf], (t >> 1) & 1);
+        ptx::tc_fence_after();
+        if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 2] = rp_gtimer();
+        const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
+        float acc[4][UH];
 #pragma unroll
-      for (int g = 0; g < 4; ++g) tmem_ld_n<UH>(tq + g * U + half * UH, acc[g]);
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&tempty[buf]);  // accumulator buffer free for step t+2
-      if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 6] = rp_gtimer();  // TMEM read
-      float h[UH];
+        for (int g = 0; g < 4; ++g) tmem_ld_n<UH>(tq + g * U + half * UH, acc[g]);
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&tempty[buf]);  // accumulator buffer free for step t+2
+        if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 6] = rp_gtimer();  // TMEM read
+        float h[UH];
 #pragma unroll
-      for (int i = 0; i < UH; ++i) {
-        const float a0 = acc[0][i] + bias[0][i], a1 = acc[1][i] + bias[1][i];
-        const float a2 = acc[2][i] + bias[2][i], a3 = acc[3][i] + bias[3][i];
-        if constexpr (KIND == EPI_LSTM) {
-          const float ig = rsig(a0), fg = rsig(a1), gg = rtanh(a2), og = rsig(a3);
-          state[i] = fg * state[i] + ig * gg;
-          h[i] = og * rtanh(state[i]);
-        } else {
-          const float r = rsig(a0), z = rsig(a1);
-          const float n = rtanh(a2 + r * a3);  // (W_in x + b_in) + r * (W_hn h + b_hn)
-          h[i] = (1.0f - z) * n + z * state[i];
-          state[i] = h[i];
+        for (int i = 0; i < UH; ++i) h[i] = cell<KIND>(acc[0][i] + bias[0][i], acc[1][i] + bias[1][i],
+                                                        acc[2][i] + bias[2][i], acc[3][i] + bias[3][i], state[i]);
+        __nv_bfloat16* dst = (t == S - 1 ? a.out : a.hbuf[buf]) + (size_t)row * H + unit0;
+        if (live) {
+#pragma unroll
+          for (int v = 0; v < UH / 8; ++v)
+            if (v * 8 < nv) store_bf16x8(dst + 8 * v, h + 8 * v);
+        }
+        if (trace && t < 64 && lane == 0) trace[t * 16 + 6 + warp] = rp_gtimer();  // [8..15] math + stores
+        if (t < S - 1) {
+          // each warp releases its own slice of h_t (no CTA-wide barrier): the generic-proxy stores
+          // are ordered before the release-add by __syncwarp; the consumer acquires the counter and
+          // issues fence.proxy.async before its TMA reads
+          fence_proxy_async_global();
+          __syncwarp();
+          if (lane == 0) red_release_gpu_add(a.counter, 1u);
+          if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 3] = rp_gtimer();
         }
       }
-      __nv_bfloat16* dst = (t == S - 1 ? a.out : a.hbuf[buf]) + (size_t)row * H + unit0;
-      if (live) {
+    } else {
+      // several tiles per CTA: the state lives in global memory (LSTM c fp32 [B, H]; GRU reads
+      // h_{t-1} back in bf16, as the per-step kernel does); chunks of 8 units bound the registers
+      int u = 0;
+      for (int t = 0; t < S; ++t) {
+        for (int i = 0; i < my_tiles; ++i, ++u) {
+          const int buf = u & 1;
+          const int row = tile_m0(i) + q * 32 + lane;
+          const int n0 = tile_n0(i);
+          wait_sleep(&tfull[buf], (u >> 1) & 1);
+          ptx::tc_fence_after();
+          const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
+          float acc[UH / 8][4][8];
 #pragma unroll
-        for (int v = 0; v < UH / 8; ++v) {
-          if (v * 8 < nv) {
-            uint32_t w[4];
+          for (int c = 0; c < UH / 8; ++c)
 #pragma unroll
-            for (int p = 0; p < 4; ++p) {
-              __nv_bfloat162 b2 = __floats2bfloat162_rn(h[v * 8 + 2 * p], h[v * 8 + 2 * p + 1]);
-              w[p] = *reinterpret_cast<uint32_t*>(&b2);
+            for (int g = 0; g < 4; ++g) ptx::tmem_ld8(tq + g * U + half * UH + 8 * c, acc[c][g]);
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive(&tempty[buf]);
+          __nv_bfloat16* dst = (t == S - 1 ? a.out : a.hbuf[t & 1]);
+          const __nv_bfloat16* hprev = a.hbuf[(t - 1) & 1];
+#pragma unroll
+          for (int c = 0; c < UH / 8; ++c) {
+            const int unit = (n0 / BN) * U + half * UH + 8 * c;
+            if (row >= a.B || unit >= H) continue;
+            const size_t off = (size_t)row * H + unit;
+            float st[8];
+            if constexpr (KIND == EPI_LSTM) {
+              if (t == 0) {
+#pragma unroll
+                for (int e = 0; e < 8; ++e) st[e] = 0.0f;
+              } else {
+                const float4 c0 = *reinterpret_cast<const float4*>(a.c_state + off);
+                const float4 c1 = *reinterpret_cast<const float4*>(a.c_state + off + 4);
+                st[0] = c0.x, st[1] = c0.y, st[2] = c0.z, st[3] = c0.w;
+                st[4] = c1.x, st[5] = c1.y, st[6] = c1.z, st[7] = c1.w;
+              }
+            } else {
+              if (t == 0) {
+#pragma unroll
+                for (int e = 0; e < 8; ++e) st[e] = 0.0f;
+              } else {
+                const uint4 raw = *reinterpret_cast<const uint4*>(hprev + off);
+                const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&raw);
+#pragma unroll
+                for (int e = 0; e < 8; ++e) st[e] = __bfloat162float(hv[e]);
+              }
             }
-            reinterpret_cast<uint4*>(dst)[v] = make_uint4(w[0], w[1], w[2], w[3]);
+            const int cb = n0 + half * UH + 8 * c;  // packed bias column of gate block 0
+            float h[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e)
+              h[e] = cell<KIND>(acc[c][0][e] + __ldg(a.bias + cb + e), acc[c][1][e] + __ldg(a.bias + cb + U + e),
+                                acc[c][2][e] + __ldg(a.bias + cb + 2 * U + e),
+                                acc[c][3][e] + __ldg(a.bias + cb + 3 * U + e), st[e]);
+            if constexpr (KIND == EPI_LSTM) {
+              *reinterpret_cast<float4*>(a.c_state + off) = make_float4(st[0], st[1], st[2], st[3]);
+              *reinterpret_cast<float4*>(a.c_state + off + 4) = make_float4(st[4], st[5], st[6], st[7]);
+            }
+            store_bf16x8(dst + off, h);
+          }
+          if (t < S - 1) {
+            fence_proxy_async_global();
+            __syncwarp();
+            if (lane == 0) red_release_gpu_add(a.counter, 1u);
           }
         }
-      }
-      if (trace && t < 64 && lane == 0) trace[t * 16 + 6 + warp] = rp_gtimer();  // [8..15] math + stores
-      if (t < S - 1) {
-        // each warp releases its own slice of h_t (no CTA-wide barrier): the generic-proxy stores
-        // are ordered before the release-add by __syncwarp; the consumer acquires the counter and
-        // issues fence.proxy.async before its TMA reads
-        if (!(a.dbg & 2)) fence_proxy_async_global();
-        __syncwarp();
-        if (lane == 0) red_release_gpu_add(a.counter, 1u);
-        if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 3] = rp_gtimer();
       }
     }
   }
@@ -333,11 +424,11 @@ __global__ void __launch_bounds__(kRThreads, 1)
   }
 }
 
-template <int BN, int KIND, bool WRES>
+template <int BN, int KIND, bool WRES, bool MULTI>
 void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1, const CUtensorMap& tw,
-               const RnnPersistArgs& a, dim3 grid, cudaStream_t st) {
+               const RnnPersistArgs& a, int grid, cudaStream_t st) {
   using C = RCfg<BN>;
-  auto kern = rnn_persist_kernel<BN, KIND, WRES>;
+  auto kern = rnn_persist_kernel<BN, KIND, WRES, MULTI>;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kRSmemBudget));
@@ -345,7 +436,7 @@ void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap&
   }
   const int smem = a.stages * R_A_BYTES + (WRES ? a.kx + a.kh : a.stages) * C::B_BYTES + C::EXTRA;
   cudaLaunchConfig_t cfg{};
-  cfg.gridDim = grid;
+  cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(kRThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
@@ -359,7 +450,13 @@ void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap&
 
 template <int BN, int KIND>
 void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1, const CUtensorMap& tw,
-                   RnnPersistArgs a, dim3 grid, cudaStream_t st) {
+                   RnnPersistArgs a, int grid, cudaStream_t st) {
+  const bool multi = a.tiles_n * a.tiles_m > grid;
+  if (multi) {  // several tiles per CTA: W changes per tile, so it is streamed
+    a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
+    if (a.stages > 10) a.stages = 10;
+    return launch_rp<BN, KIND, false, true>(tx, th0, th1, tw, a, grid, st);
+  }
   static const int wres_env = getenv("DUET_RNN_WRES") ? atoi(getenv("DUET_RNN_WRES")) : 1;
   bool wres = false;
   a.stages = rp_plan(BN, a.kx + a.kh, &wres);
@@ -368,15 +465,15 @@ void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensor
     a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
     if (a.stages > 10) a.stages = 10;
   }
-  if (wres) return launch_rp<BN, KIND, true>(tx, th0, th1, tw, a, grid, st);
-  launch_rp<BN, KIND, false>(tx, th0, th1, tw, a, grid, st);
+  if (wres) return launch_rp<BN, KIND, true, false>(tx, th0, th1, tw, a, grid, st);
+  launch_rp<BN, KIND, false, false>(tx, th0, th1, tw, a, grid, st);
 }
 
 }  // namespace
 
 void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1,
-                 const CUtensorMap& tw, const RnnPersistArgs& a, int tiles_n, int tiles_m, cudaStream_t st) {
-  const dim3 grid(tiles_n, tiles_m);
+                 const CUtensorMap& tw, const RnnPersistArgs& a_in, int grid, cudaStream_t st) {
+  RnnPersistArgs a = a_in;
   if (kind == EPI_LSTM && bn == 64) return launch_rp_any<64, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_LSTM && bn == 128) return launch_rp_any<128, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_GRU && bn == 64) return launch_rp_any<64, EPI_GRU>(tx, th0, th1, tw, a, grid, st);

@@ -190,9 +190,72 @@ __global__ void __launch_bounds__(256) rnn_step_simt_kernel(const float* __restr
 
 }  // namespace
 
+// Narrow linear (N <= 8 outputs, the per-branch logit heads): one warp per row, the row streamed
+// once with 16-byte loads (HBM-bound: M*K*esize bytes), W rows from L1, warp-shuffle reduction.
+template <typename TX, typename TW>
+__global__ void __launch_bounds__(256) linear_narrow_kernel(const TX* __restrict__ X, const TW* __restrict__ W,
+                                                            const float* __restrict__ bias, void* __restrict__ Y,
+                                                            int y_bf16, int M, int N, int K, int act) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
+  const int warps = blockDim.x >> 5, lane = threadIdx.x & 31;
+  constexpr int V = 16 / sizeof(TX);  // elements per 16-byte vector of X
+  const bool vec = (K % V == 0) && ((uintptr_t)X % 16 == 0);
+  for (int m = blockIdx.x * warps + (threadIdx.x >> 5); m < M; m += gridDim.x * warps) {
+    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    const TX* xr = X + (int64_t)m * K;
+    if (vec) {
+      for (int k0 = lane * V; k0 < K; k0 += 32 * V) {
+        const uint4 raw = __ldcs(reinterpret_cast<const uint4*>(xr + k0));
+        const TX* xv = reinterpret_cast<const TX*>(&raw);
+#pragma unroll
+        for (int n = 0; n < 8; ++n) {
+          if (n >= N) break;
+          const TW* wr = W + (int64_t)n * K + k0;
+#pragma unroll
+          for (int i = 0; i < V; ++i) acc[n] = fmaf(to_f(xv[i]), to_f(__ldg(wr + i)), acc[n]);
+        }
+      }
+    } else {
+      for (int k = lane; k < K; k += 32) {
+        const float xv = to_f(xr[k]);
+#pragma unroll
+        for (int n = 0; n < 8; ++n)
+          if (n < N) acc[n] = fmaf(xv, to_f(W[(int64_t)n * K + k]), acc[n]);
+      }
+    }
+#pragma unroll
+    for (int n = 0; n < 8; ++n) {
+      if (n >= N) break;
+      const float v = warp_sum(acc[n]);
+      if (lane == 0) {
+        const float o = apply_act(v + (bias ? bias[n] : 0.0f), act);
+        if (y_bf16) reinterpret_cast<__nv_bfloat16*>(Y)[(int64_t)m * N + n] = __float2bfloat16_rn(o);
+        else reinterpret_cast<float*>(Y)[(int64_t)m * N + n] = o;
+      }
+    }
+  }
+}
+
 void gemm_simt(const void* X, int x_bf16, const void* W, int w_bf16, const float* b, void* Y, int y_bf16, int M, int N,
                int K, int act, cudaStream_t st) {
   if (M == 0 || N == 0) return;
+  if (N <= 8) {
+    const dim3 g(grid_for((int64_t)M * 32, 256, 4));
+    if (x_bf16 && w_bf16)
+      launch_pdl(linear_narrow_kernel<__nv_bfloat16, __nv_bfloat16>, g, dim3(256), 0, st, (const __nv_bfloat16*)X,
+                 (const __nv_bfloat16*)W, b, Y, y_bf16, M, N, K, act);
+    else if (!x_bf16 && !w_bf16)
+      launch_pdl(linear_narrow_kernel<float, float>, g, dim3(256), 0, st, (const float*)X, (const float*)W, b, Y, y_bf16,
+                 M, N, K, act);
+    else if (x_bf16)
+      launch_pdl(linear_narrow_kernel<__nv_bfloat16, float>, g, dim3(256), 0, st, (const __nv_bfloat16*)X,
+                 (const float*)W, b, Y, y_bf16, M, N, K, act);
+    else
+      launch_pdl(linear_narrow_kernel<float, __nv_bfloat16>, g, dim3(256), 0, st, (const float*)X,
+                 (const __nv_bfloat16*)W, b, Y, y_bf16, M, N, K, act);
+    return;
+  }
   dim3 grid((N + 63) / 64, (M + 63) / 64);
   if (x_bf16 && w_bf16)
     gemm_simt_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 256, 0, st>>>(

@@ -311,19 +311,26 @@ void build_op(Program& P, const Node& n, Op& op) {
     const int es = dtype_bytes(x.dtype);
     void* hb[2] = {P.alloc((int64_t)B * H * es), P.alloc((int64_t)B * H * es)};
     float* cst = (float*)P.alloc((int64_t)B * H * 4);
-    // persistent recurrence (kernels/rnn_persist.cu) when the grid fits in half of the SMs (two
-    // recurrent branches on two slots co-reside); DUET_RNN_PERSIST=0 forces the per-step kernels
+    // persistent recurrence (kernels/rnn_persist.cu): one tile per CTA when the tiles fit in half of
+    // the SMs (two recurrent branches on two slots co-reside), else every SM with several tiles per
+    // CTA (large batches).  DUET_RNN_PERSIST=0 forces the per-step kernels.
     static const int rp_env = getenv("DUET_RNN_PERSIST") ? atoi(getenv("DUET_RNN_PERSIST")) : 1;
     static const int rp_bn_env = getenv("DUET_RNN_BN") ? atoi(getenv("DUET_RNN_BN")) : 0;
-    int rp_bn = 0;
+    int rp_bn = 0, rp_grid = 0;
     if (tc && rp_env) {
       const int mt = (B + 127) / 128;
       for (int cand : {64, 128}) {
         if (rp_bn_env && cand != rp_bn_env) continue;
-        if (mt * ((H + cand / 4 - 1) / (cand / 4)) <= sms / 2) {
+        const int tl = mt * ((H + cand / 4 - 1) / (cand / 4));
+        if (tl <= sms / 2) {
           rp_bn = cand;
+          rp_grid = tl;
           break;
         }
+      }
+      if (!rp_bn) {
+        rp_bn = rp_bn_env ? rp_bn_env : 128;
+        rp_grid = sms;
       }
     }
     if (rp_bn) {
@@ -334,6 +341,7 @@ void build_op(Program& P, const Node& n, Op& op) {
       const int Np = tiles * bn;
       const int Ep = (E + 63) / 64 * 64;
       const int Kc = Ep + H;
+      const int grid = std::min(rp_grid, tiles * mt);
       void* Wcat = P.alloc((int64_t)Np * Kc * 2);
       float* bias = (float*)P.alloc((int64_t)Np * 4);
       unsigned* counter = (unsigned*)P.alloc(256);
@@ -346,19 +354,21 @@ void build_op(Program& P, const Node& n, Op& op) {
       ra.hbuf[0] = (__nv_bfloat16*)hb[0];
       ra.hbuf[1] = (__nv_bfloat16*)hb[1];
       ra.counter = counter;
+      ra.c_state = cst;
       ra.S = S;
       ra.B = B;
       ra.H = H;
       ra.kx = Ep / 64;
       ra.kh = (H + 63) / 64;
-      ra.n_cta = tiles * mt;
+      ra.tiles_n = tiles;
+      ra.tiles_m = mt;
       ra.dbg = getenv("DUET_RNN_DBG") ? atoi(getenv("DUET_RNN_DBG")) : 0;
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         CK(cudaMemsetAsync(counter, 0, sizeof(unsigned), st));
         CUtensorMap tx = make_tmap_bf16_2d(T[in], (int64_t)S * B, E, 128);
         RnnPersistArgs r = ra;
         r.out = (__nv_bfloat16*)T[me];
-        rnn_persist(kind, bn, tx, t_h0, t_h1, t_w, r, tiles, mt, st);
+        rnn_persist(kind, bn, tx, t_h0, t_h1, t_w, r, grid, st);
       };
       op.n_kernels = 1;
     } else if (tc) {

@@ -1,4 +1,3 @@
-for w in 1 0; do echo "=== LSTM WRES=$w"; DUET_RNN_WRES=$w timeout 120 python tools/rnn_trace.py lstm 256 512 256 64 64 | tail -4; done
-echo "=== GRU"; timeout 120 python tools/rnn_trace.py gru 64 1024 256 64 64 | tail -4
-timeout 600 python -m pytest tests -m gpu -x -q -k "lstm or gru or c3 or c4 or rnn" 2>&1 | tail -3
-for c in c3 c4; do timeout 300 python bench.py --config $c --steps 100 --warmup 10 --no-cpu-baseline > gpurun_out/rnn_$c.log 2>&1; done
+timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+timeout 600 python tools/node_times.py c5 > gpurun_out/nodes_c5.log 2>&1
+timeout 400 python bench.py --config c5 --steps 50 --warmup 5 --no-cpu-baseline > gpurun_out/bench_c5.log 2>&1
