@@ -237,7 +237,8 @@ __global__ void __launch_bounds__(THREADS, 1)
         for (int c = 0; c < CO; c += 16) {
           float t[16];
 #pragma unroll
-          for (int u = 0; u < 16; ++u) t[u] = apply_act(v[c + u] + s_bias[c + u], g.act);
+          for (int u = 0; u < 16; ++u) t[u] = v[c + u];
+          bias_act<16>(t, s_bias + c, g.act);
           store_row16(out + c, t);
         }
       }

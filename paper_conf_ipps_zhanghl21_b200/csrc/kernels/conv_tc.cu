@@ -195,8 +195,7 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
             for (int i = 0; i < 16; ++i)
               if (col0 + i < s.Co) v[i] += __bfloat162float(res[col0 + i]);
           }
-#pragma unroll
-          for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i] + s_bias[c * 16 + i], a.act);
+          bias_act<16>(v, s_bias + c * 16, a.act);
           store_row16_any(out + col0, v, s.Co - col0);
         }
       }

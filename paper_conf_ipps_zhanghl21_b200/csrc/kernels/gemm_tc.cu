@@ -149,8 +149,7 @@ __global__ void __launch_bounds__(192, 1)
         ptx::tmem_ld16(tq + c * 16, v);
         const int col0 = n0 + c * 16;
         if (row < M && col0 < N) {
-#pragma unroll
-          for (int i = 0; i < 16; ++i) v[i] = apply_act(v[i] + s_bias[c * 16 + i], act);
+          bias_act<16>(v, s_bias + c * 16, act);
           store_row16_any(out + col0, v, N - col0);
         }
       }

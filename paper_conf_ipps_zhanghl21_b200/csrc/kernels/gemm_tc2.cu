@@ -215,8 +215,7 @@ __global__ void __launch_bounds__(kThreads2, 1)
 #pragma unroll
           for (int j = 0; j < CW / 16; ++j) ptx::tmem_ld16(tq + c0 + 16 * j, v + 16 * j);
         }
-#pragma unroll
-        for (int i = 0; i < CW; ++i) v[i] = apply_act(v[i] + s_bias[c0 + i], act);
+        bias_act<CW>(v, s_bias + c0, act);
         uint8_t* st_row = stage_base + buf * (32 * SPAN) + lane * SPAN;
         if (lane == 0) ptx::bulk_wait_read<1>();  // this buffer's previous store has read smem
         __syncwarp();
@@ -264,8 +263,7 @@ __global__ void __launch_bounds__(kThreads2, 1)
           for (int j = 0; j < CW / 16; ++j) {
             const int col0 = n0 + c0 + 16 * j;
             if (col0 < N) {
-#pragma unroll
-              for (int i = 0; i < 16; ++i) v[16 * j + i] = apply_act(v[16 * j + i] + s_bias[c0 + 16 * j + i], act);
+              bias_act<16>(v + 16 * j, s_bias + c0 + 16 * j, act);
               store_row16_any(out + col0, v + 16 * j, N - col0);
             }
           }

@@ -67,11 +67,13 @@ void rnn_pack(int kind, const void* Wih, const void* Whh, const float* bih, cons
 // U = bn/4); grid < tiles -> each CTA owns several tiles (state kept in global memory).
 struct RnnPersistArgs {
   const float* bias = nullptr;        // [tiles_n * bn] packed gate bias
-  __nv_bfloat16* hbuf[2] = {nullptr, nullptr};  // [B, H] ping-pong h_t (t even -> 0, odd -> 1)
+  __nv_bfloat16* hbuf[2] = {nullptr, nullptr};  // ping-pong h_t (t even -> 0, odd -> 1), K-blocked
+                                                // pre-swizzled [kh][Bp][64] (rnn_persist.cu)
   __nv_bfloat16* out = nullptr;       // [B, H] h_S
   unsigned* counter = nullptr;        // grid-barrier counter, zeroed before each launch
   float* c_state = nullptr;           // LSTM cell state [B, H] fp32 (several tiles per CTA only)
   int S = 0, B = 0, H = 0, kx = 0, kh = 0;
+  int Bp = 0;                         // B padded to the 128-row tiles
   int tiles_n = 0, tiles_m = 0;       // tile grid: n (gate-block tiles of bn columns) fastest
   int dbg = 0;                        // 1 = per-step timestamps (g_rp_trace)
   int stages = 0;                     // A-ring depth (set by the launcher)
@@ -80,6 +82,26 @@ struct RnnPersistArgs {
 // [tiles_n*bn, kx*64 + H] (box bn rows).
 void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1,
                  const CUtensorMap& tw, const RnnPersistArgs& a, int grid, cudaStream_t st);
+
+// Persistent chain of linear layers (mlp_chain.cu): Y_l = act_l(Y_{l-1} W_l^T + b_l), bf16, every
+// N_l % 128 == 0, 256 x 128 tiles on CTA pairs, one cooperative launch for all layers.
+constexpr int kMlpChainMax = 4;
+struct MlpChainMaps {
+  CUtensorMap a[kMlpChainMax];  // layer input [M, K_l] (box 128 rows)
+  CUtensorMap w[kMlpChainMax];  // weights [N_l, K_l] (box 64 rows)
+  CUtensorMap o[kMlpChainMax];  // layer output [M, N_l] (TMA store, box 32 rows x 64 columns)
+};
+struct MlpChainArgs {
+  int L = 0, M = 0, m_blocks = 0;
+  int K[kMlpChainMax] = {}, tiles_n[kMlpChainMax] = {}, act[kMlpChainMax] = {};
+  const float* bias[kMlpChainMax] = {};
+  int item0[kMlpChainMax + 1] = {};  // first work item of each layer (set by mlp_chain)
+  unsigned* done = nullptr;          // [L][m_blocks] tile-completion counters (zeroed per launch)
+  int dbg = 0;                       // 1 = per-item timestamps (g_chain_trace)
+};
+bool mlp_chain_ok(int M, const int* N, const int* K, int L);
+void mlp_chain(const MlpChainMaps& maps, MlpChainArgs a, int sms, cudaStream_t st);
+CUtensorMap mlp_chain_out_map(void* out, int M, int N);
 
 // CTA-pair GEMM (gemm_tc2.cu): 256 x bn tiles, bn in {64,128,256}; W map box rows = bn / 2.
 int tc2_pick_bn(int M, int N, int K, int num_sms);

@@ -91,6 +91,41 @@ __device__ __forceinline__ void tma_load_2d(const CUtensorMap* m, uint64_t* bar,
       : "memory");
 }
 
+// 1D bulk copy global -> shared (contiguous bytes, multiple of 16), completing on `bar`
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// same, multicast to every CTA of `mask` (same smem offset, each CTA's own barrier at `bar`'s offset)
+__device__ __forceinline__ void bulk_g2s_mc(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint16_t mask) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], %4;" ::"r"(
+          smem_u32(dst)),
+      "l"((uint64_t)src), "r"(bytes), "r"(smem_u32(bar)), "h"(mask)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d_mc(const CUtensorMap* m, uint64_t* bar, void* dst, int c0, int c1,
+                                               uint16_t mask) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1, {%4, "
+      "%5}], [%2], %3;" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)m), "r"(smem_u32(bar)), "h"(mask), "r"(c0), "r"(c1)
+      : "memory");
+}
+// commit (single-CTA MMA) arriving on the barrier at the same offset in every CTA of `mask`
+__device__ __forceinline__ void umma_commit_mc_elect(uint64_t* bar, uint16_t mask) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n\t}" ::"r"(
+          smem_u32(bar)),
+      "h"(mask)
+      : "memory");
+}
+
 __device__ __forceinline__ void tma_load_3d(const CUtensorMap* m, uint64_t* bar, void* dst, int c0, int c1, int c2) {
   asm volatile(
       "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(
@@ -251,6 +286,33 @@ __device__ __forceinline__ float apply_act(float x, int act) {
   }
 }
 
+// Epilogue activation for the bf16 tensor-core paths (tolerance 2e-2): tanh.approx-based sigmoid /
+// tanh (one MUFU op each) and the activation switch hoisted out of the element loop.  A
+// per-element apply_act() inlined the full-precision tanhf/expf bodies for every element of a
+// 64-wide register tile: ~8K instructions, measured at ~3.8 us per epilogue from instruction
+// fetch alone.
+__device__ __forceinline__ float tanh_fast(float x) {
+  float y;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+template <int N>
+__device__ __forceinline__ void bias_act(float* v, const float* b, int act) {
+  if (act == ACT_RELU) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] = fmaxf(v[i] + b[i], 0.0f);
+  } else if (act == ACT_SIGMOID) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] = fmaf(0.5f, tanh_fast(0.5f * (v[i] + b[i])), 0.5f);
+  } else if (act == ACT_TANH) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] = tanh_fast(v[i] + b[i]);
+  } else {
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] += b[i];
+  }
+}
+
 template <typename T>
 __device__ __forceinline__ float to_f(T v);
 template <>
@@ -324,6 +386,16 @@ __device__ __forceinline__ uint32_t mapa(uint32_t local_addr, uint32_t rank) {
   uint32_t r;
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(local_addr), "r"(rank));
   return r;
+}
+// arrive on the barrier at cluster address `cl_addr` (e.g. the pair leader's).  Default semantics:
+// an explicit .release.cluster compiles to MEMBAR.ALL.GPU, measured at ~4 us per arrive under load
+__device__ __forceinline__ void mbar_arrive_cl(uint32_t cl_addr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cl_addr) : "memory");
+}
+// relaxed variant: only orders through the barrier itself (TMEM reads are ordered by the tcgen05
+// fences around it)
+__device__ __forceinline__ void mbar_arrive_cl_relaxed(uint32_t cl_addr) {
+  asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(cl_addr) : "memory");
 }
 __device__ __forceinline__ void mbar_arrive_expect_tx_cl(uint32_t cl_addr, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cluster.b64 _, [%0], %1;" ::"r"(cl_addr), "r"(bytes) : "memory");

@@ -72,6 +72,11 @@ inline int rp_plan(int bn, int nkw, bool* wres) {
 
 // (measured: a relaxed polling loop + one fence.acq_rel.gpu passes the barrier ~0.3 us later than
 // polling with ld.acquire)
+__device__ __forceinline__ unsigned ld_relaxed_gpu(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 __device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
   unsigned v;
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -119,6 +124,13 @@ __device__ __forceinline__ float cell(float a0, float a1, float a2, float a3, fl
     return h;
   }
 }
+// h_t buffers are K-blocked and pre-swizzled: [kh][Bp][64] with the 16-byte chunk c of row r at
+// position c ^ (r & 7), i.e. exactly the SWIZZLE_128B K-major layout UMMA reads.  A (k-block, row
+// tile) of h is then one contiguous 16 KB range, fetched with a single bulk copy instead of a
+// 128-row tensor-map load.  Element index of the 8-unit group starting at `unit` (unit % 8 == 0):
+__device__ __forceinline__ size_t hs_index(int row, int unit, int Bp) {
+  return ((size_t)(unit >> 6) * Bp + row) * 64 + (size_t)((((unit & 63) >> 3) ^ (row & 7)) << 3);
+}
 __device__ __forceinline__ void store_bf16x8(__nv_bfloat16* dst, const float* h) {
   uint32_t w[4];
 #pragma unroll
@@ -135,7 +147,7 @@ __device__ __forceinline__ void tmem_ld_n(uint32_t taddr, float* v) {
   else ptx::tmem_ld8(taddr, v);
 }
 
-template <int BN, int KIND, bool WRES, bool MULTI>
+template <int BN, int KIND, bool WRES, bool MULTI, int CN>
 __global__ void __launch_bounds__(kRThreads, 1)
     rnn_persist_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmH0,
                        const __grid_constant__ CUtensorMap tmH1, const __grid_constant__ CUtensorMap tmW,
@@ -174,7 +186,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
     ptx::tma_prefetch(&tmW);
     for (int s = 0; s < STAGES; ++s) {
       ptx::mbar_init(&full[s], WRES ? 1 : 2);  // A producer (+ W producer), each with its tx bytes
-      ptx::mbar_init(&empty[s], 1);
+      ptx::mbar_init(&empty[s], CN);  // every CTA of the cluster consumed the (multicast) stage
     }
     ptx::mbar_init(w_full, 1);
     for (int b = 0; b < 2; ++b) {
@@ -189,8 +201,13 @@ __global__ void __launch_bounds__(kRThreads, 1)
   }
   if (!MULTI)
     for (int c = (int)threadIdx.x - 64; c >= 0 && c < BN; c += 32 * kREpiWarps) s_bias[c] = a.bias[tile_n0(0) + c];
+  // CN > 1: the cluster's CN CTAs are consecutive n-tiles of one row tile and read the same x_t / h
+  // blocks; k-block j is loaded once, by CTA j % CN, and multicast to all (L2 -> SM traffic / CN:
+  // with one load per CTA, 32 SMs pulling the same 128 KB of h_{t-1} saturated the L2 slices)
+  const uint32_t crank = CN > 1 ? ptx::cluster_ctarank() : 0;
+  constexpr uint16_t kMask = (uint16_t)((1u << CN) - 1);
   ptx::tc_fence_before();
-  __syncthreads();
+  if constexpr (CN > 1) ptx::cluster_sync(); else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
@@ -199,7 +216,6 @@ __global__ void __launch_bounds__(kRThreads, 1)
     int g = 0;
     for (int t = 0; t < S; ++t) {
       const int nkb = kx + (t > 0 ? kh : 0);  // h_{-1} = 0: step 0 has only the x part
-      const CUtensorMap* th = ((t - 1) & 1) ? &tmH1 : &tmH0;
       for (int i = 0; i < my_tiles; ++i) {
         const int m0 = tile_m0(i);
         for (int j = 0; j < nkb; ++j, ++g) {
@@ -220,10 +236,18 @@ __global__ void __launch_bounds__(kRThreads, 1)
           }
           if (lane == 0) {
             ptx::mbar_arrive_expect_tx(&full[s], R_A_BYTES);
-            if (j < kx)
-              ptx::tma_load_2d(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
-            else
-              ptx::tma_load_2d(th, &full[s], sA + s * R_A_BYTES, (j - kx) * RBK, m0);
+            if (CN == 1 || (int)crank == j % CN) {
+              if (j < kx) {
+                if constexpr (CN > 1)
+                  ptx::tma_load_2d_mc(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0, kMask);
+                else
+                  ptx::tma_load_2d(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
+              } else {  // h_{t-1}: one contiguous, pre-swizzled 16 KB block (see hs_index)
+                const __nv_bfloat16* src = a.hbuf[(t - 1) & 1] + ((size_t)(j - kx) * a.Bp + m0) * RBK;
+                if constexpr (CN > 1) ptx::bulk_g2s_mc(sA + s * R_A_BYTES, src, R_A_BYTES, &full[s], kMask);
+                else ptx::bulk_g2s(sA + s * R_A_BYTES, src, R_A_BYTES, &full[s]);
+              }
+            }
           }
           __syncwarp();
         }
@@ -284,7 +308,8 @@ __global__ void __launch_bounds__(kRThreads, 1)
           if (!(a.dbg & 16))
 #pragma unroll
             for (int k = 0; k < RBK / 16; ++k) ptx::umma_bf16_elect(d, da + 2 * k, db + 2 * k, idesc, (j | k) != 0);
-          ptx::umma_commit_elect(&empty[s]);
+          if constexpr (CN > 1) ptx::umma_commit_mc_elect(&empty[s], kMask);  // frees the stage cluster-wide
+          else ptx::umma_commit_elect(&empty[s]);
         }
         ptx::umma_commit_elect(&tfull[buf]);
         if (trace && t < 64 && lane == 0) trace[t * 16 + 5] = rp_gtimer();  // last UMMA issued
@@ -328,11 +353,13 @@ __global__ void __launch_bounds__(kRThreads, 1)
 #pragma unroll
         for (int i = 0; i < UH; ++i) h[i] = cell<KIND>(acc[0][i] + bias[0][i], acc[1][i] + bias[1][i],
                                                         acc[2][i] + bias[2][i], acc[3][i] + bias[3][i], state[i]);
-        __nv_bfloat16* dst = (t == S - 1 ? a.out : a.hbuf[buf]) + (size_t)row * H + unit0;
         if (live) {
 #pragma unroll
           for (int v = 0; v < UH / 8; ++v)
-            if (v * 8 < nv) store_bf16x8(dst + 8 * v, h + 8 * v);
+            if (v * 8 < nv) {
+              if (t == S - 1) store_bf16x8(a.out + (size_t)row * H + unit0 + 8 * v, h + 8 * v);
+              else store_bf16x8(a.hbuf[buf] + hs_index(row, unit0 + 8 * v, a.Bp), h + 8 * v);
+            }
         }
         if (trace && t < 64 && lane == 0) trace[t * 16 + 6 + warp] = rp_gtimer();  // [8..15] math + stores
         if (t < S - 1) {
@@ -365,7 +392,6 @@ __global__ void __launch_bounds__(kRThreads, 1)
           ptx::tc_fence_before();
           __syncwarp();
           if (lane == 0) ptx::mbar_arrive(&tempty[buf]);
-          __nv_bfloat16* dst = (t == S - 1 ? a.out : a.hbuf[t & 1]);
           const __nv_bfloat16* hprev = a.hbuf[(t - 1) & 1];
 #pragma unroll
           for (int c = 0; c < UH / 8; ++c) {
@@ -388,7 +414,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
 #pragma unroll
                 for (int e = 0; e < 8; ++e) st[e] = 0.0f;
               } else {
-                const uint4 raw = *reinterpret_cast<const uint4*>(hprev + off);
+                const uint4 raw = *reinterpret_cast<const uint4*>(hprev + hs_index(row, unit, a.Bp));
                 const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&raw);
 #pragma unroll
                 for (int e = 0; e < 8; ++e) st[e] = __bfloat162float(hv[e]);
@@ -405,7 +431,8 @@ __global__ void __launch_bounds__(kRThreads, 1)
               *reinterpret_cast<float4*>(a.c_state + off) = make_float4(st[0], st[1], st[2], st[3]);
               *reinterpret_cast<float4*>(a.c_state + off + 4) = make_float4(st[4], st[5], st[6], st[7]);
             }
-            store_bf16x8(dst + off, h);
+            if (t == S - 1) store_bf16x8(a.out + off, h);
+            else store_bf16x8(a.hbuf[t & 1] + hs_index(row, unit, a.Bp), h);
           }
           if (t < S - 1) {
             fence_proxy_async_global();
@@ -417,18 +444,19 @@ __global__ void __launch_bounds__(kRThreads, 1)
     }
   }
   ptx::tc_fence_before();
-  __syncthreads();
+  // no CTA may exit while a peer can still multicast into its shared memory / arrive on it
+  if constexpr (CN > 1) ptx::cluster_sync(); else __syncthreads();
   if (warp == 1) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc(tmem, C::TMEM_COLS);
   }
 }
 
-template <int BN, int KIND, bool WRES, bool MULTI>
+template <int BN, int KIND, bool WRES, bool MULTI, int CN>
 void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1, const CUtensorMap& tw,
                const RnnPersistArgs& a, int grid, cudaStream_t st) {
   using C = RCfg<BN>;
-  auto kern = rnn_persist_kernel<BN, KIND, WRES, MULTI>;
+  auto kern = rnn_persist_kernel<BN, KIND, WRES, MULTI, CN>;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kRSmemBudget));
@@ -440,11 +468,15 @@ void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap&
   cfg.blockDim = dim3(kRThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute at[1];
+  cudaLaunchAttribute at[2];
   at[0].id = cudaLaunchAttributeCooperative;
   at[0].val.cooperative = 1;
+  at[1].id = cudaLaunchAttributeClusterDimension;
+  at[1].val.clusterDim.x = CN;
+  at[1].val.clusterDim.y = 1;
+  at[1].val.clusterDim.z = 1;
   cfg.attrs = at;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = CN > 1 ? 2 : 1;
   CK(cudaLaunchKernelEx(&cfg, kern, tx, th0, th1, tw, a));
 }
 
@@ -455,7 +487,7 @@ void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensor
   if (multi) {  // several tiles per CTA: W changes per tile, so it is streamed
     a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
     if (a.stages > 10) a.stages = 10;
-    return launch_rp<BN, KIND, false, true>(tx, th0, th1, tw, a, grid, st);
+    return launch_rp<BN, KIND, false, true, 1>(tx, th0, th1, tw, a, grid, st);
   }
   static const int wres_env = getenv("DUET_RNN_WRES") ? atoi(getenv("DUET_RNN_WRES")) : 1;
   bool wres = false;
@@ -465,8 +497,26 @@ void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensor
     a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
     if (a.stages > 10) a.stages = 10;
   }
-  if (wres) return launch_rp<BN, KIND, true, false>(tx, th0, th1, tw, a, grid, st);
-  launch_rp<BN, KIND, false, false>(tx, th0, th1, tw, a, grid, st);
+  // cluster multicast of x_t / h blocks (DUET_RNN_CN = 2/4/8, opt-in): measured h-phase -9% (LSTM
+  // 256x512) / -13% (GRU 64x1024) only -- the per-SM receive rate, not L2, bounds it -- while
+  // clusters of 8 keep c3's two co-scheduled towers from being co-resident (c3 0.38 -> 0.66 ms)
+  static const int cn_env = getenv("DUET_RNN_CN") ? atoi(getenv("DUET_RNN_CN")) : 1;
+  int cn = 1;
+  for (int c : {8, 4, 2})
+    if (c <= cn_env && a.tiles_n % c == 0) {
+      cn = c;
+      break;
+    }
+#define DUET_RP_CN(CNV)                                                                        \
+  if (cn == CNV) {                                                                             \
+    if (wres) return launch_rp<BN, KIND, true, false, CNV>(tx, th0, th1, tw, a, grid, st);     \
+    return launch_rp<BN, KIND, false, false, CNV>(tx, th0, th1, tw, a, grid, st);              \
+  }
+  DUET_RP_CN(8)
+  DUET_RP_CN(4)
+  DUET_RP_CN(2)
+  DUET_RP_CN(1)
+#undef DUET_RP_CN
 }
 
 }  // namespace

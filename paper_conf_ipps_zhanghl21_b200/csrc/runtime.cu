@@ -37,6 +37,8 @@ struct Program {
   std::vector<void*> allocs;               // device memory to free
   std::map<int, std::pair<int, int>> fuse_res;  // conv node -> (residual node, add node it writes)
   std::set<int> fused_adds;
+  std::map<int, std::vector<int>> chains;  // head linear node -> chain of linear nodes (mlp_chain.cu)
+  std::map<int, Op> chain_ops;             // head -> one launch for the whole chain
   ~Program() {
     int prev = 0;
     cudaGetDevice(&prev);
@@ -348,11 +350,17 @@ void build_op(Program& P, const Node& n, Op& op) {
       rnn_pack(kind, Wih, Whh, bih, bhh, Wcat, bias, E, Ep, H, U, bn, tiles, 0);
       CK(cudaDeviceSynchronize());
       CUtensorMap t_w = make_tmap_bf16_2d(Wcat, Np, Kc, bn);
+      // K-blocked pre-swizzled h buffers [kh][mt*128][64] (bulk-copied per k-block)
+      const int64_t hs_bytes = (int64_t)((H + 63) / 64) * mt * 128 * 64 * 2;
+      void* hs[2] = {P.alloc(hs_bytes), P.alloc(hs_bytes)};
+      CK(cudaMemset(hs[0], 0, hs_bytes));  // units >= H of the last k-block stay zero
+      CK(cudaMemset(hs[1], 0, hs_bytes));
       CUtensorMap t_h0 = make_tmap_bf16_2d(hb[0], B, H, 128), t_h1 = make_tmap_bf16_2d(hb[1], B, H, 128);
       RnnPersistArgs ra;
       ra.bias = bias;
-      ra.hbuf[0] = (__nv_bfloat16*)hb[0];
-      ra.hbuf[1] = (__nv_bfloat16*)hb[1];
+      ra.hbuf[0] = (__nv_bfloat16*)hs[0];
+      ra.hbuf[1] = (__nv_bfloat16*)hs[1];
+      ra.Bp = mt * 128;
       ra.counter = counter;
       ra.c_state = cst;
       ra.S = S;
@@ -619,6 +627,79 @@ void plan_residual_fusion(Program& P) {
   }
 }
 
+// Chains of bf16 linear layers where each layer's only consumer is the next (the deep towers'
+// MLPs): one persistent launch runs the whole chain (kernels/mlp_chain.cu) when every member is in
+// the same subgraph at run time (launch_subgraph).  Intermediate outputs still land in their nodes'
+// buffers.  Opt-in: DUET_MLP_CHAIN=1.
+void plan_linear_chains(Program& P, int sms) {
+  // opt-in: measured slower than per-layer launches on c2 (the cross-CTA dependency hand-off costs
+  // ~3 us per layer boundary: TMA-store completion + release + polling + TMA load latency), see
+  // DESIGN.md "MLP chain"
+  static const int env = getenv("DUET_MLP_CHAIN") ? atoi(getenv("DUET_MLP_CHAIN")) : 0;
+  if (!env) return;
+  const Graph& g = *P.g;
+  std::vector<int> n_cons(g.nodes.size(), 0), consumer(g.nodes.size(), -1);
+  for (auto& n : g.nodes)
+    for (int u : n.inputs) n_cons[u]++, consumer[u] = n.id;
+  std::set<int> outs(g.outputs.begin(), g.outputs.end());
+  auto eligible = [&](const Node& n) {
+    if (n.op != "linear" || n.arg_nodes.size() != 1 || n.params.size() != 2) return false;
+    const Node& x = g.nodes[n.arg_nodes[0]];
+    const auto& w = g.params.at(n.params[0]);
+    return x.dtype == kBF16 && w.dtype == kBF16 && n.dtype == kBF16 && x.shape.size() == 2 && x.shape[0] > 128 &&
+           n.shape[1] % 128 == 0 && x.shape[1] % 8 == 0;
+  };
+  auto next_of = [&](int v) -> int {
+    if (n_cons[v] != 1 || outs.count(v)) return -1;
+    const Node& c = g.nodes[consumer[v]];
+    if (!eligible(c) || c.arg_nodes[0] != v || c.shape[0] != g.nodes[v].shape[0]) return -1;
+    return c.id;
+  };
+  std::set<int> taken;
+  for (int v : g.topo) {
+    if (taken.count(v) || !eligible(g.nodes[v])) continue;
+    std::vector<int> ch{v};
+    for (int c = next_of(v); c >= 0 && (int)ch.size() < kMlpChainMax; c = next_of(c)) ch.push_back(c);
+    if (ch.size() < 2) continue;
+    for (int c : ch) taken.insert(c);
+    P.chains[v] = ch;
+    const int M = (int)g.nodes[v].shape[0];
+    MlpChainArgs a;
+    a.L = (int)ch.size();
+    a.M = M;
+    a.m_blocks = (M + 255) / 256;
+    std::vector<int> ins, Ns, Ks;
+    std::vector<CUtensorMap> wmaps;
+    for (int l = 0; l < a.L; ++l) {
+      const Node& n = g.nodes[ch[l]];
+      const auto& w = g.params.at(n.params[0]);
+      Ns.push_back((int)w.shape[0]);
+      Ks.push_back((int)w.shape[1]);
+      a.K[l] = (int)w.shape[1];
+      a.tiles_n[l] = (int)w.shape[0] / 128;
+      a.act[l] = act_code(n.attr_str("act", "none"));
+      a.bias[l] = (const float*)P.param(n.params[1]);
+      wmaps.push_back(make_tmap_bf16_2d(P.param(n.params[0]), w.shape[0], w.shape[1], 64));
+    }
+    a.done = (unsigned*)P.alloc((int64_t)a.L * a.m_blocks * 4);
+    a.dbg = getenv("DUET_CHAIN_DBG") ? atoi(getenv("DUET_CHAIN_DBG")) : 0;
+    const int in = g.nodes[v].arg_nodes[0];
+    Op op;
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      MlpChainMaps maps;
+      for (int l = 0; l < a.L; ++l) {
+        const void* src = T[l == 0 ? in : ch[l - 1]];
+        maps.a[l] = make_tmap_bf16_2d(src, M, Ks[l], 128);
+        maps.w[l] = wmaps[l];
+        maps.o[l] = mlp_chain_out_map(T[ch[l]], M, Ns[l]);
+      }
+      mlp_chain(maps, a, sms, st);
+    };
+    op.n_kernels = 1;
+    P.chain_ops[v] = op;
+  }
+}
+
 std::shared_ptr<Program> ensure_program(Graph* g) {
   if (g->prog) return g->prog;
   for (auto& name : g->param_order)
@@ -637,14 +718,46 @@ std::shared_ptr<Program> ensure_program(Graph* g) {
   P->ops.resize(g->nodes.size());
   plan_residual_fusion(*P);
   for (auto& n : g->nodes) build_op(*P, n, P->ops[n.id]);
+  plan_linear_chains(*P, num_sms(dev));
   CK(cudaDeviceSynchronize());
   g->prog = P;
   return P;
 }
 
+bool chain_in_subgraph(const Program& P, const Partition& part, int s, int head) {
+  auto it = P.chains.find(head);
+  if (it == P.chains.end()) return false;
+  for (int c : it->second)
+    if (part.node_to_sg[c] != s) return false;
+  return true;
+}
+
 void launch_subgraph(const Program& P, const Partition& part, int s, const Ptrs& T, cudaStream_t st) {
-  for (int v : part.sg_nodes[s])
+  std::set<int> skip;
+  for (int v : part.sg_nodes[s]) {
+    if (skip.count(v)) continue;
+    if (chain_in_subgraph(P, part, s, v)) {
+      P.chain_ops.at(v).launch(T, st);
+      for (int c : P.chains.at(v)) skip.insert(c);
+      continue;
+    }
     if (P.ops[v].launch) P.ops[v].launch(T, st);
+  }
+}
+
+int subgraph_kernels(const Program& P, const Partition& part, int s) {
+  int nk = 0;
+  std::set<int> skip;
+  for (int v : part.sg_nodes[s]) {
+    if (skip.count(v)) continue;
+    if (chain_in_subgraph(P, part, s, v)) {
+      nk += 1;
+      for (int c : P.chains.at(v)) skip.insert(c);
+      continue;
+    }
+    nk += P.ops[v].n_kernels;
+  }
+  return nk;
 }
 
 int64_t tensor_numel(const duet_tensor& t) {
@@ -746,7 +859,7 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
       for (int u : preds[s])
         if (streams[S.slot_of[u]] != st) CK(cudaStreamWaitEvent(st, done[u], 0));
       launch_subgraph(P, part, s, T, st);
-      for (int v : part.sg_nodes[s]) nk += P.ops[v].n_kernels;
+      nk += subgraph_kernels(P, part, s);
       CK(cudaEventRecord(done[s], st));
       last_on[q] = s;
     }
