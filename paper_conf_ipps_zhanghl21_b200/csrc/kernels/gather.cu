@@ -35,8 +35,14 @@ __global__ void hash_mod_kernel(const int64_t* __restrict__ raw, int32_t* __rest
   ptx::pdl_wait();
   ptx::pdl_trigger();
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    int64_t r = raw[i] % V;
-    if (r < 0) r += V;
+    const int64_t x = raw[i];
+    int64_t r;
+    if ((uint64_t)x < (1ULL << 32) && V < (1LL << 32))
+      r = (int64_t)((uint32_t)x % (uint32_t)V);  // 32-bit path (the recipe's raw ids are < 2^31)
+    else {
+      r = x % V;
+      if (r < 0) r += V;
+    }
     ids[i] = (int32_t)r;
   }
 }
@@ -95,6 +101,43 @@ __global__ void gather_rows16_kernel(const int32_t* __restrict__ idx, const uint
 #pragma unroll
     for (int u = 0; u < 4; ++u)
       if (dst[u] >= 0) *reinterpret_cast<uint4*>(out + dst[u]) = val[u];
+  }
+}
+
+// Same with a power-of-two number of 16-byte vectors per row and 32-bit index math (the generic
+// kernel's 64-bit divisions per vector dominated its issue time): VPR lanes per row, four rows in
+// flight per thread.
+template <int MODE, int VPR>
+__global__ void __launch_bounds__(256) gather_rows16p2_kernel(const int32_t* __restrict__ idx,
+                                                              const uint8_t* __restrict__ tab,
+                                                              uint8_t* __restrict__ out, int rows, int F,
+                                                              int64_t R, int B, int S) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
+  constexpr int RB = VPR * 16;
+  const int k = threadIdx.x & (VPR - 1);
+  const int rows_per_pass = (int)(gridDim.x * blockDim.x) / VPR;
+  for (int r0 = (int)(blockIdx.x * blockDim.x + threadIdx.x) / VPR; r0 < rows; r0 += 4 * rows_per_pass) {
+    uint4 val[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int r = r0 + u * rows_per_pass;
+      if (r < rows) {
+        int64_t trow;
+        if (MODE == 0) {
+          trow = (int64_t)(r % F) * R + __ldg(idx + r);
+        } else {
+          const int t = r / B, b = r - t * B;
+          trow = __ldg(idx + (int64_t)b * S + t);
+        }
+        val[u] = ld_stream16(tab + trow * RB + k * 16);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int r = r0 + u * rows_per_pass;
+      if (r < rows) *reinterpret_cast<uint4*>(out + (int64_t)r * RB + k * 16) = val[u];
+    }
   }
 }
 
@@ -187,7 +230,16 @@ static void gather_rows(int mode, const int32_t* idx, const void* tab, int esize
   if (rows == 0) return;
   int64_t rb = (int64_t)D * esize;
   bool vec = (rb % 16 == 0) && ((uintptr_t)tab % 16 == 0) && ((uintptr_t)out % 16 == 0);
-  if (vec) {
+  const int vpr16 = (int)(rb / 16);
+  if (vec && rows < (1LL << 30) && (vpr16 == 4 || vpr16 == 8 || vpr16 == 16)) {
+    const int g = grid_for((rows * vpr16 + 3) / 4, 256, 16);
+#define DUET_G16(M, V)                                                                                             \
+  if (mode == M && vpr16 == V)                                                                                     \
+    launch_pdl(gather_rows16p2_kernel<M, V>, dim3(g), dim3(256), 0, st, idx, (const uint8_t*)tab, (uint8_t*)out,  \
+               (int)rows, F, R, B, S);
+    DUET_G16(0, 4) DUET_G16(0, 8) DUET_G16(0, 16) DUET_G16(1, 4) DUET_G16(1, 8) DUET_G16(1, 16)
+#undef DUET_G16
+  } else if (vec) {
     int vpr = (int)(rb / 16);
     int64_t total = rows * vpr;
     int g = grid_for((total + 3) / 4, 256, 16);
