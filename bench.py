@@ -13,7 +13,9 @@ executed by libduet's greedy-correction schedule on CUDA-stream slots (one CUDA-
   cpu_baseline float64 oracle on a bounded row sample (rank 0, N = 1)
 
 Multi-GPU (torchrun): one process per GPU, each runs its own batch (weak scaling, no data-path
-collective — inference rows are independent).
+collective — inference rows are independent).  `--placement branch`
+instead runs ONE batch with its subgraphs placed on the GPUs by greedy-correction over one slot
+per GPU, cut-edge tensors over NCCL point-to-point (strong scaling; multigpu.py).
 `--impl reference` times the oracle (the reference arm of this tier) on the host cores.
 """
 from __future__ import annotations
@@ -47,6 +49,9 @@ def parse():
     ap.add_argument("--profile-samples", type=int, default=100)
     ap.add_argument("--sched", default="measured", choices=["measured", "model"],
                     help="Step 3's `measure latency`: device measurement (default) or the C3 model")
+    ap.add_argument("--placement", default="batch", choices=["batch", "branch"],
+                    help="N>1: 'batch' = every rank runs its own batch (weak scaling); 'branch' = one batch, "
+                         "subgraphs placed on the GPUs by greedy-correction, cut edges over NCCL (strong)")
     return ap.parse_args()
 
 
@@ -242,10 +247,83 @@ def reference_arm(args):
 
 
 # ---------------------------------------------------------------------------------------------
+def bench_branch(args):
+    """--placement branch: ONE batch per step; the greedy-correction schedule over one slot per GPU
+    places the subgraphs, each rank runs its (GPU, phase) pieces through libduet, cut-edge tensors
+    move over NCCL point-to-point (paper_conf_ipps_zhanghl21_b200/multigpu.py)."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_zhanghl21_b200 import duet
+    from paper_conf_ipps_zhanghl21_b200 import multigpu as MG
+    from paper_conf_ipps_zhanghl21_b200 import multirank as MR
+    from paper_conf_ipps_zhanghl21_b200 import workloads as W
+    from paper_conf_ipps_zhanghl21_b200.harness import materialize
+
+    rank, world, local = MR.env()
+    torch.cuda.set_device(local)
+    MR.init("nccl", torch.device(f"cuda:{local}"))
+    dev = f"cuda:{local}"
+    wl = W.build(args.config, dt=args.dtype)
+    params = materialize(wl.params, dev)
+    g = duet.Graph(wl.ir)
+    g.bind_all(params)
+    part = g.partition()
+    ex = part.export()
+    t_one = None
+    if rank == 0:  # identical B200s: one GPU's per-subgraph times stand for every GPU's column
+        st = torch.cuda.Stream()
+        t_one = part.profile([(local, st)], warmup=3, samples=args.profile_samples, reps=5).export()["t_ns"][:, 0]
+        t_one = [int(v) for v in t_one]
+    if world > 1:
+        obj = [t_one]
+        dist.broadcast_object_list(obj, src=0)
+        t_one = obj[0]
+    sg_gpu, sched = MG.place_branches(ex, t_one, world, graph=g)
+    pl = MG.plan(wl.ir, ex["node_to_sg"], ex["sg_phase"], sg_gpu)
+    runner = MG.DuetPieces(pl, rank, params, local, n_slots=args.slots,
+                           profile=dict(warmup=3, samples=max(5, args.profile_samples // 4), reps=5))
+    exe = MG.Executor(pl, rank, runner, device=torch.device(dev))
+    inputs = materialize(wl.inputs, dev) if rank == 0 else None
+    torch.cuda.synchronize()
+    for _ in range(args.warmup):
+        exe.step(inputs)
+    torch.cuda.synchronize()
+    MR.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    finish_clocks, _, clk_err = clock_sampler(local)
+    e0.record()
+    for _ in range(args.steps):
+        exe.step(inputs)
+    e1.record()
+    torch.cuda.synchronize()
+    clocks = finish_clocks() if finish_clocks else clk_err
+    ms = MR.max_over_ranks(e0.elapsed_time(e1))
+    n_launch = runner.launches()
+    MR.barrier()
+    if rank == 0:
+        line = {"metric": METRIC, "value": round(wl.batch * args.steps / (ms / 1e3), 1), "unit": "samples/s",
+                "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": round(ms / args.steps, 5), "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": args.dtype or "bf16",
+                "data": "synthetic (seeded counter-based generator; random-init weights)",
+                "config": {"workload": wl.name, "global_batch": wl.batch, "parallelism":
+                           f"branch placement over {world} GPU(s) x {args.slots} stream slots",
+                           "l2": "not flushed (multi-rank step)"},
+                "placement": {"sg_gpu": sg_gpu, "model_makespan_ns": sched["makespan"],
+                              "fell_back": sched["fell_back"], "profile_t_ns": t_one,
+                              "transfers": [(t.tensor, t.src, t.dst) for t in pl.transfers]},
+                "gpu_launches_per_step_rank0": n_launch, "clocks": clocks}
+        print(json.dumps(line), flush=True)
+    MR.finalize()
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         return reference_arm(args)
+    if args.placement == "branch":
+        return bench_branch(args)
     import torch
 
     from paper_conf_ipps_zhanghl21_b200 import duet
