@@ -275,7 +275,7 @@ __global__ void __launch_bounds__(C_THREADS, 1)
       }
       __syncwarp();
     }
-    if (lane == 0) ptx::bulk_wait_all();
+    if (lane == 0) ptx::bulk_wait_read<0>();
   }
   ptx::tc_fence_before();
   ptx::cluster_sync();

@@ -381,6 +381,11 @@ __device__ __forceinline__ uint32_t cluster_ctarank() {
 __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
+// relaxed arrive: for the start-of-kernel sync after mbarrier init (fence.mbarrier_init already
+// releases the inits at cluster scope); the .release arrive compiles to MEMBAR.ALL.GPU
+__device__ __forceinline__ void cluster_sync_relaxed() {
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
+}
 // shared::cluster address of `local_addr`'s counterpart in CTA `rank` of the cluster
 __device__ __forceinline__ uint32_t mapa(uint32_t local_addr, uint32_t rank) {
   uint32_t r;
