@@ -109,26 +109,32 @@ def reduce_sum(x, b):
     return (x.sum(axis=1) + b[0]).reshape(-1, 1)
 
 
-def lstm(x, Wih, Whh, bih, bhh):
-    """A6+A7, PyTorch nn.LSTM conventions (gate order i,f,g,o; h0 = c0 = 0); returns h_S."""
+def lstm(x, Wih, Whh, bih, bhh, seq=False):
+    """A6+A7, PyTorch nn.LSTM conventions (gate order i,f,g,o; h0 = c0 = 0); returns h_S, or
+    with `seq` every h_t as [S, B, H] (the input of the next layer of a stacked RNN, PAPER.md:89
+    "Varying the stacked RNN layers", Fig. 14)."""
     S, B, _ = x.shape
     H = Whh.shape[1]
     h = np.zeros((B, H))
     c = np.zeros((B, H))
+    hs = []
     for t in range(S):
         g = x[t] @ Wih.T + bih + h @ Whh.T + bhh
         i, f, gg, o = g[:, :H], g[:, H:2 * H], g[:, 2 * H:3 * H], g[:, 3 * H:]
         i, f, gg, o = sigmoid(i), sigmoid(f), np.tanh(gg), sigmoid(o)
         c = f * c + i * gg
         h = o * np.tanh(c)
-    return h
+        hs.append(h)
+    return np.stack(hs) if seq else h
 
 
-def gru(x, Wih, Whh, bih, bhh):
-    """A6+A8, PyTorch nn.GRU conventions (r,z,n; b_hn inside r*(.); h0 = 0); returns h_S."""
+def gru(x, Wih, Whh, bih, bhh, seq=False):
+    """A6+A8, PyTorch nn.GRU conventions (r,z,n; b_hn inside r*(.); h0 = 0); returns h_S, or
+    with `seq` every h_t as [S, B, H] (stacked layers, as lstm)."""
     S, B, _ = x.shape
     H = Whh.shape[1]
     h = np.zeros((B, H))
+    hs = []
     for t in range(S):
         gx = x[t] @ Wih.T + bih
         gh = h @ Whh.T + bhh
@@ -136,7 +142,8 @@ def gru(x, Wih, Whh, bih, bhh):
         z = sigmoid(gx[:, H:2 * H] + gh[:, H:2 * H])
         n = np.tanh(gx[:, 2 * H:] + r * gh[:, 2 * H:])
         h = (1.0 - z) * n + z * h
-    return h
+        hs.append(h)
+    return np.stack(hs) if seq else h
 
 
 def conv2d(x, W, stride, pad):
@@ -253,9 +260,9 @@ def run(ir, params: dict, inputs: dict, keep_all: bool = False) -> dict:
         elif op == "reduce_sum":
             v = reduce_sum(A[0], P(pn[0]))
         elif op == "lstm":
-            v = lstm(A[0], *(P(p) for p in pn))
+            v = lstm(A[0], *(P(p) for p in pn), seq=bool(int(at.get("seq", 0))))
         elif op == "gru":
-            v = gru(A[0], *(P(p) for p in pn))
+            v = gru(A[0], *(P(p) for p in pn), seq=bool(int(at.get("seq", 0))))
         elif op == "conv2d_bn":
             v = conv2d_bn(A[0], *(P(p) for p in pn), at["stride"], at["pad"], at.get("act", "none"))
         elif op == "add":

@@ -70,6 +70,7 @@ struct RnnPersistArgs {
   __nv_bfloat16* hbuf[2] = {nullptr, nullptr};  // ping-pong h_t (t even -> 0, odd -> 1), K-blocked
                                                 // pre-swizzled [kh][Bp][64] (rnn_persist.cu)
   __nv_bfloat16* out = nullptr;       // [B, H] h_S
+  __nv_bfloat16* seq = nullptr;       // optional [S, B, H]: every h_t (a lower stacked-RNN layer)
   unsigned* counter = nullptr;        // grid-barrier counter, zeroed before each launch
   float* c_state = nullptr;           // LSTM cell state [B, H] fp32 (several tiles per CTA only)
   int S = 0, B = 0, H = 0, kx = 0, kh = 0;

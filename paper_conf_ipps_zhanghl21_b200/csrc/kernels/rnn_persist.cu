@@ -357,6 +357,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
 #pragma unroll
           for (int v = 0; v < UH / 8; ++v)
             if (v * 8 < nv) {
+              if (a.seq) store_bf16x8(a.seq + ((size_t)t * a.B + row) * H + unit0 + 8 * v, h + 8 * v);
               if (t == S - 1) store_bf16x8(a.out + (size_t)row * H + unit0 + 8 * v, h + 8 * v);
               else store_bf16x8(a.hbuf[buf] + hs_index(row, unit0 + 8 * v, a.Bp), h + 8 * v);
             }
@@ -431,6 +432,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
               *reinterpret_cast<float4*>(a.c_state + off) = make_float4(st[0], st[1], st[2], st[3]);
               *reinterpret_cast<float4*>(a.c_state + off + 4) = make_float4(st[4], st[5], st[6], st[7]);
             }
+            if (a.seq) store_bf16x8(a.seq + (size_t)t * a.B * H + off, h);
             if (t == S - 1) store_bf16x8(a.out + off, h);
             else store_bf16x8(a.hbuf[t & 1] + hs_index(row, unit, a.Bp), h);
           }

@@ -299,8 +299,12 @@ void build_op(Program& P, const Node& n, Op& op) {
     const auto& whh = pdecl(1);
     if (x.shape.size() != 3) fail(DUET_ESHAPE, "%" + n.name + ": input must be [S, B, E]");
     const int S = (int)x.shape[0], B = (int)x.shape[1], E = (int)x.shape[2], H = (int)whh.shape[1];
-    if (wih.shape[0] != G * H || wih.shape[1] != E || whh.shape[0] != G * H || n.shape[1] != H || n.shape[0] != B)
+    // seq=1: the output is every h_t, [S, B, H] time-major (a lower layer of a stacked RNN)
+    const bool seq = n.attr_int("seq", 0) != 0;
+    if (wih.shape[0] != G * H || wih.shape[1] != E || whh.shape[0] != G * H)
       fail(DUET_ESHAPE, "%" + n.name + ": rnn weight shapes");
+    if (seq ? n.shape != std::vector<int64_t>{S, B, H} : n.shape != std::vector<int64_t>{B, H})
+      fail(DUET_ESHAPE, "%" + n.name + (seq ? ": output must be [S, B, H]" : ": output must be [B, H]"));
     need_dtype(n, wih.dtype, whh.dtype, "W_ih");
     need_dtype(n, x.dtype, wih.dtype, "input");
     need_dtype(n, n.dtype, x.dtype, "output");
@@ -375,7 +379,12 @@ void build_op(Program& P, const Node& n, Op& op) {
         CK(cudaMemsetAsync(counter, 0, sizeof(unsigned), st));
         CUtensorMap tx = make_tmap_bf16_2d(T[in], (int64_t)S * B, E, 128);
         RnnPersistArgs r = ra;
-        r.out = (__nv_bfloat16*)T[me];
+        if (seq) {
+          r.seq = (__nv_bfloat16*)T[me];
+          r.out = r.seq + (size_t)(S - 1) * B * H;
+        } else {
+          r.out = (__nv_bfloat16*)T[me];
+        }
         rnn_persist(kind, bn, tx, t_h0, t_h1, t_w, r, grid, st);
       };
       op.n_kernels = 1;
@@ -403,12 +412,15 @@ void build_op(Program& P, const Node& n, Op& op) {
           e2.bias = bias;
           e2.c_state = cst;
           e2.h_prev = hb[(t + 1) & 1];
-          e2.h_next = (t == S - 1) ? T[me] : hb[t & 1];
+          e2.h_next = (t == S - 1 && !seq) ? T[me] : hb[t & 1];
           e2.H = H;
           e2.kx = Ep / 64;
           e2.x_row0 = t * B;
           // t = 0: h_{-1} = 0, so only the x_t part of K contributes
           gemm_tc_maps(t_h[(t + 1) & 1], t_w, B, Np, t == 0 ? Ep : Kc, bn, e2, kind, 1, st, &tx);
+          if (seq)
+            CK(cudaMemcpyAsync((char*)T[me] + (size_t)t * B * H * es, hb[t & 1], (size_t)B * H * es,
+                               cudaMemcpyDeviceToDevice, st));
         }
       };
       op.n_kernels = S;
@@ -429,8 +441,10 @@ void build_op(Program& P, const Node& n, Op& op) {
         if (kind == EPI_LSTM) CK(cudaMemsetAsync(cst, 0, (size_t)B * H * 4, st));
         gemm_simt(T[in], xb, Wih, xb, bias, gx, 0, S * B, G * H, E, ACT_NONE, st);
         for (int t = 0; t < S; ++t) {
-          void* hn = (t == S - 1) ? T[me] : hb[t & 1];
-          rnn_step_simt(kind, gx + (size_t)t * B * G * H, Whh, xb, bhn, hb[(t + 1) & 1], hn, xb, cst, B, H, st);
+          // seq: h_t goes straight into its slice of the [S, B, H] output and is read back from there
+          void* hn = seq ? (char*)T[me] + (size_t)t * B * H * es : (t == S - 1) ? T[me] : hb[t & 1];
+          const void* hp = (seq && t > 0) ? (const char*)T[me] + (size_t)(t - 1) * B * H * es : hb[(t + 1) & 1];
+          rnn_step_simt(kind, gx + (size_t)t * B * G * H, Whh, xb, bhn, hp, hn, xb, cst, B, H, st);
         }
       };
       op.n_kernels = 1 + S;

@@ -106,14 +106,24 @@ class _Builder:
         return self.node(name, "mlp", args, out_dt or self.dt, (m, dims[-1]), act=act,
                          last_act=last_act)
 
-    def rnn(self, name, kind, x, e, h, s, b):
+    def rnn(self, name, kind, x, e, h, s, b, seq=False):
+        """seq=True: output every h_t as [S, B, H] (a lower layer of a stacked RNN)."""
         g = 4 if kind == "lstm" else 3
         bd = 1.0 / math.sqrt(h)
         Wih = self.param(f"{name}_Wih", self.dt, (g * h, e), ("uniform", bd))
         Whh = self.param(f"{name}_Whh", self.dt, (g * h, h), ("uniform", bd))
         bih = self.param(f"{name}_bih", "f32", (g * h,), ("uniform", bd))
         bhh = self.param(f"{name}_bhh", "f32", (g * h,), ("uniform", bd))
+        if seq:
+            return self.node(name, kind, [x, Wih, Whh, bih, bhh], self.dt, (s, b, h), seq=1)
         return self.node(name, kind, [x, Wih, Whh, bih, bhh], self.dt, (b, h))
+
+    def stacked_rnn(self, name, kind, x, e, h, s, b, layers=1):
+        """`layers` stacked RNNs (Fig. 14): layers 0..L-2 return their whole output
+        sequence, the top layer h_S.  The top layer keeps the plain name (layers=1 is the plain RNN)."""
+        for li in range(layers - 1):
+            x = self.rnn(f"{name}_l{li}", kind, x, e if li == 0 else h, h, s, b, seq=True)
+        return self.rnn(name, kind, x, e if layers == 1 else h, h, s, b)
 
     def conv_bn(self, name, x, n, h, w, cin, cout, k, stride, pad, act, gamma=(0.5, 1.5)):
         ho = (h + 2 * pad - k) // stride + 1
@@ -130,25 +140,45 @@ class _Builder:
 
     def resnet18(self, prefix, x, n, h, w):
         """torchvision ResNet-18 topology in NHWC -> [n, 512]."""
+        return self.resnet(prefix, x, n, h, w, 18)
+
+    RESNET_BLOCKS = {18: ("basic", (2, 2, 2, 2)), 34: ("basic", (3, 4, 6, 3)),
+                     50: ("bottleneck", (3, 4, 6, 3)), 101: ("bottleneck", (3, 4, 23, 3))}
+
+    def resnet(self, prefix, x, n, h, w, depth=18):
+        """torchvision ResNet-`depth` (He et al.; 18/34 BasicBlock, 50/101 Bottleneck with the stride
+        on the 3x3 conv, "v1.5") in NHWC -> [n, 512] (18/34) or [n, 2048] (50/101).  The depths
+        are Fig. 15's ("Varying the CNN depths")."""
+        kind, blocks = self.RESNET_BLOCKS[depth]
+        exp = 1 if kind == "basic" else 4
         c, h, w = self.conv_bn(f"{prefix}_stem", x, n, h, w, 3, 64, 7, 2, 3, "relu")
         ho, wo = (h + 2 - 3) // 2 + 1, (w + 2 - 3) // 2 + 1
         c = self.node(f"{prefix}_pool", "maxpool", [c], self.dt, (n, ho, wo, 64), k=3, stride=2, pad=1)
         h, w, cin = ho, wo, 64
-        for li, cout in enumerate([64, 128, 256, 512]):
-            for bi in range(2):
+        for li, width in enumerate([64, 128, 256, 512]):
+            cout = width * exp
+            for bi in range(blocks[li]):
                 stride = 2 if (li > 0 and bi == 0) else 1
                 nm = f"{prefix}_l{li + 1}b{bi}"
-                y, h2, w2 = self.conv_bn(nm + "_c1", c, n, h, w, cin, cout, 3, stride, 1, "relu")
-                # residual-branch BN gamma ~ U(0.1, 0.3): keeps activations O(1) through the stack
-                # like a trained network (an untrained Kaiming ResNet doubles the variance per block)
-                y, h2, w2 = self.conv_bn(nm + "_c2", y, n, h2, w2, cout, cout, 3, 1, 1, "none", gamma=(0.1, 0.3))
+                # residual-branch BN gamma ~ U(0.1, 0.3) on the block's last conv: keeps activations
+                # O(1) through the stack like a trained network (an untrained Kaiming ResNet doubles
+                # the variance per block)
+                if kind == "basic":
+                    y, h2, w2 = self.conv_bn(nm + "_c1", c, n, h, w, cin, cout, 3, stride, 1, "relu")
+                    y, h2, w2 = self.conv_bn(nm + "_c2", y, n, h2, w2, cout, cout, 3, 1, 1, "none",
+                                             gamma=(0.1, 0.3))
+                else:
+                    y, _, _ = self.conv_bn(nm + "_c1", c, n, h, w, cin, width, 1, 1, 0, "relu")
+                    y, h2, w2 = self.conv_bn(nm + "_c2", y, n, h, w, width, width, 3, stride, 1, "relu")
+                    y, h2, w2 = self.conv_bn(nm + "_c3", y, n, h2, w2, width, cout, 1, 1, 0, "none",
+                                             gamma=(0.1, 0.3))
                 if stride != 1 or cin != cout:
                     sc, _, _ = self.conv_bn(nm + "_ds", c, n, h, w, cin, cout, 1, stride, 0, "none")
                 else:
                     sc = c
                 c = self.node(nm + "_add", "add", [y, sc], self.dt, (n, h2, w2, cout), act="relu")
                 h, w, cin = h2, w2, cout
-        return self.node(f"{prefix}_gap", "avgpool", [c], self.dt, (n, 512))
+        return self.node(f"{prefix}_gap", "avgpool", [c], self.dt, (n, cin))
 
 
 # ------------------------------------------------------------------------------------------
@@ -222,26 +252,32 @@ def c3_two_tower(batch=256, seq=64, vocab=32768, emb=256, hidden=512, dt="bf16")
 # Join sigma(w . concat[512, 1024, 256] + b).
 # ------------------------------------------------------------------------------------------
 def c4_hybrid(batch=64, image=224, seq=64, vocab=32768, emb=256, gru_hidden=1024, fields=8,
-              rows=100_000, mlp_out=256, dt="bf16") -> Workload:
+              rows=100_000, mlp_out=256, rnn_layers=1, resnet=18, ffn_layers=1, dt="bf16") -> Workload:
+    """`rnn_layers`, `resnet` and `ffn_layers` are the model variations of PAPER.md:89 (§VI-D,
+    Figs. 14-16: stacked RNN 1/2/4/8, ResNet 18/34/50/101, FFN depth); `batch` is Fig. 17's.
+    The defaults are BASELINE.json:10's configuration."""
     B = _Builder("c4_hybrid", 4, dt)
     img = B.input("image", dt, (batch, image, image, 3), ("normal", 1.0))
-    cnn = B.resnet18("cnn", img, batch, image, image)
+    cnn = B.resnet("cnn", img, batch, image, image, resnet)
+    d_cnn = 512 if resnet in (18, 34) else 2048
     tok = B.input("tok", "i32", (batch, seq), ("randint", vocab))
     E = B.param("tok_E", dt, (vocab, emb), ("normal", 1.0))
     x = B.node("tok_x", "embed_seq", [tok, E], dt, (seq, batch, emb))
-    rnn = B.rnn("gru", "gru", x, emb, gru_hidden, seq, batch)
+    rnn = B.stacked_rnn("gru", "gru", x, emb, gru_hidden, seq, batch, rnn_layers)
     raw = B.input("raw", "i64", (batch, fields), ("randint", 1 << 31))
     ids = B.node("ids", "hash_mod", [raw], "i32", (batch, fields), V=rows)
     T = B.param("mlp_E", dt, (fields, rows, 64), ("normal", 1.0))
     f = B.node("mlp_x", "gather_concat", [ids, T], dt, (batch, fields * 64))
     m = B.linear("mlp_fc", f, fields * 64, mlp_out, batch, act="relu")
-    d = 512 + gru_hidden + mlp_out
+    for li in range(1, ffn_layers):
+        m = B.linear(f"mlp_fc{li}", m, mlp_out, mlp_out, batch, act="relu")
+    d = d_cnn + gru_hidden + mlp_out
     hw = B.param("head_w", "f32", (d,), ("uniform", 1.0 / math.sqrt(d)))
     hb = B.param("head_b", "f32", (1,), ("uniform", 0.1))
     y = B.node("y", "concat_head", [cnn, rnn, m, hw, hb], "f32", (batch, 1), act="sigmoid")
     B.output(y)
     B.outputs = [("y", "f32", (batch, 1))]
-    return B.build(batch, config=4)
+    return B.build(batch, config=4, rnn_layers=rnn_layers, resnet=resnet, ffn_layers=ffn_layers)
 
 
 # ------------------------------------------------------------------------------------------

@@ -74,6 +74,17 @@ def test_partition_bit_exact_configs(cfg, small, gran):
     _same_partition(W.build(cfg, small=small).ir, gran)
 
 
+@pytest.mark.parametrize("var", [dict(rnn_layers=8), dict(resnet=34), dict(resnet=50), dict(resnet=101),
+                                 dict(ffn_layers=8), dict(batch=2)])
+@pytest.mark.parametrize("gran", ["coarse", "op"])
+def test_partition_bit_exact_model_variations(var, gran):
+    """PAPER.md:89 §VI-D variations of c4 (full size): libduet's partition == the oracle's; at
+    coarse granularity the branches stay one subgraph each (CNN, RNN, FFN + join)."""
+    p, _ = _same_partition(W.build("c4", **var).ir, gran)
+    if gran == "coarse":
+        assert p["n_sg"] == 4
+
+
 def random_dag_ir(rng, n_nodes, n_inputs=2):
     lines = [f"%x{i} = input() : f32[8,{4 + i}]" for i in range(n_inputs)]
     names = []

@@ -242,6 +242,80 @@ def test_rnn_node(kind, S, B, E, H, dt):
     assert err <= TOL[dt], err
 
 
+@pytest.mark.parametrize("kind,S,B,E,H,dt", [
+    ("gru", 5, 200, 64, 72, "bf16"),      # persistent kernel, one tile per CTA
+    ("lstm", 4, 300, 64, 136, "bf16"),
+    ("lstm", 3, 2048, 128, 256, "bf16"),  # persistent kernel, several tiles per CTA (state in HBM)
+    ("gru", 4, 33, 24, 40, "f32"),        # CUDA-core parity path
+])
+def test_rnn_node_seq_output(kind, S, B, E, H, dt):
+    """Stacked-RNN lower layer (seq=1, Fig. 14): every h_t, [S, B, H] time-major."""
+    G = 4 if kind == "lstm" else 3
+    ir = _single_node_graph(
+        f"%y = {kind}(%x, @Wih, @Whh, @bih, @bhh) {{seq=1}} : {dt}[{S},{B},{H}]",
+        {"Wih": (dt, (G * H, E)), "Whh": (dt, (G * H, H)), "bih": ("f32", (G * H,)), "bhh": ("f32", (G * H,))},
+        {"x": (dt, (S, B, E))})
+    sc = 1.0 / np.sqrt(H)
+    x = _rand((S, B, E), dt, 1.0, 21)
+    Wih, Whh = _rand((G * H, E), dt, sc, 22), _rand((G * H, H), dt, sc, 23)
+    bih, bhh = _rand((G * H,), "f32", sc, 24), _rand((G * H,), "f32", sc, 25)
+    g = duet.Graph(ir)
+    g.bind_all({"Wih": Wih.cuda(), "Whh": Whh.cuda(), "bih": bih.cuda(), "bhh": bhh.cuda()})
+    y = torch.empty((S, B, H), dtype=torch.bfloat16 if dt == "bf16" else torch.float32, device="cuda")
+    g.node_run("y", [x.cuda()], y)
+    torch.cuda.synchronize()
+    f = lambda t, d: OF.to_f64(to_np(t), d)
+    want = (OF.lstm if kind == "lstm" else OF.gru)(f(x, dt), f(Wih, dt), f(Whh, dt), f(bih, "f32"), f(bhh, "f32"),
+                                                   seq=True)
+    assert want.shape == (S, B, H)
+    err = rel_err(y.float().cpu().numpy(), want)
+    print(f"[parity] {kind} seq S{S} B{B} E{E} H{H} {dt}: rel err {err:.3e}")
+    assert err <= TOL[dt], err
+
+
+VARIATIONS = [  # PAPER.md:89 §VI-D on c4 (Figs. 14-17): (rnn_layers, resnet, ffn_layers, batch, dt)
+    (2, 18, 1, 3, "bf16"), (4, 18, 1, 3, "bf16"), (1, 34, 1, 3, "bf16"), (1, 50, 1, 3, "bf16"),
+    (1, 101, 1, 2, "bf16"), (1, 18, 4, 3, "bf16"), (1, 18, 1, 32, "bf16"), (2, 50, 3, 2, "f32"),
+]
+
+
+@pytest.mark.parametrize("layers,resnet,ffn,batch,dt", VARIATIONS)
+def test_model_variation_parity(layers, resnet, ffn, batch, dt):
+    wl = W.build("c4", small=True, dt=dt, branch_outputs=True, rnn_layers=layers, resnet=resnet,
+                 ffn_layers=ffn, batch=batch)
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    want = _oracle_outputs(wl, sess.params, dict(zip(wl.inputs, inputs)))
+    outs = sess.outputs()
+    sess.run(sess.schedule(), inputs, outs)
+    torch.cuda.synchronize()
+    for (name, _, _), y in zip(wl.outputs, outs):
+        err = rel_err(y.float().cpu().numpy(), want[name])
+        print(f"[parity] c4 L{layers} R{resnet} F{ffn} B{batch} {dt} {name}: rel err {err:.3e}")
+        assert err <= TOL[dt], (name, err)
+
+
+@pytest.mark.parametrize("layers,resnet,ffn", [(8, 18, 1), (1, 101, 1), (1, 18, 8)])
+def test_model_variation_full_size_sampled(layers, resnet, ffn):
+    """The deepest Fig. 14-16 variations at c4's full size (bench launch configuration); the oracle
+    evaluates 2 sampled rows."""
+    wl = W.build("c4", branch_outputs=True, rnn_layers=layers, resnet=resnet, ffn_layers=ffn)
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    outs = sess.outputs()
+    sess.run(sess.schedule(), inputs, outs)
+    torch.cuda.synchronize()
+    rows = np.array([wl.batch - 1, 17])
+    oparams = {k: (lazy_rows(spec) if spec.numel > 10_000_000 else to_np(sess.params[k]))
+               for k, spec in wl.params.items()}
+    oin = {k: to_np(t)[rows] for k, t in zip(wl.inputs, inputs)}
+    want = OF.run(wl.ir, oparams, oin)
+    for (name, _, _), y in zip(wl.outputs, outs):
+        err = rel_err(y.float().cpu().numpy()[rows], want[name])
+        print(f"[parity] full c4 L{layers} R{resnet} F{ffn} {name}: rel err {err:.3e}")
+        assert err <= TOL["bf16"], (name, err)
+
+
 @pytest.mark.parametrize("cfg,mode", [("c5", duet.GREEDY_CORRECTION), ("c5", duet.RANDOM_CORRECTION),
                                       ("c3", duet.GREEDY_CORRECTION)])
 def test_measured_correction(cfg, mode):

@@ -155,11 +155,13 @@ def test_maxpool_avgpool_vs_torch():
     np.testing.assert_allclose(F.avgpool(x), x.reshape(2, -1, 3).mean(1), rtol=1e-14)
 
 
-def test_resnet18_small_vs_torch_f64():
-    """The workload's ResNet-18 IR through the oracle == a torch float64 ResNet-18 built here
-    from nn.Conv2d / nn.BatchNorm2d (torchvision BasicBlock topology)."""
+@pytest.mark.parametrize("depth", [18, 34, 50, 101])
+def test_resnet_small_vs_torch_f64(depth):
+    """The workload's ResNet-`depth` IR through the oracle == a torch float64 ResNet built here
+    from nn.functional conv2d / batch_norm (torchvision BasicBlock for 18/34, Bottleneck with the
+    stride on the 3x3 conv for 50/101; Fig. 15's depths)."""
     from paper_conf_ipps_zhanghl21_b200 import workloads as W
-    wl = W.build("c4", small=True, dt="f32")
+    wl = W.build("c4", small=True, dt="f32", resnet=depth)
     params = {k: s.materialize().numpy() for k, s in wl.params.items()}
     img = wl.inputs["image"].materialize().numpy()
     vals = F.run(wl.ir, params, {"image": img, "tok": wl.inputs["tok"].materialize().numpy(),
@@ -174,21 +176,73 @@ def test_resnet18_small_vs_torch_f64():
                                            P(name + "_beta"), training=False, eps=1e-5)
         return torch.relu(y) if relu else y
 
+    blocks = {18: (2, 2, 2, 2), 34: (3, 4, 6, 3), 50: (3, 4, 6, 3), 101: (3, 4, 23, 3)}[depth]
+    exp = 1 if depth < 50 else 4
     x = torch.tensor(img, dtype=torch.float64).permute(0, 3, 1, 2)
     x = cbn(x, "cnn_stem", 2, 3, True)
     x = torch.nn.functional.max_pool2d(x, 3, 2, 1)
     cin = 64
-    for li, cout in enumerate([64, 128, 256, 512]):
-        for bi in range(2):
+    for li, width in enumerate([64, 128, 256, 512]):
+        cout = width * exp
+        for bi in range(blocks[li]):
             s = 2 if (li > 0 and bi == 0) else 1
             nm = f"cnn_l{li + 1}b{bi}"
-            y = cbn(x, nm + "_c1", s, 1, True)
-            y = cbn(y, nm + "_c2", 1, 1, False)
+            if exp == 1:
+                y = cbn(x, nm + "_c1", s, 1, True)
+                y = cbn(y, nm + "_c2", 1, 1, False)
+            else:
+                y = cbn(x, nm + "_c1", 1, 0, True)
+                y = cbn(y, nm + "_c2", s, 1, True)
+                y = cbn(y, nm + "_c3", 1, 0, False)
             sc = cbn(x, nm + "_ds", s, 0, False) if (s != 1 or cin != cout) else x
             x = torch.relu(y + sc)
             cin = cout
     want = x.mean(dim=(2, 3)).numpy()
+    assert want.shape[1] == 512 * exp
     np.testing.assert_allclose(vals["cnn_gap"], want, rtol=1e-10, atol=1e-12)
+
+
+@pytest.mark.parametrize("layers", [1, 2, 4])
+def test_stacked_gru_vs_torch_f64(layers):
+    """Stacked RNN (Fig. 14): the workload's `layers`-deep GRU IR (lower layers emit
+    their whole sequence, `seq=1`) through the oracle == torch nn.GRU(num_layers=layers) in f64."""
+    from paper_conf_ipps_zhanghl21_b200 import workloads as W
+    wl = W.build("c4", small=True, dt="f32", rnn_layers=layers)
+    params = {k: s.materialize().numpy() for k, s in wl.params.items()}
+    ins = {k: s.materialize().numpy() for k, s in wl.inputs.items()}
+    vals = F.run(wl.ir, params, ins, keep_all=True)
+    E, H = params["tok_E"].shape[1], params["gru_Whh"].shape[1]
+    mod = torch.nn.GRU(E, H, num_layers=layers).double()
+    names = [f"gru_l{i}" for i in range(layers - 1)] + ["gru"]
+    with torch.no_grad():
+        for i, nm in enumerate(names):
+            for a, b in (("Wih", "weight_ih"), ("Whh", "weight_hh"), ("bih", "bias_ih"), ("bhh", "bias_hh")):
+                getattr(mod, f"{b}_l{i}").copy_(torch.tensor(params[f"{nm}_{a}"], dtype=torch.float64))
+    x = torch.tensor(vals["tok_x"])
+    with torch.no_grad():
+        out, hn = mod(x)
+    np.testing.assert_allclose(vals["gru"], hn[-1].numpy(), rtol=1e-11, atol=1e-13)
+    if layers > 1:  # a lower layer's seq output is torch's per-layer output sequence
+        sub = torch.nn.GRU(E, H).double()
+        with torch.no_grad():
+            for a, b in (("Wih", "weight_ih"), ("Whh", "weight_hh"), ("bih", "bias_ih"), ("bhh", "bias_hh")):
+                getattr(sub, f"{b}_l0").copy_(getattr(mod, f"{b}_l0"))
+            seq0, _ = sub(x)
+        np.testing.assert_allclose(vals["gru_l0"], seq0.numpy(), rtol=1e-11, atol=1e-13)
+
+
+def test_stacked_lstm_vs_torch_f64():
+    S, B, E, H = 5, 4, 6, 7
+    torch.manual_seed(3)
+    mod = torch.nn.LSTM(E, H, num_layers=3).double()
+    x = torch.randn(S, B, E, dtype=torch.float64)
+    with torch.no_grad():
+        out, (hn, _) = mod(x)
+    v = x.numpy()
+    for i in range(3):
+        w = [getattr(mod, f"{n}_l{i}").detach().numpy() for n in ("weight_ih", "weight_hh", "bias_ih", "bias_hh")]
+        v = F.lstm(v, *w, seq=i < 2)
+    np.testing.assert_allclose(v, hn[-1].numpy(), rtol=1e-11, atol=1e-13)
 
 
 # ---- joins --------------------------------------------------------------------------------------
