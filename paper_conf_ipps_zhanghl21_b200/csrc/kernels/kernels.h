@@ -39,6 +39,11 @@ struct TcEpilogue {
   int kx = 0;                  // k-blocks read from the X map (x_t) before switching to A (h)
   int x_row0 = 0;              // row offset of x_t in the X map ([S*B, E] time-major)
   int tma_store = 0;  // EPI_BIAS_ACT: 1 = output tile leaves through TMA stores (map passed separately)
+  int early_a = 0;  // pair GEMM: issue the first A stages right after the PDL wait (before TMEM alloc)
+  // pair GEMM with a gathered A operand (gather-concat fused into the GEMM, gemm2_gather): row b of
+  // A is [E[0, ids[b,0]], ..., E[F-1, ids[b,F-1]]], E = [F, R, 64] bf16, K = 64 F
+  const int32_t* g_ids = nullptr;  // [M, F]
+  int g_F = 0, g_R = 0;
   int dbg = 0;  // micro-benchmark switches: 1 = skip UMMA, 2 = skip TMA, 4 = epilogue backoff
 };
 
@@ -104,6 +109,14 @@ bool mlp_chain_ok(int M, const int* N, const int* K, int L);
 void mlp_chain(const MlpChainMaps& maps, MlpChainArgs a, int sms, cudaStream_t st);
 CUtensorMap mlp_chain_out_map(void* out, int M, int N);
 
+// CTA-pair GEMM with the deep tower's gather-concat fused into the A producer (gemm_tc2.cu):
+// tE = make_tmap_gather4(E, F * R) ([F*R, 64] rows, box 64 x 1, tile::gather4 loads 4 rows each);
+// ep.g_ids / g_F / g_R set; K = 64 F, F <= kGatherMaxF.  bf16 output.
+constexpr int kGatherMaxF = 32;
+CUtensorMap make_tmap_gather4(const void* E, int64_t rows);
+bool gemm_tc2_gather_ok(int M, int N, int K, int F, int64_t R);
+void gemm_tc2_gather(const CUtensorMap& tE, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
+                     cudaStream_t st);
 // CTA-pair GEMM (gemm_tc2.cu): 256 x bn tiles, bn in {64,128,256}; W map box rows = bn / 2.
 int tc2_pick_bn(int M, int N, int K, int num_sms);
 // pairs per cluster that share the A tile by TMA multicast (A map box rows = 128 / np)

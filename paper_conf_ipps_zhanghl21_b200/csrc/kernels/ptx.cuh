@@ -414,6 +414,16 @@ __device__ __forceinline__ void tma_load_2d_2sm(const CUtensorMap* m, uint32_t b
       "l"((uint64_t)m), "r"(bar_cl), "r"(c0), "r"(c1)
       : "memory");
 }
+// 2-SM gather of 4 rows (tile::gather4): rows r0..r3 of a [rows, cols] map whose box is
+// {cols_box, 1}; the 4 rows land contiguously at dst (swizzled by address like a tile load).
+__device__ __forceinline__ void tma_gather4_2sm(const CUtensorMap* m, uint32_t bar_cl, void* dst, int c0, int r0,
+                                                int r1, int r2, int r3) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes "
+      "[%0], [%1, {%3, %4, %5, %6, %7}], [%2];" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)m), "r"(bar_cl), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3)
+      : "memory");
+}
 // 2-SM TMA with multicast: copies land at the same smem offset in every CTA of `mask`; each
 // destination's transaction bytes complete on its pair leader's barrier (peer bit cleared).
 __device__ __forceinline__ void tma_load_2d_2sm_mc(const CUtensorMap* m, uint64_t* bar, void* dst, int c0, int c1,

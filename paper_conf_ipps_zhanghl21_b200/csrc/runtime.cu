@@ -39,6 +39,9 @@ struct Program {
   std::set<int> fused_adds;
   std::map<int, std::vector<int>> chains;  // head linear node -> chain of linear nodes (mlp_chain.cu)
   std::map<int, Op> chain_ops;             // head -> one launch for the whole chain
+  std::map<int, int> gather_fused;         // linear node -> the gather_concat it absorbs (gemm2 GA)
+  std::map<int, int> fused_gathers;        // gather_concat node -> the linear that gathers its rows
+  std::map<int, Op> gather_ops;            // linear node -> fused gather + GEMM launch
   ~Program() {
     int prev = 0;
     cudaGetDevice(&prev);
@@ -714,6 +717,56 @@ void plan_linear_chains(Program& P, int sms) {
   }
 }
 
+// gather_concat -> linear (the deep tower's first layer, SURVEY.md §8(a) A4 + A5): when the gather's
+// only consumer is a bf16 pair-GEMM linear with D = 64 rows and both sit in the same subgraph at
+// run time, the GEMM's producer warp gathers the embedding rows straight into the swizzled A stages
+// (tile::gather4 TMA) -- no [B, 64 F] round trip through HBM and one launch fewer.  The node-level
+// ops stay unfused (duet_node_run, or the two nodes in different subgraphs).  Opt-in
+// (DUET_GATHER_FUSE=1): measured slower than the two kernels (gemm_tc2.cu gemm_tc2_gather_ok).
+void plan_gather_fusion(Program& P, int sms) {
+  const Graph& g = *P.g;
+  std::vector<int> n_cons(g.nodes.size(), 0);
+  for (auto& n : g.nodes)
+    for (int u : n.inputs) n_cons[u]++;
+  std::set<int> outs(g.outputs.begin(), g.outputs.end()), in_chain;
+  for (auto& kv : P.chains)
+    for (int c : kv.second) in_chain.insert(c);
+  for (auto& c : g.nodes) {
+    if (c.op != "linear" || c.arg_nodes.size() != 1 || c.params.size() != 2 || in_chain.count(c.id)) continue;
+    const Node& x = g.nodes[c.arg_nodes[0]];
+    if (x.op != "gather_concat" || n_cons[x.id] != 1 || outs.count(x.id) || x.params.size() != 1) continue;
+    const auto& e = g.params.at(x.params[0]);
+    const auto& w = g.params.at(c.params[0]);
+    if (e.dtype != kBF16 || w.dtype != kBF16 || c.dtype != kBF16 || e.shape.size() != 3 || e.shape[2] != 64) continue;
+    const int M = (int)x.shape[0], F = (int)e.shape[0], N = (int)w.shape[0], K = (int)w.shape[1];
+    const int64_t R = e.shape[1];
+    if (!gemm_tc2_gather_ok(M, N, K, F, R)) continue;
+    const char* bn_env = getenv("DUET_GEMM_BN");
+    const int bn = bn_env ? atoi(bn_env) : tc2_pick_bn(M, N, K, sms);
+    CUtensorMap tw = make_tmap_bf16_2d(P.param(c.params[0]), N, K, bn / 2);
+    CUtensorMap tE = make_tmap_gather4(P.param(x.params[0]), (int64_t)F * R);
+    const float* bias = (const float*)P.param(c.params[1]);
+    const int act = act_code(c.attr_str("act", "none"));
+    const int ids = x.arg_nodes[0], me = c.id;
+    Op op;
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      TcEpilogue ep;
+      ep.bias = bias;
+      ep.out = T[me];
+      ep.ldo = N;
+      ep.act = act;
+      ep.g_ids = (const int32_t*)T[ids];
+      ep.g_F = F;
+      ep.g_R = (int)R;
+      gemm_tc2_gather(tE, tw, M, N, K, bn, ep, st);
+    };
+    op.n_kernels = 1;
+    P.gather_fused[c.id] = x.id;
+    P.fused_gathers[x.id] = c.id;
+    P.gather_ops[c.id] = op;
+  }
+}
+
 std::shared_ptr<Program> ensure_program(Graph* g) {
   if (g->prog) return g->prog;
   for (auto& name : g->param_order)
@@ -733,6 +786,7 @@ std::shared_ptr<Program> ensure_program(Graph* g) {
   plan_residual_fusion(*P);
   for (auto& n : g->nodes) build_op(*P, n, P->ops[n.id]);
   plan_linear_chains(*P, num_sms(dev));
+  plan_gather_fusion(*P, num_sms(dev));
   CK(cudaDeviceSynchronize());
   g->prog = P;
   return P;
@@ -746,10 +800,25 @@ bool chain_in_subgraph(const Program& P, const Partition& part, int s, int head)
   return true;
 }
 
+// the gather is done by its consumer GEMM (plan_gather_fusion) when both run in subgraph s
+bool gather_absorbed(const Program& P, const Partition& part, int s, int v) {
+  auto it = P.fused_gathers.find(v);
+  return it != P.fused_gathers.end() && part.node_to_sg[v] == s && part.node_to_sg[it->second] == s;
+}
+const Op* gathering_linear(const Program& P, const Partition& part, int s, int v) {
+  auto it = P.gather_fused.find(v);
+  if (it == P.gather_fused.end() || part.node_to_sg[it->second] != s || part.node_to_sg[v] != s) return nullptr;
+  return &P.gather_ops.at(v);
+}
+
 void launch_subgraph(const Program& P, const Partition& part, int s, const Ptrs& T, cudaStream_t st) {
   std::set<int> skip;
   for (int v : part.sg_nodes[s]) {
-    if (skip.count(v)) continue;
+    if (skip.count(v) || gather_absorbed(P, part, s, v)) continue;
+    if (const Op* go = gathering_linear(P, part, s, v)) {
+      go->launch(T, st);
+      continue;
+    }
     if (chain_in_subgraph(P, part, s, v)) {
       P.chain_ops.at(v).launch(T, st);
       for (int c : P.chains.at(v)) skip.insert(c);
@@ -763,7 +832,11 @@ int subgraph_kernels(const Program& P, const Partition& part, int s) {
   int nk = 0;
   std::set<int> skip;
   for (int v : part.sg_nodes[s]) {
-    if (skip.count(v)) continue;
+    if (skip.count(v) || gather_absorbed(P, part, s, v)) continue;
+    if (gathering_linear(P, part, s, v)) {
+      nk += 1;
+      continue;
+    }
     if (chain_in_subgraph(P, part, s, v)) {
       nk += 1;
       for (int c : P.chains.at(v)) skip.insert(c);

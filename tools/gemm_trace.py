@@ -22,13 +22,15 @@ x = torch.randn(M, K, device="cuda").to(torch.bfloat16)
 y = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
 s = torch.cuda.Stream()
 lib = ctypes.CDLL(duet.LIB_PATH)
-names = ["entry", "prologue", "first TMA", "first stage in", "last commit", "acc ready", "epi done", "exit"]
+names = ["entry", "prologue", "first TMA", "first stage in", "last commit", "acc ready", "epi done", "exit",
+         "tmem loaded", "smem staged", "store issued", "store read", "cluster sync", "pdl wait", "tmem alloc",
+         "bias staged"]
 for rep in range(4):
     g.node_run("y", [x], y, s)
     s.synchronize()
-buf = (ctypes.c_ulonglong * (8 * 4096))()
-lib.duet_debug_tc2_trace(buf, 8 * 4096)
-a = np.frombuffer(buf, dtype=np.uint64).reshape(4096, 8).astype(np.int64)
+buf = (ctypes.c_ulonglong * (16 * 4096))()
+lib.duet_debug_tc2_trace(buf, 16 * 4096)
+a = np.frombuffer(buf, dtype=np.uint64).reshape(4096, 16).astype(np.int64)
 ctas = a[a[:, 0] > 0]
 t0 = ctas[:, 0].min()
 try:
