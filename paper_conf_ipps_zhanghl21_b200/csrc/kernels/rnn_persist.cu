@@ -52,7 +52,7 @@ struct RCfg {
   static constexpr int U = BN / 4;   // hidden units per tile
   static constexpr int UH = U / 2;   // units per epilogue thread
   static constexpr int B_BYTES = BN * RBK * 2;
-  static constexpr int TMEM_COLS = 2 * BN <= 128 ? 128 : 256;
+  static constexpr int TMEM_COLS = 2 * BN <= 128 ? 128 : 2 * BN <= 256 ? 256 : 512;
   static constexpr int EXTRA = 1024 + 512 + BN * 4;  // alignment slack + barriers + bias
 };
 // Shared-memory plan: [A ring: stages x 16 KB][W: resident (kx + kh blocks) or a ring of `stages`
@@ -385,17 +385,31 @@ __global__ void __launch_bounds__(kRThreads, 1)
           wait_sleep(&tfull[buf], (u >> 1) & 1);
           ptx::tc_fence_after();
           const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
+          // UH <= 16: every chunk's accumulators are read before the buffer is released; UH = 32
+          // (bn = 256) reads chunk by chunk (128 live floats would spill) and releases at the end
+          constexpr int CH = UH <= 16 ? UH / 8 : 1;
           float acc[UH / 8][4][8];
-#pragma unroll
-          for (int c = 0; c < UH / 8; ++c)
+          auto load_chunk = [&](int c) {
 #pragma unroll
             for (int g = 0; g < 4; ++g) ptx::tmem_ld8(tq + g * U + half * UH + 8 * c, acc[c][g]);
-          ptx::tc_fence_before();
-          __syncwarp();
-          if (lane == 0) ptx::mbar_arrive(&tempty[buf]);
+          };
+          auto release = [&]() {
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&tempty[buf]);
+          };
+          if constexpr (CH > 1) {
+#pragma unroll
+            for (int c = 0; c < UH / 8; ++c) load_chunk(c);
+            release();
+          }
           const __nv_bfloat16* hprev = a.hbuf[(t - 1) & 1];
 #pragma unroll
           for (int c = 0; c < UH / 8; ++c) {
+            if constexpr (CH == 1) {
+              load_chunk(c);
+              if (c == UH / 8 - 1) release();
+            }
             const int unit = (n0 / BN) * U + half * UH + 8 * c;
             if (row >= a.B || unit >= H) continue;
             const size_t off = (size_t)row * H + unit;
@@ -483,14 +497,19 @@ void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap&
 }
 
 template <int BN, int KIND>
+void launch_rp_multi(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1, const CUtensorMap& tw,
+                     RnnPersistArgs a, int grid, cudaStream_t st) {
+  // several tiles per CTA: W changes per tile, so it is streamed
+  a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
+  if (a.stages > 10) a.stages = 10;
+  return launch_rp<BN, KIND, false, true, 1>(tx, th0, th1, tw, a, grid, st);
+}
+
+template <int BN, int KIND>
 void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1, const CUtensorMap& tw,
                    RnnPersistArgs a, int grid, cudaStream_t st) {
   const bool multi = a.tiles_n * a.tiles_m > grid;
-  if (multi) {  // several tiles per CTA: W changes per tile, so it is streamed
-    a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
-    if (a.stages > 10) a.stages = 10;
-    return launch_rp<BN, KIND, false, true, 1>(tx, th0, th1, tw, a, grid, st);
-  }
+  if (multi) return launch_rp_multi<BN, KIND>(tx, th0, th1, tw, a, grid, st);
   static const int wres_env = getenv("DUET_RNN_WRES") ? atoi(getenv("DUET_RNN_WRES")) : 1;
   bool wres = false;
   a.stages = rp_plan(BN, a.kx + a.kh, &wres);
@@ -530,7 +549,13 @@ void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0
   if (kind == EPI_LSTM && bn == 128) return launch_rp_any<128, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_GRU && bn == 64) return launch_rp_any<64, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_GRU && bn == 128) return launch_rp_any<128, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
-  fail(DUET_EUNSUPPORTED, "rnn_persist: bn must be 64 or 128");
+  // 128 x 256 tiles (64 units) only with several tiles per CTA (large batches): half the W bytes per
+  // FLOP of bn = 128, double-buffered accumulators fill all 512 TMEM columns
+  if (bn == 256 && a.tiles_n * a.tiles_m > grid) {
+    if (kind == EPI_LSTM) return launch_rp_multi<256, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
+    return launch_rp_multi<256, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
+  }
+  fail(DUET_EUNSUPPORTED, "rnn_persist: bn must be 64 or 128 (256: several tiles per CTA only)");
 }
 
 }  // namespace duet

@@ -338,7 +338,11 @@ void build_op(Program& P, const Node& n, Op& op) {
         }
       }
       if (!rp_bn) {
-        rp_bn = rp_bn_env ? rp_bn_env : 128;
+        // several tiles per CTA: 128 x 256 tiles (64 units; half the W bytes per FLOP of 128 x 128,
+        // c5's b2/b4/b5 -9/-24/-25%) while they still outnumber the SMs (rnn_persist's bn = 256
+        // path is the multi-tile one), else 128 x 128
+        const int t256 = mt * ((H + 63) / 64);
+        rp_bn = (rp_bn_env == 256 || !rp_bn_env) ? (t256 > sms ? 256 : 128) : rp_bn_env;
         rp_grid = sms;
       }
     }

@@ -302,6 +302,8 @@ def test_rnn_node(kind, S, B, E, H, dt):
     ("gru", 5, 200, 64, 72, "bf16"),      # persistent kernel, one tile per CTA
     ("lstm", 4, 300, 64, 136, "bf16"),
     ("lstm", 3, 2048, 128, 256, "bf16"),  # persistent kernel, several tiles per CTA (state in HBM)
+    ("lstm", 3, 4096, 256, 512, "bf16"),  # several 128 x 256 tiles per CTA
+    ("gru", 3, 4000, 136, 520, "bf16"),   # 128 x 256 tiles, ragged B, H and E
     ("gru", 4, 33, 24, 40, "f32"),        # CUDA-core parity path
 ])
 def test_rnn_node_seq_output(kind, S, B, E, H, dt):
