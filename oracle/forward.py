@@ -45,6 +45,12 @@ def sigmoid(x):
     return out
 
 
+def gelu(x):
+    """GELU(x) = x * Phi(x) = 0.5 x (1 + erf(x / sqrt 2)) (the exact form BERT / MT-DNN use)."""
+    from scipy.special import erf
+    return 0.5 * x * (1.0 + erf(x / np.sqrt(2.0)))
+
+
 def act(x, name: str):
     if name in (None, "none"):
         return x
@@ -54,6 +60,8 @@ def act(x, name: str):
         return sigmoid(x)
     if name == "tanh":
         return np.tanh(x)
+    if name == "gelu":
+        return gelu(x)
     raise ValueError(name)
 
 
@@ -221,6 +229,55 @@ def mean_join(parts):
     return sigmoid(sum(p[:, 0] for p in parts) / len(parts)).reshape(-1, 1)
 
 
+# ---- MT-DNN ("shared layer ... lexicon encoder and a multi-layer bidirectional
+# Transformer encoder ... task-specific output layers", Fig. 3) ----------
+LN_EPS = 1e-12  # BERT's LayerNorm epsilon (MT-DNN's encoder is BERT's)
+
+
+def layernorm(x, gamma, beta, eps=LN_EPS):
+    """Over the last axis: (x - mean) / sqrt(var + eps) * gamma + beta (biased variance)."""
+    mu = x.mean(axis=-1, keepdims=True)
+    var = ((x - mu) ** 2).mean(axis=-1, keepdims=True)
+    return (x - mu) / np.sqrt(var + eps) * gamma + beta
+
+
+def bert_embed(tok, seg, Wtok, Wpos, Wseg, gamma, beta, eps=LN_EPS):
+    """Lexicon encoder: LN(E_tok[tok[b, s]] + E_pos[s] + E_seg[seg[b, s]]), rows b*S + s -> [B*S, H]."""
+    tok = np.asarray(tok, dtype=np.int64)
+    seg = np.asarray(seg, dtype=np.int64)
+    B, S = tok.shape
+    x = Wtok[tok] + Wpos[:S][None, :, :] + Wseg[seg]
+    return layernorm(x, gamma, beta, eps).reshape(B * S, -1)
+
+
+def attention(qkv, heads, seq):
+    """Bidirectional multi-head self-attention (Vaswani et al.; no mask: fixed length, R-31).
+    qkv = [Q | K | V] per row ([B*S, 3H], rows b*S + s; head h = columns h*dh .. of each part);
+    out[b, s, h] = softmax(Q_h K_h^T / sqrt(dh)) V_h -> [B*S, H]."""
+    M, H3 = qkv.shape
+    H = H3 // 3
+    dh = H // heads
+    B = M // seq
+    q = qkv[:, :H].reshape(B, seq, heads, dh).transpose(0, 2, 1, 3)
+    k = qkv[:, H:2 * H].reshape(B, seq, heads, dh).transpose(0, 2, 1, 3)
+    v = qkv[:, 2 * H:].reshape(B, seq, heads, dh).transpose(0, 2, 1, 3)
+    sc = q @ k.transpose(0, 1, 3, 2) / np.sqrt(dh)          # [B, heads, S, S]
+    sc = sc - sc.max(axis=-1, keepdims=True)
+    p = np.exp(sc)
+    p = p / p.sum(axis=-1, keepdims=True)
+    return (p @ v).transpose(0, 2, 1, 3).reshape(M, H)
+
+
+def add_layernorm(a, b, gamma, beta, eps=LN_EPS):
+    """Post-LN residual: LN(a + b)."""
+    return layernorm(a + b, gamma, beta, eps)
+
+
+def select_rows(x, stride, offset=0):
+    """Rows offset, offset + stride, ... (the [CLS] token of every sequence)."""
+    return x[offset::stride]
+
+
 # ---- graph evaluation -----------------------------------------------------------------------
 def run(ir, params: dict, inputs: dict, keep_all: bool = False) -> dict:
     """Evaluate the graph in topological order.  Returns {output name: float64 array}
@@ -283,6 +340,14 @@ def run(ir, params: dict, inputs: dict, keep_all: bool = False) -> dict:
             v = mean_join(A)
         elif op == "sigmoid":
             v = sigmoid(A[0])
+        elif op == "bert_embed":
+            v = bert_embed(A[0], A[1], *(P(p) for p in pn))
+        elif op == "attention":
+            v = attention(A[0], int(at["heads"]), int(at["seq"]))
+        elif op == "add_layernorm":
+            v = add_layernorm(A[0], A[1], P(pn[0]), P(pn[1]))
+        elif op == "select_rows":
+            v = select_rows(A[0], int(at["stride"]), int(at.get("offset", 0)))
         else:
             raise ValueError(f"oracle has no operator {op!r}")
         val[n.name] = v

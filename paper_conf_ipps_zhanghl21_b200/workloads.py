@@ -338,12 +338,57 @@ def c5_ensemble(batch=4096, fields=26, rows=1_000_000, vocab=32768, image=32,
     return B.build(batch, config=5)
 
 
+# ------------------------------------------------------------------------------------------
+# c6 — MT-DNN (Fig. 3; not a BASELINE.json config): shared
+# lexicon encoder + L-layer bidirectional Transformer encoder (BERT-base: L=12, H=768, 12 heads,
+# FFN 3072, post-LN, GELU) over S=128 tokens, then independent task-specific heads on the [CLS]
+# vector (MT-DNN's four GLUE task types: single-sentence classification (2), pairwise similarity
+# (1), pairwise classification (3), relevance ranking (1)), each pooler linear + tanh -> linear.
+# Batch 1 is the paper's inference setting.  All sizes (p).
+# ------------------------------------------------------------------------------------------
+def c6_mtdnn(batch=1, seq=128, layers=12, hidden=768, heads=12, ffn=3072, vocab=30522, tasks=(2, 1, 3, 1),
+             dt="bf16") -> Workload:
+    B = _Builder("c6_mtdnn", 6, dt)
+    M = batch * seq
+    tok = B.input("tok", "i32", (batch, seq), ("randint", vocab))
+    seg = B.input("seg", "i32", (batch, seq), ("randint", 2))
+    args = [tok, seg, B.param("tok_E", dt, (vocab, hidden), ("normal", 1.0)),
+            B.param("pos_E", dt, (seq, hidden), ("normal", 1.0)),
+            B.param("seg_E", dt, (2, hidden), ("normal", 1.0)),
+            B.param("emb_g", "f32", (hidden,), ("uniform_range", 0.8, 1.2)),
+            B.param("emb_b", "f32", (hidden,), ("normal", 0.1))]
+    x = B.node("emb", "bert_embed", args, dt, (M, hidden))
+
+    def ln_params(name):
+        return [B.param(f"{name}_g", "f32", (hidden,), ("uniform_range", 0.8, 1.2)),
+                B.param(f"{name}_b", "f32", (hidden,), ("normal", 0.1))]
+
+    for li in range(layers):
+        nm = f"L{li}"
+        qkv = B.linear(f"{nm}_qkv", x, hidden, 3 * hidden, M, act="none")
+        a = B.node(f"{nm}_att", "attention", [qkv], dt, (M, hidden), heads=heads, seq=seq)
+        o = B.linear(f"{nm}_o", a, hidden, hidden, M, act="none")
+        x1 = B.node(f"{nm}_ln1", "add_layernorm", [o, x] + ln_params(f"{nm}_ln1"), dt, (M, hidden))
+        f = B.linear(f"{nm}_ff1", x1, hidden, ffn, M, act="gelu")
+        f2 = B.linear(f"{nm}_ff2", f, ffn, hidden, M, act="none")
+        x = B.node(f"{nm}_ln2", "add_layernorm", [f2, x1] + ln_params(f"{nm}_ln2"), dt, (M, hidden))
+    cls = B.node("cls", "select_rows", [x], dt, (batch, hidden), stride=seq, offset=0)
+    outs = []
+    for ti, c in enumerate(tasks):
+        p = B.linear(f"task{ti}_pool", cls, hidden, hidden, batch, act="tanh")
+        outs.append(B.linear(f"task{ti}", p, hidden, c, batch, act="none", out_dt="f32"))
+    B.output(*outs)
+    B.outputs = [(f"task{ti}", "f32", (batch, c)) for ti, c in enumerate(tasks)]
+    return B.build(batch, config=6)
+
+
 CONFIGS = {
     "c1": c1_tiny_wd,
     "c2": c2_wide_deep,
     "c3": c3_two_tower,
     "c4": c4_hybrid,
     "c5": c5_ensemble,
+    "c6": c6_mtdnn,
 }
 
 # Small instances (oracle in seconds; several tiles + ragged tails) used by the parity tests.
@@ -354,6 +399,7 @@ SMALL = {
     "c4": dict(batch=3, image=40, seq=5, vocab=400, emb=64, gru_hidden=72, fields=3, rows=500,
                mlp_out=40),
     "c5": dict(batch=200, fields=4, rows=800, vocab=300, image=32, scale=0.125),
+    "c6": dict(batch=3, seq=40, layers=2, hidden=128, heads=2, ffn=256, vocab=500),
 }
 
 

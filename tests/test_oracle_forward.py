@@ -273,3 +273,75 @@ def test_ir_errors():
         parse("%a = input() : f16[1]\n")  # bad dtype
     g = parse("# c\n%x = input() : f32[2,3]\n%y = sigmoid(%x) : f32[2,3]\noutput %y\n")
     assert [n.op for n in g.nodes] == ["input", "sigmoid"] and g.outputs == [1]
+
+
+# ---- MT-DNN operators (Fig. 3) -----------------------------
+def test_gelu_identities_and_torch():
+    x = np.linspace(-6, 6, 97)
+    g = F.gelu(x)
+    np.testing.assert_allclose(g - F.gelu(-x), x, rtol=0, atol=1e-14)       # Phi(x) + Phi(-x) = 1
+    assert F.gelu(np.array([0.0]))[0] == 0.0
+    np.testing.assert_allclose(F.gelu(np.array([1.0])), [0.8413447460685429], rtol=1e-15)  # Phi(1)
+    want = torch.nn.functional.gelu(torch.tensor(x, dtype=torch.float64)).numpy()
+    np.testing.assert_allclose(g, want, rtol=1e-14, atol=1e-15)
+
+
+def test_layernorm_vs_torch_and_invariants():
+    rng = np.random.default_rng(4)
+    x = rng.normal(size=(7, 33)) * 3 + 1
+    g, b = rng.uniform(0.5, 1.5, 33), rng.normal(size=33)
+    want = torch.nn.functional.layer_norm(torch.tensor(x), (33,), torch.tensor(g), torch.tensor(b), eps=1e-12)
+    np.testing.assert_allclose(F.layernorm(x, g, b), want.numpy(), rtol=1e-12, atol=1e-12)
+    y = F.layernorm(x, np.ones(33), np.zeros(33))
+    np.testing.assert_allclose(y.mean(axis=1), 0, atol=1e-12)
+    np.testing.assert_allclose(y.var(axis=1), 1, rtol=1e-10)
+
+
+def test_attention_vs_torch_sdpa():
+    rng = np.random.default_rng(5)
+    B, S, heads, dh = 2, 9, 3, 8
+    H = heads * dh
+    qkv = rng.normal(size=(B * S, 3 * H))
+    got = F.attention(qkv, heads, S)
+    t = torch.tensor(qkv).reshape(B, S, 3, heads, dh).permute(2, 0, 3, 1, 4)   # [3, B, heads, S, dh]
+    want = torch.nn.functional.scaled_dot_product_attention(t[0], t[1], t[2])   # no mask, 1/sqrt(dh)
+    np.testing.assert_allclose(got, want.permute(0, 2, 1, 3).reshape(B * S, H).numpy(), rtol=1e-12, atol=1e-13)
+    # a single key: attention returns its value row for every query
+    one = F.attention(rng.normal(size=(4, 3 * H)), heads, 1)
+    assert one.shape == (4, H)
+
+
+def test_mtdnn_layer_vs_torch_encoder_layer():
+    """c6's embedding + first encoder layer through the oracle == torch nn.Embedding / layer_norm +
+    nn.TransformerEncoderLayer (post-LN, GELU, eps 1e-12) in float64 with the same weights."""
+    from paper_conf_ipps_zhanghl21_b200 import workloads as W
+    wl = W.build("c6", small=True, dt="f32")
+    prm = {k: s.materialize().numpy() for k, s in wl.params.items()}
+    ins = {k: s.materialize().numpy() for k, s in wl.inputs.items()}
+    vals = F.run(wl.ir, prm, ins, keep_all=True)
+    T = lambda n: torch.tensor(prm[n], dtype=torch.float64)
+    tok, seg = torch.tensor(ins["tok"]).long(), torch.tensor(ins["seg"]).long()
+    B, S = tok.shape
+    H = prm["tok_E"].shape[1]
+    e = torch.nn.functional.embedding(tok, T("tok_E")) + T("pos_E")[:S] + torch.nn.functional.embedding(seg, T("seg_E"))
+    e = torch.nn.functional.layer_norm(e, (H,), T("emb_g"), T("emb_b"), eps=1e-12)
+    np.testing.assert_allclose(vals["emb"], e.reshape(B * S, H).numpy(), rtol=1e-11, atol=1e-11)
+    layer = torch.nn.TransformerEncoderLayer(H, 2, prm["L0_ff1_W"].shape[0], dropout=0.0, activation="gelu",
+                                             layer_norm_eps=1e-12, batch_first=True, norm_first=False).double()
+    with torch.no_grad():
+        layer.self_attn.in_proj_weight.copy_(T("L0_qkv_W"))
+        layer.self_attn.in_proj_bias.copy_(T("L0_qkv_b"))
+        layer.self_attn.out_proj.weight.copy_(T("L0_o_W"))
+        layer.self_attn.out_proj.bias.copy_(T("L0_o_b"))
+        layer.linear1.weight.copy_(T("L0_ff1_W"))
+        layer.linear1.bias.copy_(T("L0_ff1_b"))
+        layer.linear2.weight.copy_(T("L0_ff2_W"))
+        layer.linear2.bias.copy_(T("L0_ff2_b"))
+        for ln in ("ln1", "ln2"):
+            getattr(layer, "norm" + ln[-1]).weight.copy_(T(f"L0_{ln}_g"))
+            getattr(layer, "norm" + ln[-1]).bias.copy_(T(f"L0_{ln}_b"))
+        layer.eval()
+        want = layer(e)
+    np.testing.assert_allclose(vals["L0_ln2"], want.reshape(B * S, H).numpy(), rtol=1e-10, atol=1e-10)
+    # [CLS] rows feed the task heads
+    np.testing.assert_allclose(vals["cls"], vals["L1_ln2"][::S])

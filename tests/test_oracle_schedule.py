@@ -78,6 +78,7 @@ def test_placeholders_and_independent_towers():
     ("c3", 3, 5, [MULTI, SEQ]),
     ("c4", 4, None, [MULTI, SEQ]),
     ("c5", 9, None, [MULTI, SEQ]),
+    ("c6", 5, None, [SEQ, MULTI]),
 ])
 def test_config_partitions(cfg, coarse, op, kinds):
     wl = W.build(cfg, small=True)
