@@ -41,7 +41,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=300)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="duet", choices=["duet", "reference"])
-    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5"])
+    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5", "c6"],
+                    help="c1-c5 = BASELINE.json configs[0..4]; c6 = MT-DNN (SURVEY.md §8(f) N4(b), not a BASELINE config)")
     ap.add_argument("--slots", type=int, default=2, help="CUDA-stream slots on the GPU")
     ap.add_argument("--dtype", default=None, choices=[None, "bf16", "f32"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -434,7 +435,7 @@ def main():
         "vs_baseline": None,
         "dtype": wl.params[next(iter(wl.params))].dtype if args.dtype is None else args.dtype,
         "data": "synthetic (seeded counter-based generator; random-init weights)",
-        "config": {"workload": wl.name, "baseline_config": {"c1": 0, "c2": 1, "c3": 2, "c4": 3, "c5": 4}[args.config],
+        "config": {"workload": wl.name, "baseline_config": {"c1": 0, "c2": 1, "c3": 2, "c4": 3, "c5": 4}.get(args.config),
                    "global_batch": wl.batch * world, "per_gpu_batch": wl.batch, "slots": args.slots,
                    "parallelism": f"dp{world} (independent batches per rank) x {args.slots} stream slots",
                    "l2": "flushed (512 MB write) before every timed step"},

@@ -21,7 +21,7 @@ namespace duet {
   } while (0)
 
 enum { EPI_BIAS_ACT = 0, EPI_LSTM = 1, EPI_GRU = 2 };
-enum Act { ACT_NONE = 0, ACT_RELU = 1, ACT_SIGMOID = 2, ACT_TANH = 3 };
+enum Act { ACT_NONE = 0, ACT_RELU = 1, ACT_SIGMOID = 2, ACT_TANH = 3, ACT_GELU = 4 };
 
 struct TcEpilogue {
   // EPI_BIAS_ACT
@@ -134,6 +134,21 @@ void mlp_small(const void* X, int bf16, const void* const* Ws, const float* cons
 // RNN step, SIMT (f32 parity path): gates from h_prev W_hh^T + gx (original PyTorch layout).
 void rnn_step_simt(int kind, const float* gx, const void* Whh, int w_bf16, const float* bhh_n, const void* h_prev,
                    void* h_next, int h_bf16, float* c_state, int M, int H, cudaStream_t st);
+
+// ---- MT-DNN encoder (transformer.cu) ----
+// y[b*S + s] = LN(Etok[tok[b,s]] + Epos[s] + Eseg[seg[b,s]]) * g + beta, H <= 1024 (eps 1e-12)
+void bert_embed(const int32_t* tok, const int32_t* seg, const void* Etok, const void* Epos, const void* Eseg,
+                const float* g, const float* beta, void* y, int bf16, int B, int S, int H, int64_t V, cudaStream_t st);
+// y = LN(a + b) * g + beta over rows of H <= 1024
+void add_layernorm(const void* a, const void* b, const float* g, const float* beta, void* y, int bf16, int64_t rows,
+                   int H, cudaStream_t st);
+// qkv [B*S, 3H] (Q | K | V, head h = columns h*dh..) -> out [B*S, H], softmax(Q K^T / sqrt dh) V per
+// (b, head); S <= 512, dh in {32, 64, 128}, K^T and V (fp32) within 227 KB of shared memory
+bool attention_ok(int S, int dh);
+void attention(const void* qkv, void* out, int bf16, int B, int S, int heads, int dh, cudaStream_t st);
+// y[i] = x[offset + i * stride] (rows of `cols` elements of `esize` bytes)
+void select_rows(const void* x, void* y, int esize, int64_t rows, int64_t cols, int64_t stride, int64_t offset,
+                 cudaStream_t st);
 
 // ---- gathers (gather.cu) ----
 void hash_mod(const int64_t* raw, int32_t* ids, int64_t n, int64_t V, cudaStream_t st);

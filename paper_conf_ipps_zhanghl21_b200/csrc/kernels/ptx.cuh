@@ -282,6 +282,7 @@ __device__ __forceinline__ float apply_act(float x, int act) {
     case ACT_RELU: return fmaxf(x, 0.0f);
     case ACT_SIGMOID: return sigmoidf_acc(x);
     case ACT_TANH: return tanhf(x);
+    case ACT_GELU: return 0.5f * x * (1.0f + erff(x * 0.70710678118654752f));
     default: return x;
   }
 }
@@ -307,6 +308,12 @@ __device__ __forceinline__ void bias_act(float* v, const float* b, int act) {
   } else if (act == ACT_TANH) {
 #pragma unroll
     for (int i = 0; i < N; ++i) v[i] = tanh_fast(v[i] + b[i]);
+  } else if (act == ACT_GELU) {  // exact erf form (MT-DNN's BERT encoder)
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+      const float x = v[i] + b[i];
+      v[i] = 0.5f * x * (1.0f + erff(x * 0.70710678118654752f));
+    }
   } else {
 #pragma unroll
     for (int i = 0; i < N; ++i) v[i] += b[i];

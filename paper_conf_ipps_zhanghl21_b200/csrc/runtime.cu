@@ -86,6 +86,7 @@ int act_code(const std::string& a) {
   if (a == "relu") return ACT_RELU;
   if (a == "sigmoid") return ACT_SIGMOID;
   if (a == "tanh") return ACT_TANH;
+  if (a == "gelu") return ACT_GELU;
   fail(DUET_EPARSE, "unknown activation '" + a + "'");
 }
 
@@ -545,6 +546,70 @@ void build_op(Program& P, const Node& n, Op& op) {
     const int a = n.arg_nodes[0], bf = n.dtype == kBF16;
     const int64_t cnt = n.numel();
     op.launch = [=](const Ptrs& T, cudaStream_t st) { sigmoid_ew(T[a], T[me], bf, cnt, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "bert_embed") {
+    // MT-DNN lexicon encoder: [B*S, H] = LN(E_tok[tok] + E_pos[s] + E_seg[seg])
+    nargs(2, 5);
+    need_dtype(n, argn(0).dtype, kI32, "tokens");
+    need_dtype(n, argn(1).dtype, kI32, "segments");
+    const auto& et = pdecl(0);
+    const auto& ep_ = pdecl(1);
+    const auto& es = pdecl(2);
+    need_dtype(n, n.dtype, et.dtype, "output");
+    need_dtype(n, ep_.dtype, et.dtype, "position table");
+    need_dtype(n, es.dtype, et.dtype, "segment table");
+    if (argn(0).shape.size() != 2 || argn(1).shape != argn(0).shape) fail(DUET_ESHAPE, "%" + n.name + ": tokens [B, S]");
+    const int B = (int)argn(0).shape[0], S = (int)argn(0).shape[1], H = (int)et.shape[1];
+    if (et.shape.size() != 2 || ep_.shape.size() != 2 || es.shape.size() != 2 || ep_.shape[0] < S ||
+        ep_.shape[1] != H || es.shape[1] != H || pdecl(3).numel() != H || pdecl(4).numel() != H ||
+        n.shape != std::vector<int64_t>{(int64_t)B * S, H})
+      fail(DUET_ESHAPE, "%" + n.name + ": bert_embed shapes");
+    const int a0 = n.arg_nodes[0], a1 = n.arg_nodes[1], bf = n.dtype == kBF16;
+    const void *Et = P.param(n.params[0]), *Ep = P.param(n.params[1]), *Es = P.param(n.params[2]);
+    const float* gm = (const float*)P.param(n.params[3]);
+    const float* bt = (const float*)P.param(n.params[4]);
+    const int64_t V = et.shape[0];
+    op.launch = [=](const Ptrs& T, cudaStream_t st) {
+      bert_embed((const int32_t*)T[a0], (const int32_t*)T[a1], Et, Ep, Es, gm, bt, T[me], bf, B, S, H, V, st);
+    };
+    op.n_kernels = 1;
+  } else if (n.op == "attention") {
+    nargs(1, 0);
+    const Node& x = argn(0);
+    need_dtype(n, x.dtype, n.dtype, "qkv");
+    const int heads = (int)n.attr_int("heads", 0), S = (int)n.attr_int("seq", 0);
+    if (x.shape.size() != 2 || heads <= 0 || S <= 0 || x.shape[0] % S || x.shape[1] % (3 * heads) ||
+        n.shape != std::vector<int64_t>{x.shape[0], x.shape[1] / 3})
+      fail(DUET_ESHAPE, "%" + n.name + ": attention needs qkv [B*S, 3H] and output [B*S, H]");
+    const int B = (int)(x.shape[0] / S), dh = (int)(x.shape[1] / 3 / heads);
+    if (!attention_ok(S, dh)) fail(DUET_EUNSUPPORTED, "%" + n.name + ": attention needs S <= 512, dh in {32, 64, 128}, K and V in shared memory");
+    const int a = n.arg_nodes[0], bf = n.dtype == kBF16;
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { attention(T[a], T[me], bf, B, S, heads, dh, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "add_layernorm") {
+    nargs(2, 2);
+    need_dtype(n, argn(0).dtype, n.dtype, "a");
+    need_dtype(n, argn(1).dtype, n.dtype, "b");
+    if (argn(0).shape != n.shape || argn(1).shape != n.shape || n.shape.size() != 2 ||
+        pdecl(0).numel() != n.shape[1] || pdecl(1).numel() != n.shape[1])
+      fail(DUET_ESHAPE, "%" + n.name + ": add_layernorm shapes");
+    const int a = n.arg_nodes[0], b = n.arg_nodes[1], bf = n.dtype == kBF16, H = (int)n.shape[1];
+    const int64_t rows = n.shape[0];
+    const float* gm = (const float*)P.param(n.params[0]);
+    const float* bt = (const float*)P.param(n.params[1]);
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { add_layernorm(T[a], T[b], gm, bt, T[me], bf, rows, H, st); };
+    op.n_kernels = 1;
+  } else if (n.op == "select_rows") {
+    nargs(1, 0);
+    const Node& x = argn(0);
+    need_dtype(n, x.dtype, n.dtype, "input");
+    const int64_t stride = n.attr_int("stride", 1), offset = n.attr_int("offset", 0);
+    if (x.shape.size() != 2 || n.shape.size() != 2 || n.shape[1] != x.shape[1] || stride < 1 || offset < 0 ||
+        offset + (n.shape[0] - 1) * stride >= x.shape[0])
+      fail(DUET_ESHAPE, "%" + n.name + ": select_rows shapes");
+    const int a = n.arg_nodes[0], es = dtype_bytes(n.dtype);
+    const int64_t rows = n.shape[0], cols = n.shape[1];
+    op.launch = [=](const Ptrs& T, cudaStream_t st) { select_rows(T[a], T[me], es, rows, cols, stride, offset, st); };
     op.n_kernels = 1;
   } else if (n.op == "maxpool") {
     nargs(1, 0);

@@ -140,7 +140,7 @@ def _oracle_outputs(wl, params, inputs):
 
 
 CASES = [("c1", "f32"), ("c1", "bf16"), ("c2", "bf16"), ("c2", "f32"), ("c3", "bf16"), ("c3", "f32"),
-         ("c4", "bf16"), ("c4", "f32"), ("c5", "bf16")]
+         ("c4", "bf16"), ("c4", "f32"), ("c5", "bf16"), ("c6", "bf16"), ("c6", "f32")]
 
 
 @pytest.mark.parametrize("cfg,dt", CASES)
@@ -164,7 +164,7 @@ def test_config_small_parity(cfg, dt):
         np.testing.assert_array_equal(a, b)
 
 
-@pytest.mark.parametrize("cfg", ["c1", "c2", "c3", "c4", "c5"])
+@pytest.mark.parametrize("cfg", ["c1", "c2", "c3", "c4", "c5", "c6"])
 def test_host_buffers_e2e_equal_device(cfg):
     """Pinned HOST inputs/outputs through duet_run (zero-copy reads/stores where eligible, memcpy
     nodes elsewhere; branch outputs exercise both) give the same bytes as device tensors."""
@@ -371,6 +371,57 @@ def test_model_variation_full_size_sampled(layers, resnet, ffn):
     for (name, _, _), y in zip(wl.outputs, outs):
         err = rel_err(y.float().cpu().numpy()[rows], want[name])
         print(f"[parity] full c4 L{layers} R{resnet} F{ffn} {name}: rel err {err:.3e}")
+        assert err <= TOL["bf16"], (name, err)
+
+
+@pytest.mark.parametrize("B,S,heads,dh,dt", [(2, 40, 2, 64, "bf16"), (1, 128, 12, 64, "bf16"), (3, 77, 3, 32, "f32"),
+                                              (2, 300, 2, 64, "bf16"), (1, 5, 4, 32, "f32"),
+                                              (2, 128, 2, 128, "bf16"), (1, 512, 1, 32, "f32")])
+def test_attention_node(B, S, heads, dh, dt):
+    """MT-DNN self-attention against the float64 oracle."""
+    H = heads * dh
+    ir = _single_node_graph(f"%y = attention(%x) {{heads={heads}, seq={S}}} : {dt}[{B * S},{H}]", {},
+                            {"x": (dt, (B * S, 3 * H))})
+    x = _rand((B * S, 3 * H), dt, 1.5, 31)
+    g = duet.Graph(ir)
+    y = torch.empty((B * S, H), dtype=torch.bfloat16 if dt == "bf16" else torch.float32, device="cuda")
+    g.node_run("y", [x.cuda()], y)
+    torch.cuda.synchronize()
+    want = OF.attention(OF.to_f64(to_np(x), dt), heads, S)
+    err = rel_err(y.float().cpu().numpy(), want)
+    print(f"[parity] attention B{B} S{S} h{heads} dh{dh} {dt}: rel err {err:.3e}")
+    assert err <= TOL[dt], err
+
+
+@pytest.mark.parametrize("rows,H,dt", [(120, 128, "bf16"), (128, 768, "bf16"), (33, 1000, "f32"), (7, 40, "f32")])
+def test_add_layernorm_node(rows, H, dt):
+    ir = _single_node_graph(f"%y = add_layernorm(%a, %b, @g, @be) : {dt}[{rows},{H}]",
+                            {"g": ("f32", (H,)), "be": ("f32", (H,))}, {"a": (dt, (rows, H)), "b": (dt, (rows, H))})
+    a, b = _rand((rows, H), dt, 2.0, 41), _rand((rows, H), dt, 1.0, 42)
+    gm, be = _rand((H,), "f32", 0.5, 43) + 1.0, _rand((H,), "f32", 0.2, 44)
+    g = duet.Graph(ir)
+    g.bind_all({"g": gm.cuda(), "be": be.cuda()})
+    y = torch.empty((rows, H), dtype=torch.bfloat16 if dt == "bf16" else torch.float32, device="cuda")
+    g.node_run("y", [a.cuda(), b.cuda()], y)
+    torch.cuda.synchronize()
+    f = lambda t, d: OF.to_f64(to_np(t), d)
+    want = OF.add_layernorm(f(a, dt), f(b, dt), f(gm, "f32"), f(be, "f32"))
+    assert rel_err(y.float().cpu().numpy(), want) <= TOL[dt]
+
+
+def test_c6_full_size():
+    """MT-DNN at its full (proposed) model size (BERT-base encoder + 4 task heads) in the bench's
+    launch configuration: every task output and the [CLS] vector against the float64 oracle."""
+    wl = W.build("c6", branch_outputs=True, batch=4)  # batch 4: 1-element task outputs make R-25 degenerate
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    want = _oracle_outputs(wl, sess.params, dict(zip(wl.inputs, inputs)))
+    outs = sess.outputs()
+    sess.run(sess.schedule(), inputs, outs)
+    torch.cuda.synchronize()
+    for (name, _, _), y in zip(wl.outputs, outs):
+        err = rel_err(y.float().cpu().numpy(), want[name])
+        print(f"[parity] full c6 {name}: rel err {err:.3e}")
         assert err <= TOL["bf16"], (name, err)
 
 
