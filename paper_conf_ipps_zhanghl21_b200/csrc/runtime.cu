@@ -344,7 +344,8 @@ void build_op(Program& P, const Node& n, Op& op) {
         // path is the multi-tile one), else 128 x 128
         const int t256 = mt * ((H + 63) / 64);
         rp_bn = (rp_bn_env == 256 || !rp_bn_env) ? (t256 > sms ? 256 : 128) : rp_bn_env;
-        rp_grid = sms;
+        static const int grid_env = getenv("DUET_RNN_GRID") ? atoi(getenv("DUET_RNN_GRID")) : 0;  // experiments
+        rp_grid = grid_env > 0 && grid_env <= sms ? grid_env : sms;
       }
     }
     if (rp_bn) {

@@ -17,3 +17,5 @@ full fc1 "gemm2_kernel" 2 python tools/gemm_micro_one.py 2048 1024 1664
 full gather "gather_rows16" 2 python tools/gemm_micro_one.py gather
 full lstm "rnn_persist" 1 python tools/rnn_trace_plain.py lstm 256 512 256 64
 full gru "rnn_persist" 1 python tools/rnn_trace_plain.py gru 64 1024 256 64
+# 3) r1c additions: c5-size LSTM (several 128x256 tiles per CTA) and the MT-DNN attention
+full lstmB4096 "rnn_persist" 1 python tools/rnn_trace_plain.py lstm 4096 512 256 8
