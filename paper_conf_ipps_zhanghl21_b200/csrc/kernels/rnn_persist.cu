@@ -226,7 +226,10 @@ __global__ void __launch_bounds__(kRThreads, 1)
             // barrier), then order the generic-proxy writes it observed before this thread's
             // async-proxy (TMA) reads
             if (lane == 0) {
-              const unsigned target = (unsigned)t * (unsigned)n_tiles * kREpiWarps;
+              // releases per tile and step: one per epilogue warp (one tile per CTA), one per tile
+              // (several tiles per CTA: thousands of same-address releases per step serialised at
+              // the L2 -- measured ~6-10 ns each, the whole step time at B = 4096)
+              const unsigned target = (unsigned)t * (unsigned)n_tiles * (MULTI ? 1u : (unsigned)kREpiWarps);
               while (ld_acquire_gpu(a.counter) < target) {
               }
               fence_proxy_async_global();
@@ -382,6 +385,31 @@ __global__ void __launch_bounds__(kRThreads, 1)
           const int buf = u & 1;
           const int row = tile_m0(i) + q * 32 + lane;
           const int n0 = tile_n0(i);
+          // the recurrent state of this thread's cells (written by this thread a step ago) is
+          // fetched before the accumulator wait, off the epilogue's critical path
+          float stp[UH / 8][8];
+          {
+            const __nv_bfloat16* hprev = a.hbuf[(t - 1) & 1];
+#pragma unroll
+            for (int c = 0; c < UH / 8; ++c) {
+              const int unit = (n0 / BN) * U + half * UH + 8 * c;
+              if (t == 0 || row >= a.B || unit >= H) {
+#pragma unroll
+                for (int e = 0; e < 8; ++e) stp[c][e] = 0.0f;
+              } else if constexpr (KIND == EPI_LSTM) {
+                const size_t off = (size_t)row * H + unit;
+                const float4 c0 = *reinterpret_cast<const float4*>(a.c_state + off);
+                const float4 c1 = *reinterpret_cast<const float4*>(a.c_state + off + 4);
+                stp[c][0] = c0.x, stp[c][1] = c0.y, stp[c][2] = c0.z, stp[c][3] = c0.w;
+                stp[c][4] = c1.x, stp[c][5] = c1.y, stp[c][6] = c1.z, stp[c][7] = c1.w;
+              } else {
+                const uint4 raw = *reinterpret_cast<const uint4*>(hprev + hs_index(row, unit, a.Bp));
+                const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&raw);
+#pragma unroll
+                for (int e = 0; e < 8; ++e) stp[c][e] = __bfloat162float(hv[e]);
+              }
+            }
+          }
           wait_sleep(&tfull[buf], (u >> 1) & 1);
           ptx::tc_fence_after();
           const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
@@ -403,7 +431,6 @@ __global__ void __launch_bounds__(kRThreads, 1)
             for (int c = 0; c < UH / 8; ++c) load_chunk(c);
             release();
           }
-          const __nv_bfloat16* hprev = a.hbuf[(t - 1) & 1];
 #pragma unroll
           for (int c = 0; c < UH / 8; ++c) {
             if constexpr (CH == 1) {
@@ -413,28 +440,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
             const int unit = (n0 / BN) * U + half * UH + 8 * c;
             if (row >= a.B || unit >= H) continue;
             const size_t off = (size_t)row * H + unit;
-            float st[8];
-            if constexpr (KIND == EPI_LSTM) {
-              if (t == 0) {
-#pragma unroll
-                for (int e = 0; e < 8; ++e) st[e] = 0.0f;
-              } else {
-                const float4 c0 = *reinterpret_cast<const float4*>(a.c_state + off);
-                const float4 c1 = *reinterpret_cast<const float4*>(a.c_state + off + 4);
-                st[0] = c0.x, st[1] = c0.y, st[2] = c0.z, st[3] = c0.w;
-                st[4] = c1.x, st[5] = c1.y, st[6] = c1.z, st[7] = c1.w;
-              }
-            } else {
-              if (t == 0) {
-#pragma unroll
-                for (int e = 0; e < 8; ++e) st[e] = 0.0f;
-              } else {
-                const uint4 raw = *reinterpret_cast<const uint4*>(hprev + hs_index(row, unit, a.Bp));
-                const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&raw);
-#pragma unroll
-                for (int e = 0; e < 8; ++e) st[e] = __bfloat162float(hv[e]);
-              }
-            }
+            float* st = stp[c];
             const int cb = n0 + half * UH + 8 * c;  // packed bias column of gate block 0
             float h[8];
 #pragma unroll
@@ -451,9 +457,13 @@ __global__ void __launch_bounds__(kRThreads, 1)
             else store_bf16x8(a.hbuf[t & 1] + hs_index(row, unit, a.Bp), h);
           }
           if (t < S - 1) {
+            // the tile's 8 epilogue warps meet at a named barrier; one thread releases the tile
             fence_proxy_async_global();
-            __syncwarp();
-            if (lane == 0) red_release_gpu_add(a.counter, 1u);
+            asm volatile("bar.sync 1, %0;" ::"n"(32 * kREpiWarps) : "memory");
+            if (threadIdx.x == 64) {
+              __threadfence();
+              red_release_gpu_add(a.counter, 1u);
+            }
           }
         }
       }
