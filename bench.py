@@ -151,6 +151,59 @@ def time_node(torch, graph, node, args, out, stream, iters=50, replays=20):
     return e0.elapsed_time(e1) / (iters * replays)  # ms
 
 
+def secondary_rooflines(torch, sess, wl, inputs, cfg, stream, dev, hbm_peak, bf16_peak):
+    """c2's other kernels against their own roofline: the hash, the two gathers
+    (HBM bytes: ids + rows + output) and fc2 / fc3 (tensor), each timed like the dominant kernel
+    (CUDA graph of back-to-back launches, events on `stream`); plus the deep gather at the
+    capability size B = 65536 (c2's 13.6 MB gather is too small to saturate HBM)."""
+    if cfg != "c2":
+        return None
+    from paper_conf_ipps_zhanghl21_b200 import duet
+    g = sess.graph
+    B, F, D = wl.batch, 26, 64
+    raw = inputs[0]
+    ids = torch.empty(B, F, dtype=torch.int32, device=dev)
+    g.node_run("ids", [raw], ids, stream)
+    out = {}
+
+    def hbm(name, node, args, y, nbytes, what):
+        ms = time_node(torch, g, node, args, y, stream)
+        gbs = nbytes / (ms / 1e3) / 1e9
+        out[name] = {"bound": "hbm", "kernel": what, "achieved": round(gbs, 1), "peak": hbm_peak, "unit": "GB/s",
+                     "frac": round(gbs / hbm_peak, 4), "bytes_per_launch": nbytes, "ms_per_launch": round(ms, 5)}
+
+    def tensor(name, node, M, N, K, what):
+        x = torch.randn(M, K, device=dev).to(torch.bfloat16)
+        y = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
+        ms = time_node(torch, g, node, [x], y, stream)
+        tf = 2 * M * N * K / (ms / 1e3) / 1e12
+        out[name] = {"bound": "tensor", "kernel": what, "achieved": round(tf, 1), "peak": bf16_peak,
+                     "unit": "TFLOP/s", "frac": round(tf / bf16_peak, 4), "ms_per_launch": round(ms, 5)}
+
+    hbm("hash", "ids", [raw], ids, B * F * (8 + 4), "hash_mod_kernel: int64 raw -> int32 ids")
+    X = torch.empty(B, F * D, dtype=torch.bfloat16, device=dev)
+    hbm("deep_gather", "deep_x", [ids], X, B * F * (4 + 2 * D * 2), "gather_rows16p2_kernel (B=2048; repeated launches: rows L2-warm)")
+    w = torch.empty(B, 1, dtype=torch.float32, device=dev)
+    hbm("wide_gather", "wide", [ids], w, B * F * (4 + 2) + 4 * B, "gather_sum_kernel (algorithmic; 32-B sectors)")
+    tensor("fc2", "fc2", B, 512, 1024, "gemm2_kernel 2048x512x1024")
+    tensor("fc3", "fc3", B, 256, 512, "gemm2_kernel 2048x256x512")
+    # capability size: the same table and kernel, 65536 rows
+    Bc = 65536
+    ir = (f"param @E : bf16[{F},1000000,{D}]\n%ids = input() : i32[{Bc},{F}]\n"
+          f"%x = gather_concat(%ids, @E) : bf16[{Bc},{F * D}]\noutput %x\n")
+    gc = duet.Graph(ir)
+    gc.bind_all({"E": sess.params["deep_E"]})
+    idc = torch.randint(0, 1000000, (Bc, F), dtype=torch.int32, device=dev)
+    Xc = torch.empty(Bc, F * D, dtype=torch.bfloat16, device=dev)
+    ms = time_node(torch, gc, "x", [idc], Xc, stream, iters=10, replays=10)
+    nb = Bc * F * (4 + 2 * D * 2)
+    gbs = nb / (ms / 1e3) / 1e9
+    out["deep_gather_B65536"] = {"bound": "hbm", "kernel": "gather_rows16p2_kernel at the capability size",
+                                 "achieved": round(gbs, 1), "peak": hbm_peak, "unit": "GB/s",
+                                 "frac": round(gbs / hbm_peak, 4), "bytes_per_launch": nb, "ms_per_launch": round(ms, 5)}
+    return out
+
+
 def load_traffic(node):
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
@@ -409,6 +462,8 @@ def main():
                     "peak_source": f"{peak_src} (MEASURED_PEAKS.json bf16_tflops, burst)",
                     "algorithmic_per_launch": work, "ms_per_launch": round(ms, 5)}
 
+    kernels = secondary_rooflines(torch, sess, wl, inputs, args.config, home, dev, hbm_peak, bf16_peak)
+
     cpu_baseline = None
     if world == 1 and not args.no_cpu_baseline:
         import numpy as np
@@ -456,6 +511,7 @@ def main():
         "gpu_launches": n_launch * args.steps,
         "gpu_launches_per_step": n_launch,
         "roofline": roof,
+        "kernels": kernels,
         "cpu_baseline": cpu_baseline,
         "clocks": clocks,
     }
