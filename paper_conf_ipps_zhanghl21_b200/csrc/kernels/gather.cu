@@ -31,24 +31,38 @@ __device__ __forceinline__ uint4 ld_stream16(const void* p) {
   return r;
 }
 
+// id = x mod V (floor modulo)
+__device__ __forceinline__ int32_t hash_id(int64_t x, int64_t V) {
+  int64_t r;
+  if ((uint64_t)x < (1ULL << 32) && V < (1LL << 32))
+    r = (int64_t)((uint32_t)x % (uint32_t)V);  // 32-bit path (the recipe's raw ids are < 2^31)
+  else {
+    r = x % V;
+    if (r < 0) r += V;
+  }
+  return (int32_t)r;
+}
+
+// Where a gather's ids come from: the hash node's int32 output, or (hash absorbed into its gathers,
+// runtime.cu plan_hash_fusion) the raw int64 features hashed on the fly.
+struct IdSrc {
+  const int32_t* ids;
+  const int64_t* raw;
+  int64_t V;
+  __device__ __forceinline__ int32_t operator()(int64_t i) const {
+    return raw ? hash_id(__ldg(raw + i), V) : __ldg(ids + i);
+  }
+};
+
 __global__ void hash_mod_kernel(const int64_t* __restrict__ raw, int32_t* __restrict__ ids, int64_t n, int64_t V) {
   ptx::pdl_wait();
   ptx::pdl_trigger();
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t x = raw[i];
-    int64_t r;
-    if ((uint64_t)x < (1ULL << 32) && V < (1LL << 32))
-      r = (int64_t)((uint32_t)x % (uint32_t)V);  // 32-bit path (the recipe's raw ids are < 2^31)
-    else {
-      r = x % V;
-      if (r < 0) r += V;
-    }
-    ids[i] = (int32_t)r;
-  }
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    ids[i] = hash_id(raw[i], V);
 }
 
 template <typename T>
-__global__ void gather_sum_kernel(const int32_t* __restrict__ ids, const T* __restrict__ tab,
+__global__ void gather_sum_kernel(const IdSrc ids, const T* __restrict__ tab,
                                   const float* __restrict__ b, float* __restrict__ y, int B, int F, int64_t R) {
   ptx::pdl_wait();
   ptx::pdl_trigger();
@@ -58,7 +72,7 @@ __global__ void gather_sum_kernel(const int32_t* __restrict__ ids, const T* __re
   if (row >= B) return;
   float acc = 0.0f;
   for (int f = lane; f < F; f += 32) {
-    int id = __ldg(ids + (size_t)row * F + f);
+    int id = ids((int64_t)row * F + f);
     acc += to_f(tab[(size_t)f * R + id]);
   }
   acc = warp_sum(acc);
@@ -67,7 +81,7 @@ __global__ void gather_sum_kernel(const int32_t* __restrict__ ids, const T* __re
 
 // out row r (of `rows`) <- table row src_row(r); vpr 16-byte vectors per row.
 template <int MODE>  // 0: gather_concat (row r = b*F + f), 1: embed_seq (row r = t*B + b)
-__global__ void gather_rows16_kernel(const int32_t* __restrict__ idx, const uint8_t* __restrict__ tab,
+__global__ void gather_rows16_kernel(const IdSrc idx, const uint8_t* __restrict__ tab,
                                      uint8_t* __restrict__ out, int64_t rows, int vpr, int64_t row_bytes, int F,
                                      int64_t R, int B, int S) {
   ptx::pdl_wait();
@@ -88,11 +102,11 @@ __global__ void gather_rows16_kernel(const int32_t* __restrict__ idx, const uint
         int64_t trow;
         if (MODE == 0) {
           int f = (int)(r % F);
-          trow = (int64_t)f * R + __ldg(idx + r);
+          trow = (int64_t)f * R + idx(r);
         } else {
           int64_t t = r / B;
           int64_t b = r - t * B;
-          trow = __ldg(idx + b * S + t);
+          trow = idx(b * S + t);
         }
         val[u] = ld_stream16(tab + trow * row_bytes + (int64_t)k * 16);
         dst[u] = r * row_bytes + (int64_t)k * 16;
@@ -108,7 +122,7 @@ __global__ void gather_rows16_kernel(const int32_t* __restrict__ idx, const uint
 // kernel's 64-bit divisions per vector dominated its issue time): VPR lanes per row, four rows in
 // flight per thread.
 template <int MODE, int VPR>
-__global__ void __launch_bounds__(256) gather_rows16p2_kernel(const int32_t* __restrict__ idx,
+__global__ void __launch_bounds__(256) gather_rows16p2_kernel(const IdSrc idx,
                                                               const uint8_t* __restrict__ tab,
                                                               uint8_t* __restrict__ out, int rows, int F,
                                                               int64_t R, int B, int S) {
@@ -125,10 +139,10 @@ __global__ void __launch_bounds__(256) gather_rows16p2_kernel(const int32_t* __r
       if (r < rows) {
         int64_t trow;
         if (MODE == 0) {
-          trow = (int64_t)(r % F) * R + __ldg(idx + r);
+          trow = (int64_t)(r % F) * R + idx(r);
         } else {
           const int t = r / B, b = r - t * B;
-          trow = __ldg(idx + (int64_t)b * S + t);
+          trow = idx((int64_t)b * S + t);
         }
         val[u] = ld_stream16(tab + trow * RB + k * 16);
       }
@@ -142,7 +156,7 @@ __global__ void __launch_bounds__(256) gather_rows16p2_kernel(const int32_t* __r
 }
 
 template <int MODE>
-__global__ void gather_rows_bytes_kernel(const int32_t* __restrict__ idx, const uint8_t* __restrict__ tab,
+__global__ void gather_rows_bytes_kernel(const IdSrc idx, const uint8_t* __restrict__ tab,
                                          uint8_t* __restrict__ out, int64_t rows, int64_t row_bytes, int F,
                                          int64_t R, int B, int S) {
   ptx::pdl_wait();
@@ -153,10 +167,10 @@ __global__ void gather_rows_bytes_kernel(const int32_t* __restrict__ idx, const 
     int64_t k = v - r * row_bytes;
     int64_t trow;
     if (MODE == 0) {
-      trow = (int64_t)(r % F) * R + idx[r];
+      trow = (int64_t)(r % F) * R + idx(r);
     } else {
       int64_t t = r / B, b = r - t * B;
-      trow = idx[b * S + t];
+      trow = idx(b * S + t);
     }
     out[v] = tab[trow * row_bytes + k];
   }
@@ -214,9 +228,10 @@ void hash_mod(const int64_t* raw, int32_t* ids, int64_t n, int64_t V, cudaStream
   CK(cudaGetLastError());
 }
 
-void gather_sum(const int32_t* ids, const void* T, int t_bf16, const float* b, float* y, int B, int F, int64_t R,
-                cudaStream_t st) {
+void gather_sum(const int32_t* ids_, const void* T, int t_bf16, const float* b, float* y, int B, int F, int64_t R,
+                cudaStream_t st, const int64_t* raw, int64_t V) {
   if (B == 0) return;
+  const IdSrc ids{ids_, raw, V};
   int blocks = (B + 7) / 8;
   if (t_bf16)
     launch_pdl(gather_sum_kernel<__nv_bfloat16>, dim3(blocks), dim3(256), 0, st, ids, (const __nv_bfloat16*)T, b, y, B, F, R);
@@ -225,7 +240,7 @@ void gather_sum(const int32_t* ids, const void* T, int t_bf16, const float* b, f
   CK(cudaGetLastError());
 }
 
-static void gather_rows(int mode, const int32_t* idx, const void* tab, int esize, void* out, int64_t rows, int D,
+static void gather_rows(int mode, const IdSrc idx, const void* tab, int esize, void* out, int64_t rows, int D,
                         int F, int64_t R, int B, int S, cudaStream_t st) {
   if (rows == 0) return;
   int64_t rb = (int64_t)D * esize;
@@ -258,13 +273,13 @@ static void gather_rows(int mode, const int32_t* idx, const void* tab, int esize
 }
 
 void gather_concat(const int32_t* ids, const void* E, int esize, void* X, int B, int F, int64_t R, int D,
-                   cudaStream_t st) {
-  gather_rows(0, ids, E, esize, X, (int64_t)B * F, D, F, R, B, 0, st);
+                   cudaStream_t st, const int64_t* raw, int64_t V) {
+  gather_rows(0, IdSrc{ids, raw, V}, E, esize, X, (int64_t)B * F, D, F, R, B, 0, st);
 }
 
 void embed_seq(const int32_t* tok, const void* E, int esize, void* X, int B, int S, int64_t V, int D,
                cudaStream_t st) {
-  gather_rows(1, tok, E, esize, X, (int64_t)B * S, D, 1, V, B, S, st);
+  gather_rows(1, IdSrc{tok, nullptr, 0}, E, esize, X, (int64_t)B * S, D, 1, V, B, S, st);
 }
 
 void fill_random(void* p, int dtype, int64_t n, int64_t high, uint64_t seed, cudaStream_t st) {

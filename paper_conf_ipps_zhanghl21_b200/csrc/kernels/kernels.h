@@ -152,10 +152,11 @@ void select_rows(const void* x, void* y, int esize, int64_t rows, int64_t cols, 
 
 // ---- gathers (gather.cu) ----
 void hash_mod(const int64_t* raw, int32_t* ids, int64_t n, int64_t V, cudaStream_t st);
+// raw != nullptr: the hash is absorbed (runtime.cu plan_hash_fusion) -- ids = raw mod V on the fly
 void gather_sum(const int32_t* ids, const void* T, int t_bf16, const float* b, float* y, int B, int F, int64_t R,
-                cudaStream_t st);
+                cudaStream_t st, const int64_t* raw = nullptr, int64_t V = 0);
 void gather_concat(const int32_t* ids, const void* E, int esize, void* X, int B, int F, int64_t R, int D,
-                   cudaStream_t st);
+                   cudaStream_t st, const int64_t* raw = nullptr, int64_t V = 0);
 void embed_seq(const int32_t* tok, const void* E, int esize, void* X, int B, int S, int64_t V, int D,
                cudaStream_t st);
 void fill_random(void* p, int dtype, int64_t n, int64_t high, uint64_t seed, cudaStream_t st);

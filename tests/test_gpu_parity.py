@@ -103,6 +103,32 @@ def test_gather_fused_linear_opt_in():
     assert r.returncode == 0 and r.stdout.count("ok") == 4, r.stdout + r.stderr
 
 
+_HASH_FUSED_SCRIPT = r'''
+import os, sys
+sys.path.insert(0, os.environ["REPO"])
+import torch
+from tests.test_gpu_parity import test_config_small_parity, test_host_buffers_e2e_equal_device
+for cfg, dt in [("c1", "f32"), ("c2", "bf16"), ("c5", "bf16")]:
+    test_config_small_parity(cfg, dt)
+    test_host_buffers_e2e_equal_device(cfg)
+    print("ok", cfg)
+'''
+
+
+def test_hash_absorbed_by_gathers_opt_in():
+    """The opt-in hash_mod -> gathers fusion (DUET_HASH_FUSE=1, runtime.cu plan_hash_fusion): config
+    parity against the oracle (both schedules bit-identical) and host-buffer runs, in a subprocess
+    because the switch is read once."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, DUET_HASH_FUSE="1", REPO=root)
+    r = subprocess.run([sys.executable, "-c", _HASH_FUSED_SCRIPT], env=env, capture_output=True, text=True,
+                       timeout=600, cwd=root)
+    assert r.returncode == 0 and r.stdout.count("ok") == 3, r.stdout[-3000:] + r.stderr[-3000:]
+
+
 def gather_fused_case(B, F, R, N, act):
     """gather_concat -> linear fused into one pair GEMM (tile::gather4 A producer, runtime.cu
     plan_gather_fusion) == the unfused node kernels bit for bit, and == the float64 oracle."""
