@@ -14,9 +14,13 @@ import torch.distributed as dist
 
 
 def env():
-    """(rank, world_size, local_rank) from the torchrun environment (defaults: single process)."""
-    return (int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")),
-            int(os.environ.get("LOCAL_RANK", "0")))
+    """(rank, world_size, local_rank) from the torchrun environment (defaults: single process).
+    DUET_FORCE_DEVICE=<i> (test only) puts every rank on GPU i, so the multi-rank flow can run on a
+    one-GPU box (with DUET_DIST_BACKEND=gloo: NCCL refuses two ranks on one GPU)."""
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("DUET_FORCE_DEVICE") is not None:
+        local = int(os.environ["DUET_FORCE_DEVICE"])
+    return (int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")), local)
 
 
 def init(backend: str | None = None, device: torch.device | None = None) -> bool:
@@ -25,6 +29,7 @@ def init(backend: str | None = None, device: torch.device | None = None) -> bool
     if world <= 1 or dist.is_initialized():
         return dist.is_initialized()
     os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    backend = os.environ.get("DUET_DIST_BACKEND", backend)  # test override (see env())
     if backend is None:
         backend = "nccl" if torch.cuda.is_available() else "gloo"
     kw = {"device_id": device} if (backend == "nccl" and device is not None) else {}

@@ -80,3 +80,25 @@ def test_single_process_noops():
     assert MR.max_over_ranks(3.5) == 3.5
     t = torch.arange(4)
     assert MR.gather_rows(t, 4) is t
+
+
+@pytest.mark.gpu
+def test_bench_two_ranks_on_one_gpu():
+    """bench.py under torchrun with 2 ranks (the driver's N>1 launch): barrier, max-over-ranks timing
+    and rank 0's single JSON line.  This box has one GPU, so both ranks sit on GPU 0 and the process
+    group is gloo (DUET_FORCE_DEVICE / DUET_DIST_BACKEND; NCCL refuses two ranks per GPU)."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, DUET_DIST_BACKEND="gloo", DUET_FORCE_DEVICE="0")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
+           "127.0.0.1", "--master-port", "29541", "bench.py", "--config", "c1", "--gpus", "2", "--steps", "5",
+           "--warmup", "3", "--no-cpu-baseline", "--profile-samples", "5"]
+    r = subprocess.run(cmd, env=env, cwd=root, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["config"]["global_batch"] == 2 and d["value"] > 0
