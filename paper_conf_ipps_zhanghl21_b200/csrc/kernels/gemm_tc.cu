@@ -59,7 +59,12 @@ __global__ void __launch_bounds__(192, 1)
   const int lane = threadIdx.x & 31;
   const int n0 = blockIdx.x * BN;
   const int m0 = blockIdx.y * BM;
-  const int nk = (K + BK - 1) / BK;
+  // split-K (EPI_BIAS_ACT with ep.splits > 1): CTA z accumulates k-blocks [kb0, kb1) and stores the
+  // raw fp32 partial tile to ep.ws[z]; gemm_splitk_reduce adds the splits in order (deterministic)
+  const int nk_all = (K + BK - 1) / BK;
+  const int per = ep.splits > 1 ? (nk_all + ep.splits - 1) / ep.splits : nk_all;
+  const int kb0 = ep.splits > 1 ? (int)blockIdx.z * per : 0;
+  const int nk = ep.splits > 1 ? min(nk_all, kb0 + per) - kb0 : nk_all;
 
   if (warp == 0 && lane == 0) {
     ptx::tma_prefetch(&tmA);
@@ -88,9 +93,10 @@ __global__ void __launch_bounds__(192, 1)
 
   if (warp == 0) {
     if (lane == 0) {
-      for (int kb = 0; kb < nk; ++kb) {
-        const int s = kb % Cfg::STAGES;
-        if (kb >= Cfg::STAGES) ptx::mbar_wait(&empty[s], ((kb / Cfg::STAGES) - 1) & 1);
+      for (int i = 0; i < nk; ++i) {
+        const int s = i % Cfg::STAGES;
+        const int kb = kb0 + i;
+        if (i >= Cfg::STAGES) ptx::mbar_wait(&empty[s], ((i / Cfg::STAGES) - 1) & 1);
         if (ep.dbg & 2) {
           ptx::mbar_arrive(&full[s]);
         } else {
@@ -108,7 +114,7 @@ __global__ void __launch_bounds__(192, 1)
     constexpr uint32_t idesc = ptx::idesc_bf16(BM, BN);
     const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
     const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
-    for (int kb = 0; kb < nk; ++kb) {
+    for (int kb = 0; kb < nk; ++kb) {  // kb counts this CTA's k-blocks (split-K: from kb0)
       const int s = kb % Cfg::STAGES;
       ptx::mbar_wait(&full[s], (kb / Cfg::STAGES) & 1);
       ptx::tc_fence_after();
@@ -143,6 +149,16 @@ __global__ void __launch_bounds__(192, 1)
     if constexpr (EPI == EPI_BIAS_ACT) {
       OutT* out = reinterpret_cast<OutT*>(ep.out) + (size_t)row * ep.ldo;
       const int act = ep.act;
+      if (ep.splits > 1) {  // raw fp32 partial -> ws[z][row][col]
+        float* wsr = ep.ws + ((size_t)blockIdx.z * M + row) * N;
+#pragma unroll 1
+        for (int c = 0; c < BN / 16; ++c) {
+          float v[16];
+          ptx::tmem_ld16(tq + c * 16, v);
+          const int col0 = n0 + c * 16;
+          if (row < M && col0 < N) store_row16_any(wsr + col0, v, N - col0);
+        }
+      } else
 #pragma unroll 1
       for (int c = 0; c < BN / 16; ++c) {
         float v[16];
@@ -244,6 +260,21 @@ __global__ void __launch_bounds__(192, 1)
   }
 }
 
+// out[m, n] = act(sum_z ws[z, m, n] + bias[n]), z in order (deterministic split-K)
+template <typename OutT>
+__global__ void gemm_splitk_reduce_kernel(const float* __restrict__ ws, const float* __restrict__ bias, OutT* out,
+                                          int M, int N, int ldo, int splits, int act) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
+  const int64_t total = (int64_t)M * N;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int m = (int)(e / N), n = (int)(e - (int64_t)m * N);
+    float v = 0.0f;
+    for (int z = 0; z < splits; ++z) v += __ldcg(ws + (size_t)z * total + e);
+    out[(size_t)m * ldo + n] = from_f<OutT>(apply_act(v + (bias ? bias[n] : 0.0f), act));
+  }
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   if (!fn) {
@@ -267,7 +298,7 @@ void launch_tc(const CUtensorMap& a, const CUtensorMap& w, const CUtensorMap& x,
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
     attr_done = true;
   }
-  dim3 grid((N + BN - 1) / BN, (M + BM - 1) / BM);
+  dim3 grid((N + BN - 1) / BN, (M + BM - 1) / BM, ep.splits > 1 ? ep.splits : 1);
   launch_pdl_if(pdl_on(true), kern, grid, dim3(192), Cfg::SMEM, st, a, w, x, ep, M, N, K);
 }
 
@@ -349,6 +380,30 @@ bool make_tmap_store_2d(CUtensorMap* m, void* base, int eb, int64_t rows, int64_
                             dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
                             CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS;
+}
+
+void gemm_splitk_reduce(const TcEpilogue& ep, int M, int N, int out_bf16, cudaStream_t st) {
+  const int64_t total = (int64_t)M * N;
+  const unsigned grid = (unsigned)std::min<int64_t>((total + 255) / 256, 1184);
+  if (out_bf16)
+    launch_pdl(gemm_splitk_reduce_kernel<__nv_bfloat16>, dim3(grid), dim3(256), 0, st, (const float*)ep.ws, ep.bias,
+               (__nv_bfloat16*)ep.out, M, N, ep.ldo, ep.splits, ep.act);
+  else
+    launch_pdl(gemm_splitk_reduce_kernel<float>, dim3(grid), dim3(256), 0, st, (const float*)ep.ws, ep.bias,
+               (float*)ep.out, M, N, ep.ldo, ep.splits, ep.act);
+}
+
+int tc_splitk(int M, int N, int K, int bn, int num_sms) {
+  static const bool off = getenv("DUET_SPLITK") && atoi(getenv("DUET_SPLITK")) == 0;
+  const int tiles = ((M + BM - 1) / BM) * ((N + bn - 1) / bn);
+  const int nk = (K + BK - 1) / BK;
+  // only long K pays for the extra reduce launch (~3 us): measured on MT-DNN at batch 1, FFN2
+  // (K = 3072, 48 k-blocks) 13.0 -> 8.4 us, but QKV / out / FFN1 (12 k-blocks) 4.9-5.5 -> 7.2-9.6 us
+  if (off || tiles * 2 > num_sms || nk < 32) return 1;
+  int splits = std::min(num_sms / tiles, nk / 2);
+  if (splits < 2) return 1;
+  const int per = (nk + splits - 1) / splits;
+  return (nk + per - 1) / per;  // every split non-empty
 }
 
 int tc_pick_bn(int M, int N, int num_sms) {

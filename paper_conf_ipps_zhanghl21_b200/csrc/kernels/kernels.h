@@ -40,6 +40,10 @@ struct TcEpilogue {
   int x_row0 = 0;              // row offset of x_t in the X map ([S*B, E] time-major)
   int tma_store = 0;  // EPI_BIAS_ACT: 1 = output tile leaves through TMA stores (map passed separately)
   int early_a = 0;  // pair GEMM: issue the first A stages right after the PDL wait (before TMEM alloc)
+  // single-CTA GEMM split-K (EPI_BIAS_ACT): grid.z = splits CTAs per tile store raw fp32 partials to
+  // ws [splits, M, N]; gemm_splitk_reduce then applies bias + activation
+  int splits = 1;
+  float* ws = nullptr;
   // pair GEMM with a gathered A operand (gather-concat fused into the GEMM, gemm2_gather): row b of
   // A is [E[0, ids[b,0]], ..., E[F-1, ids[b,F-1]]], E = [F, R, 64] bf16, K = 64 F
   const int32_t* g_ids = nullptr;  // [M, F]
@@ -48,6 +52,10 @@ struct TcEpilogue {
 };
 
 // ---- tcgen05 GEMM (gemm_tc.cu) ----
+// split-K for skinny GEMMs (one 128-row tile, few N tiles, long K: MT-DNN at batch 1): the split
+// count that fills the SMs with >= 2 k-blocks per split (1 = off; DUET_SPLITK=0 disables)
+int tc_splitk(int M, int N, int K, int bn, int num_sms);
+void gemm_splitk_reduce(const TcEpilogue& ep, int M, int N, int out_bf16, cudaStream_t st);
 CUtensorMap make_tmap_bf16_2d(const void* base, int64_t rows, int64_t cols, int box_rows);
 }  // namespace duet
 #include <cudaTypedefs.h>

@@ -252,7 +252,11 @@ void build_op(Program& P, const Node& n, Op& op) {
       const char* dbg_env = getenv("DUET_GEMM_DBG");
       const int dbg = dbg_env ? atoi(dbg_env) : 0;
       const char* bn_env = getenv("DUET_GEMM_BN");
-      const int bn = bn_env ? atoi(bn_env) : tc_pick_bn(M, N, sms);
+      int bn = bn_env ? atoi(bn_env) : tc_pick_bn(M, N, sms);
+      // skinny GEMM (MT-DNN at batch 1: M = 128, K up to 3072): 64-wide tiles split along K
+      int splits = tc_splitk(M, N, K, bn_env ? bn : 64, sms);
+      if (splits > 1 && !bn_env) bn = 64;
+      float* ws = splits > 1 ? (float*)P.alloc((int64_t)splits * M * N * 4) : nullptr;
       CUtensorMap tw = make_tmap_bf16_2d(W, N, K, bn);
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         CUtensorMap ta = make_tmap_bf16_2d(T[in], M, K, 128);
@@ -262,12 +266,16 @@ void build_op(Program& P, const Node& n, Op& op) {
         ep.ldo = N;
         ep.act = act;
         ep.dbg = dbg;
+        ep.splits = splits;
+        ep.ws = ws;
         gemm_tc_maps(ta, tw, M, N, K, bn, ep, EPI_BIAS_ACT, yb, st);
+        if (splits > 1) gemm_splitk_reduce(ep, M, N, yb, st);
       };
+      op.n_kernels = splits > 1 ? 2 : 1;
     } else {
       op.launch = [=](const Ptrs& T, cudaStream_t st) { gemm_simt(T[in], xb, W, wb, b, T[me], yb, M, N, K, act, st); };
     }
-    op.n_kernels = 1;
+    if (!op.n_kernels) op.n_kernels = 1;
   } else if (n.op == "mlp") {
     if (n.arg_nodes.size() != 1 || n.params.size() < 2 || n.params.size() % 2)
       fail(DUET_EPARSE, "%" + n.name + ": mlp(%x, @W0, @b0, ...)");

@@ -39,6 +39,9 @@ def _rand(shape, dt, scale=1.0, seed=0):
     (513, 272, 200, "bf16", "f32"),
     (300, 136, 320, "f32", "f32"),
     (5, 3, 7, "f32", "f32"),
+    (128, 768, 3072, "bf16", "bf16"),   # split-K (12 splits of 4 k-blocks) + reduce
+    (120, 136, 2500, "bf16", "f32"),    # split-K, ragged M / N / K
+    (3, 768, 768, "bf16", "bf16"),      # MT-DNN task pooler at batch 3
 ])
 def test_linear_node(M, N, K, dt, out):
     ir = _single_node_graph(f"%y = linear(%x, @W, @b) {{act=relu}} : {out}[{M},{N}]",
