@@ -118,7 +118,7 @@ __global__ void add_layernorm_kernel(const T* a, const T* b, const float* g, con
 }
 
 constexpr int kAttWarps = 8;
-constexpr int kAttQ = 16;      // query rows per CTA (2 per warp)
+constexpr int kAttQ = 8;       // query rows per CTA (1 per warp: B * heads * S warps in flight)
 constexpr int kAttMaxT = 16;   // S <= 32 * 16
 constexpr int kAttMaxDV = 4;   // dh <= 128
 
@@ -144,30 +144,44 @@ __global__ void __launch_bounds__(32 * kAttWarps) attention_kernel(const void* q
   ptx::pdl_wait();
   ptx::pdl_trigger();
   const int64_t base = (int64_t)b * S * ld + (int64_t)h * dh;
-  // K / V rows -> smem: each warp takes rows warp, warp + 8, ...; 4 rows' loads are issued before
-  // their stores so a warp keeps 4 * 2 * dv loads in flight (one latency per 4 rows)
-  for (int j0 = warp; j0 < Sp; j0 += 4 * kAttWarps) {
-    float kv[4][2][DV];
+  // K / V rows -> smem in 16-byte chunks (8 bf16 / 4 fp32 of one row): every thread issues up to 8
+  // independent chunk loads before converting and storing them (ncu: the scalar 2-byte loads of
+  // the first version left ~45% of the samples stalled on this phase)
+  {
+    const int esz = bf16 ? 2 : 4, epc = 16 / esz, cpr = dh / epc, per = Sp * cpr, nch = 2 * per;
+    const uint8_t* src = reinterpret_cast<const uint8_t*>(qkv);
+    for (int c0 = threadIdx.x; c0 < nch; c0 += 8 * blockDim.x) {
+      uint4 raw[8];
 #pragma unroll
-    for (int r = 0; r < 4; ++r) {
-      const int j = j0 + r * kAttWarps;
-#pragma unroll
-      for (int v = 0; v < DV; ++v) {
-        const bool in = j < S;
-        const int64_t e = base + (int64_t)j * ld + 32 * v + lane;
-        kv[r][0][v] = in ? ldv(qkv, e + H, bf16) : 0.0f;
-        kv[r][1][v] = in ? ldv(qkv, e + 2 * H, bf16) : 0.0f;
+      for (int u = 0; u < 8; ++u) {
+        const int c = c0 + u * blockDim.x;
+        raw[u] = make_uint4(0u, 0u, 0u, 0u);
+        if (c < nch) {
+          const int kvs = c / per, rem = c - kvs * per, j = rem / cpr, d0 = (rem - j * cpr) * epc;
+          if (j < S)
+            raw[u] = __ldg(reinterpret_cast<const uint4*>(src + (base + (int64_t)j * ld + (1 + kvs) * H + d0) * esz));
+        }
       }
-    }
 #pragma unroll
-    for (int r = 0; r < 4; ++r) {
-      const int j = j0 + r * kAttWarps;
-      if (j < Sp)
+      for (int u = 0; u < 8; ++u) {
+        const int c = c0 + u * blockDim.x;
+        if (c >= nch) break;
+        const int kvs = c / per, rem = c - kvs * per, j = rem / cpr, d0 = (rem - j * cpr) * epc;
+        float f[8];
+        if (bf16) {
+          const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&raw[u]);
 #pragma unroll
-        for (int v = 0; v < DV; ++v) {
-            Kt[(32 * v + lane) * ldk + j] = kv[r][0][v];
-            Vs[j * dh + 32 * v + lane] = kv[r][1][v];
-          }
+          for (int i = 0; i < 8; ++i) f[i] = __bfloat162float(hv[i]);
+        } else {
+          f[0] = __uint_as_float(raw[u].x), f[1] = __uint_as_float(raw[u].y);
+          f[2] = __uint_as_float(raw[u].z), f[3] = __uint_as_float(raw[u].w);
+        }
+        if (kvs == 0) {
+          for (int i = 0; i < epc; ++i) Kt[(d0 + i) * ldk + j] = f[i];
+        } else {
+          for (int i = 0; i < epc; ++i) Vs[j * dh + d0 + i] = f[i];
+        }
+      }
     }
   }
   __syncthreads();
