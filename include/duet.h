@@ -50,6 +50,8 @@
  *                                                  (PyTorch gate order i,f,g,o; h0=c0=0)
  *     gru(%x[S,B,E], @Wih[3H,E], @Whh[3H,H], @bih f32[3H], @bhh f32[3H])   h_S -> [B,H]
  *                                                  (PyTorch r,z,n; b_hn inside r*(.))
+ *     lstm / gru {seq=1}                           every h_t -> [S,B,H] (a lower layer of a stacked
+ *                                                  RNN, Fig. 14)
  *     conv2d_bn(%x[N,H,W,C], @W[Co,kh,kw,C], @gamma,@beta,@mean,@var f32[Co]) {stride,pad,act}
  *                                                  NHWC conv + inference BN (eps 1e-5) + act
  *     add(%a, %b) {act}   maxpool(%x) {k,stride,pad}   avgpool(%x[N,H,W,C]) -> [N,C]
@@ -58,9 +60,16 @@
  *     concat_head(%a1, ..., @w f32[sum K], @b f32[1]) {act}  act(concat(a).w + b) -> f32[B,1]
  *     sum_join(%l1, ...)  sigma(sum l_i)    mean_join(%l1, ...)  sigma(mean l_i)  -> f32[B,1]
  *     sigmoid(%x)
+ *   MT-DNN (Fig. 3; LayerNorm eps 1e-12):
+ *     bert_embed(%tok i32[B,S], %seg i32[B,S], @Etok[V,H], @Epos[>=S,H], @Eseg[2,H], @g f32[H], @b f32[H])
+ *                                                  LN(Etok[tok] + Epos[s] + Eseg[seg]) -> [B*S,H]
+ *     attention(%qkv[B*S,3H]) {heads,seq}          softmax(Q K^T/sqrt(dh)) V per head -> [B*S,H]
+ *                                                  (no mask; seq <= 512, dh in {32,64,128})
+ *     add_layernorm(%a[M,H], %b[M,H], @g, @b)      LN(a + b) -> [M,H]
+ *     select_rows(%x[M,K]) {stride,offset}         rows offset + i*stride -> [rows,K]
  *     opaque(%in...)   structure + declared output bytes only; no kernel (scheduler fixtures
  *                      used with duet_profile_from_table; duet_run rejects it)
- *   act := none | relu | sigmoid | tanh.  Activations are stored in the node's declared dtype
+ *   act := none | relu | sigmoid | tanh | gelu (erf form).  Activations are stored in the node's declared dtype
  *   (bf16 graphs: bf16 weights/activations, fp32 accumulation, fp32 LSTM cell state).
  */
 #ifndef DUET_H_
