@@ -188,20 +188,29 @@ class Executor:
         self.store = {}
 
     def _exchange(self, phase: int):
-        ops = []
+        ops, landed = [], []
+        # gloo moves host tensors only: device tensors are staged through host memory (the one-GPU
+        # test of the multi-rank path; NCCL sends and receives device memory directly)
+        staged = self.device.type == "cuda" and dist.get_backend() == "gloo"
         for t in self.pl.transfers:
             if t.phase != phase or self.rank not in (t.src, t.dst):
                 continue
             if self.rank == t.src:
-                ops.append(dist.P2POp(dist.isend, self.store[t.tensor].contiguous(), t.dst))
+                x = self.store[t.tensor].contiguous()
+                ops.append(dist.P2POp(dist.isend, x.cpu() if staged else x, t.dst))
             else:
                 buf = self.store.get(t.tensor)
                 if buf is None:
                     buf = self.store[t.tensor] = self.alloc(*self.pl.tensor_meta[t.tensor])
-                ops.append(dist.P2POp(dist.irecv, buf, t.src))
+                tmp = torch.empty(buf.shape, dtype=buf.dtype) if staged else buf
+                if staged:
+                    landed.append((buf, tmp))
+                ops.append(dist.P2POp(dist.irecv, tmp, t.src))
         if ops:
             for w in dist.batch_isend_irecv(ops):
                 w.wait()
+        for buf, tmp in landed:
+            buf.copy_(tmp)
 
     def step(self, inputs: dict | None = None):
         if inputs:

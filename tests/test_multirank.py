@@ -102,3 +102,25 @@ def test_bench_two_ranks_on_one_gpu():
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["config"]["global_batch"] == 2 and d["value"] > 0
+
+
+@pytest.mark.gpu
+def test_bench_branch_placement_two_ranks_on_one_gpu():
+    """bench.py --placement branch under torchrun with 2 ranks (both on GPU 0 over gloo, tensors staged
+    through host memory): c3's two towers placed on the 2 ranks by greedy-correction, cut edges sent
+    point-to-point, rank 0 prints one JSON line with the placement."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, DUET_DIST_BACKEND="gloo", DUET_FORCE_DEVICE="0")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
+           "127.0.0.1", "--master-port", "29543", "bench.py", "--config", "c3", "--placement", "branch", "--gpus",
+           "2", "--steps", "3", "--warmup", "3", "--profile-samples", "5"]
+    r = subprocess.run(cmd, env=env, cwd=root, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["scaling"] == "strong" and len(set(d["placement"]["sg_gpu"])) >= 1
