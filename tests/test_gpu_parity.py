@@ -571,3 +571,28 @@ def test_branch_placement_pieces_on_device():
     for o in pl.graph_outputs:
         err = rel_err(store[o].float().cpu().numpy(), want[o])
         assert err <= TOL["bf16"], (o, err)
+
+
+def test_bench_contract_keys():
+    """`python bench.py` (the driver's default N=1 run, shortened): one JSON line with the contract's
+    keys, the roofline of the dominant kernel measured live, the CPU-oracle baseline and the e2e leg."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "bench.py", "--steps", "10", "--warmup", "3", "--cpu-seconds", "1",
+                        "--profile-samples", "5"], cwd=root, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "e2e", "gpu_launches", "roofline", "cpu_baseline", "clocks"):
+        assert k in d, k
+    assert d["steps"] == 10 and d["warmup"] == 3 and d["n_gpus"] == 1 and d["value"] > 0
+    assert d["config"]["workload"] == "c2_wide_deep"
+    assert d["roofline"]["bound"] == "tensor" and 0 < d["roofline"]["frac"] < 1
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["value"] > 0
+    assert d["e2e"]["h2d_bytes_per_step"] == 2048 * 26 * 8 and d["e2e"]["d2h_bytes_per_step"] == 2048 * 4
+    assert d["gpu_launches"] >= d["steps"]
