@@ -325,17 +325,23 @@ __global__ void __launch_bounds__(kRThreads, 1)
     const int half = (warp - 2) >> 2;
     const int H = a.H;
     if constexpr (!MULTI) {
-      // one tile for the whole sequence: bias and the recurrent state (LSTM c, GRU h in fp32) stay
-      // in registers
+      // one tile for the whole sequence: the recurrent state (LSTM c, GRU h in fp32) stays in
+      // registers, and so does the bias for UH <= 16; 128 x 256 tiles (UH = 32) work in chunks of
+      // 16 units with the bias read from shared memory (128 accumulator + 128 bias registers would
+      // spill)
+      constexpr int CU = UH <= 16 ? UH : 16;  // units per chunk
+      constexpr int NCH = UH / CU;
       const int row = tile_m0(0) + q * 32 + lane;
       const int unit0 = (tile_n0(0) / BN) * U + half * UH;
       const int nv = min(UH, H - unit0);  // multiple of 8 (H % 8 == 0)
       const bool live = row < a.B && nv > 0;
-      float bias[4][UH];
+      float bias[4][NCH == 1 ? UH : 1];
+      if constexpr (NCH == 1) {
 #pragma unroll
-      for (int g = 0; g < 4; ++g)
+        for (int g = 0; g < 4; ++g)
 #pragma unroll
-        for (int i = 0; i < UH; ++i) bias[g][i] = s_bias[g * U + half * UH + i];
+          for (int i = 0; i < UH; ++i) bias[g][i] = s_bias[g * U + half * UH + i];
+      }
       float state[UH];  // LSTM: c_{t-1}; GRU: h_{t-1} (fp32)
 #pragma unroll
       for (int i = 0; i < UH; ++i) state[i] = 0.0f;
@@ -345,25 +351,40 @@ __global__ void __launch_bounds__(kRThreads, 1)
         ptx::tc_fence_after();
         if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 2] = rp_gtimer();
         const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
-        float acc[4][UH];
 #pragma unroll
-        for (int g = 0; g < 4; ++g) tmem_ld_n<UH>(tq + g * U + half * UH, acc[g]);
-        ptx::tc_fence_before();
-        __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&tempty[buf]);  // accumulator buffer free for step t+2
-        if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 6] = rp_gtimer();  // TMEM read
-        float h[UH];
+        for (int ch = 0; ch < NCH; ++ch) {
+          float acc[4][CU];
 #pragma unroll
-        for (int i = 0; i < UH; ++i) h[i] = cell<KIND>(acc[0][i] + bias[0][i], acc[1][i] + bias[1][i],
-                                                        acc[2][i] + bias[2][i], acc[3][i] + bias[3][i], state[i]);
-        if (live) {
+          for (int g = 0; g < 4; ++g) tmem_ld_n<CU>(tq + g * U + half * UH + ch * CU, acc[g]);
+          if (ch == NCH - 1) {
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&tempty[buf]);  // accumulator buffer free for step t+2
+            if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 6] = rp_gtimer();  // TMEM read
+          }
+          float h[CU];
 #pragma unroll
-          for (int v = 0; v < UH / 8; ++v)
-            if (v * 8 < nv) {
-              if (a.seq) store_bf16x8(a.seq + ((size_t)t * a.B + row) * H + unit0 + 8 * v, h + 8 * v);
-              if (t == S - 1) store_bf16x8(a.out + (size_t)row * H + unit0 + 8 * v, h + 8 * v);
-              else store_bf16x8(a.hbuf[buf] + hs_index(row, unit0 + 8 * v, a.Bp), h + 8 * v);
+          for (int i = 0; i < CU; ++i) {
+            float b0, b1, b2, b3;
+            if constexpr (NCH == 1) {
+              b0 = bias[0][i], b1 = bias[1][i], b2 = bias[2][i], b3 = bias[3][i];
+            } else {
+              const int c = half * UH + ch * CU + i;
+              b0 = s_bias[c], b1 = s_bias[U + c], b2 = s_bias[2 * U + c], b3 = s_bias[3 * U + c];
             }
+            h[i] = cell<KIND>(acc[0][i] + b0, acc[1][i] + b1, acc[2][i] + b2, acc[3][i] + b3, state[ch * CU + i]);
+          }
+          if (live) {
+#pragma unroll
+            for (int v = 0; v < CU / 8; ++v) {
+              const int uo = ch * CU + 8 * v;  // unit offset within this thread's UH units
+              if (uo < nv) {
+                if (a.seq) store_bf16x8(a.seq + ((size_t)t * a.B + row) * H + unit0 + uo, h + 8 * v);
+                if (t == S - 1) store_bf16x8(a.out + (size_t)row * H + unit0 + uo, h + 8 * v);
+                else store_bf16x8(a.hbuf[buf] + hs_index(row, unit0 + uo, a.Bp), h + 8 * v);
+              }
+            }
+          }
         }
         if (trace && t < 64 && lane == 0) trace[t * 16 + 6 + warp] = rp_gtimer();  // [8..15] math + stores
         if (t < S - 1) {
@@ -559,13 +580,12 @@ void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0
   if (kind == EPI_LSTM && bn == 128) return launch_rp_any<128, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_GRU && bn == 64) return launch_rp_any<64, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_GRU && bn == 128) return launch_rp_any<128, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
-  // 128 x 256 tiles (64 units) only with several tiles per CTA (large batches): half the W bytes per
-  // FLOP of bn = 128, double-buffered accumulators fill all 512 TMEM columns
-  if (bn == 256 && a.tiles_n * a.tiles_m > grid) {
-    if (kind == EPI_LSTM) return launch_rp_multi<256, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
-    return launch_rp_multi<256, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
-  }
-  fail(DUET_EUNSUPPORTED, "rnn_persist: bn must be 64 or 128 (256: several tiles per CTA only)");
+  // 128 x 256 tiles (64 units): half the W bytes per FLOP of bn = 128, double-buffered accumulators
+  // fill all 512 TMEM columns; one tile per CTA when 128 x 256 tiles fit the SMs (c5's LSTM256),
+  // else several
+  if (bn == 256 && kind == EPI_LSTM) return launch_rp_any<256, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
+  if (bn == 256 && kind == EPI_GRU) return launch_rp_any<256, EPI_GRU>(tx, th0, th1, tw, a, grid, st);
+  fail(DUET_EUNSUPPORTED, "rnn_persist: bn must be 64, 128 or 256");
 }
 
 }  // namespace duet

@@ -369,6 +369,16 @@ void build_op(Program& P, const Node& n, Op& op) {
           break;
         }
       }
+      // else one tile per CTA on all SMs when 128 x 128 or 128 x 256 tiles fit (c5's LSTM256 at
+      // B = 4096: 128 tiles of 128 x 256, 11.0 -> 6.8 us per step; several tiles per CTA cost about
+      // one step per tile)
+      for (int cand : {128, 256}) {
+        const int tl = mt * ((H + cand / 4 - 1) / (cand / 4));
+        if (!rp_bn && !rp_bn_env && tl <= sms) {
+          rp_bn = cand;
+          rp_grid = tl;
+        }
+      }
       if (!rp_bn) {
         // several tiles per CTA: 128 x 256 tiles (64 units; half the W bytes per FLOP of 128 x 128,
         // c5's b2/b4/b5 -9/-24/-25%) while they still outnumber the SMs (rnn_persist's bn = 256

@@ -333,6 +333,8 @@ def test_rnn_node(kind, S, B, E, H, dt):
     ("lstm", 3, 2048, 128, 256, "bf16"),  # persistent kernel, several tiles per CTA (state in HBM)
     ("lstm", 3, 4096, 256, 512, "bf16"),  # several 128 x 256 tiles per CTA
     ("gru", 3, 4000, 136, 520, "bf16"),   # 128 x 256 tiles, ragged B, H and E
+    ("lstm", 4, 2304, 128, 264, "bf16"),  # one 128 x 256 tile per CTA (90 tiles), ragged H
+    ("gru", 3, 4096, 128, 256, "bf16"),   # one 128 x 256 tile per CTA (c5's b3 shape, GRU)
     ("gru", 4, 33, 24, 40, "f32"),        # CUDA-core parity path
 ])
 def test_rnn_node_seq_output(kind, S, B, E, H, dt):
