@@ -178,6 +178,10 @@ __global__ void __launch_bounds__(kRThreads, 1)
   auto tile_m0 = [&](int i) { return ((int)(blockIdx.x + i * gridDim.x) / a.tiles_n) * RBM; };
   const int cta = blockIdx.x;
   unsigned long long* trace = (a.dbg & 1) && !MULTI && cta < 128 ? g_rp_trace + (size_t)cta * 64 * 16 : nullptr;
+  // several tiles per CTA: stamps per work unit u = t * my_tiles + i < 64 (tools/rnn_trace_multi.py):
+  // 0 barrier observed (i = 0), 7 first A load issued, 11 first W load issued, 1 first stage landed,
+  // 4 first h stage landed, 5 last UMMA issued, 2 accumulator ready, 6 TMEM read, 3 released
+  unsigned long long* mtr = (a.dbg & 1) && MULTI && cta < 128 ? g_rp_trace + (size_t)cta * 64 * 16 : nullptr;
 
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tmX);
@@ -234,9 +238,11 @@ __global__ void __launch_bounds__(kRThreads, 1)
               }
               fence_proxy_async_global();
               if (trace && t < 64) trace[t * 16 + 0] = rp_gtimer();
+              if (mtr && t * my_tiles < 64) mtr[(t * my_tiles) * 16 + 0] = rp_gtimer();
             }
             __syncwarp();
           }
+          if (mtr && lane == 0 && j == 0 && t * my_tiles + i < 64) mtr[(t * my_tiles + i) * 16 + 7] = rp_gtimer();
           if (lane == 0) {
             ptx::mbar_arrive_expect_tx(&full[s], R_A_BYTES);
             if (CN == 1 || (int)crank == j % CN) {
@@ -274,6 +280,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
           for (int j = 0; j < nkb; ++j, ++g) {
             const int s = g % STAGES;
             if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
+            if (mtr && lane == 0 && j == 0 && t * my_tiles + i < 64) mtr[(t * my_tiles + i) * 16 + 11] = rp_gtimer();
             if (lane == 0) {
               ptx::mbar_arrive_expect_tx(&full[s], C::B_BYTES);
               // packed weight columns: [x part (kx blocks) | h part (kh blocks)] -> column block j
@@ -306,6 +313,10 @@ __global__ void __launch_bounds__(kRThreads, 1)
             if (j == 0) trace[t * 16 + 1] = rp_gtimer();
             if (j == kx) trace[t * 16 + 4] = rp_gtimer();  // first h stage landed
           }
+          if (mtr && u < 64 && lane == 0) {
+            if (j == 0) mtr[u * 16 + 1] = rp_gtimer();
+            if (j == kx) mtr[u * 16 + 4] = rp_gtimer();
+          }
           const uint64_t da = da0 + (uint64_t)((s * R_A_BYTES) >> 4);
           const uint64_t db = db0 + (uint64_t)(((WRES ? j : s) * C::B_BYTES) >> 4);
           if (!(a.dbg & 16))
@@ -316,6 +327,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
         }
         ptx::umma_commit_elect(&tfull[buf]);
         if (trace && t < 64 && lane == 0) trace[t * 16 + 5] = rp_gtimer();  // last UMMA issued
+        if (mtr && u < 64 && lane == 0) mtr[u * 16 + 5] = rp_gtimer();
       }
     }
   } else {
@@ -433,6 +445,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
           }
           wait_sleep(&tfull[buf], (u >> 1) & 1);
           ptx::tc_fence_after();
+          if (mtr && u < 64 && threadIdx.x == 64) mtr[u * 16 + 2] = rp_gtimer();
           const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
           // UH <= 16: every chunk's accumulators are read before the buffer is released; UH = 32
           // (bn = 256) reads chunk by chunk (128 live floats would spill) and releases at the end
@@ -446,6 +459,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
             ptx::tc_fence_before();
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&tempty[buf]);
+            if (mtr && u < 64 && threadIdx.x == 64) mtr[u * 16 + 6] = rp_gtimer();
           };
           if constexpr (CH > 1) {
 #pragma unroll
@@ -484,6 +498,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
             if (threadIdx.x == 64) {
               __threadfence();
               red_release_gpu_add(a.counter, 1u);
+              if (mtr && u < 64) mtr[u * 16 + 3] = rp_gtimer();
             }
           }
         }
