@@ -410,8 +410,18 @@ __global__ void __launch_bounds__(kRThreads, 1)
         }
       }
     } else {
-      // several tiles per CTA: the state lives in global memory (LSTM c fp32 [B, H]; GRU reads
-      // h_{t-1} back in bf16, as the per-step kernel does); chunks of 8 units bound the registers
+      // several tiles per CTA: with two tiles the recurrent state (LSTM c, GRU h, fp32) stays in
+      // registers, one array per tile (its global round trip cost c5's LSTM512 ~4.4 us per step,
+      // DESIGN.md "Persistent recurrence"); with more tiles it lives in global memory (LSTM c fp32
+      // [B, H]; GRU reads h_{t-1} back in bf16, as the per-step kernel does).  Chunks of 8 units
+      // bound the registers.
+      // (LSTM only: GRU's bf16 h read-back is cheap, and the extra registers measured slower there)
+      constexpr bool kRegs = KIND == EPI_LSTM;
+      constexpr int RS = kRegs ? UH : 1;
+      const bool regs = kRegs && my_tiles <= 2;
+      float rs0[RS], rs1[RS];
+#pragma unroll
+      for (int k2 = 0; k2 < RS; ++k2) rs0[k2] = rs1[k2] = 0.0f;
       int u = 0;
       for (int t = 0; t < S; ++t) {
         for (int i = 0; i < my_tiles; ++i, ++u) {
@@ -426,7 +436,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
 #pragma unroll
             for (int c = 0; c < UH / 8; ++c) {
               const int unit = (n0 / BN) * U + half * UH + 8 * c;
-              if (t == 0 || row >= a.B || unit >= H) {
+              if (regs || t == 0 || row >= a.B || unit >= H) {
 #pragma unroll
                 for (int e = 0; e < 8; ++e) stp[c][e] = 0.0f;
               } else if constexpr (KIND == EPI_LSTM) {
@@ -475,7 +485,12 @@ __global__ void __launch_bounds__(kRThreads, 1)
             const int unit = (n0 / BN) * U + half * UH + 8 * c;
             if (row >= a.B || unit >= H) continue;
             const size_t off = (size_t)row * H + unit;
-            float* st = stp[c];
+            float st[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+              if constexpr (kRegs) st[e] = regs ? (i == 0 ? rs0[8 * c + e] : rs1[8 * c + e]) : stp[c][e];
+              else st[e] = stp[c][e];
+            }
             const int cb = n0 + half * UH + 8 * c;  // packed bias column of gate block 0
             float h[8];
 #pragma unroll
@@ -483,7 +498,15 @@ __global__ void __launch_bounds__(kRThreads, 1)
               h[e] = cell<KIND>(acc[c][0][e] + __ldg(a.bias + cb + e), acc[c][1][e] + __ldg(a.bias + cb + U + e),
                                 acc[c][2][e] + __ldg(a.bias + cb + 2 * U + e),
                                 acc[c][3][e] + __ldg(a.bias + cb + 3 * U + e), st[e]);
-            if constexpr (KIND == EPI_LSTM) {
+            if (regs) {
+              if constexpr (kRegs) {
+#pragma unroll
+                for (int e = 0; e < 8; ++e) {
+                  if (i == 0) rs0[8 * c + e] = st[e];
+                  else rs1[8 * c + e] = st[e];
+                }
+              }
+            } else if constexpr (KIND == EPI_LSTM) {
               *reinterpret_cast<float4*>(a.c_state + off) = make_float4(st[0], st[1], st[2], st[3]);
               *reinterpret_cast<float4*>(a.c_state + off + 4) = make_float4(st[4], st[5], st[6], st[7]);
             }
