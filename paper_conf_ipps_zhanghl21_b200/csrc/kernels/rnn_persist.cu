@@ -519,7 +519,8 @@ __global__ void __launch_bounds__(kRThreads, 1)
             fence_proxy_async_global();
             asm volatile("bar.sync 1, %0;" ::"n"(32 * kREpiWarps) : "memory");
             if (threadIdx.x == 64) {
-              __threadfence();
+              // bar.sync orders the CTA's h stores before this thread's release, which is
+              // cumulative at gpu scope (no separate __threadfence)
               red_release_gpu_add(a.counter, 1u);
               if (mtr && u < 64) mtr[u * 16 + 3] = rp_gtimer();
             }
