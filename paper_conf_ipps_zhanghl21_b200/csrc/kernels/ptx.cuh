@@ -219,6 +219,28 @@ __device__ __forceinline__ void tmem_ld64(uint32_t taddr, float* v) {
 #pragma unroll
   for (int i = 0; i < 64; ++i) v[i] = __uint_as_float(r[i]);
 }
+// four 32-lane x 8-column loads (addresses a0..a3) behind one wait::ld
+__device__ __forceinline__ void tmem_ld8x4(uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3, float (*v)[8]) {
+  uint32_t r[4][8];
+#define DUET_LD8(I, A)                                                                                     \
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"                  \
+               : "=r"(r[I][0]), "=r"(r[I][1]), "=r"(r[I][2]), "=r"(r[I][3]), "=r"(r[I][4]), "=r"(r[I][5]), \
+                 "=r"(r[I][6]), "=r"(r[I][7])                                                            \
+               : "r"(A));
+  DUET_LD8(0, a0) DUET_LD8(1, a1) DUET_LD8(2, a2) DUET_LD8(3, a3)
+#undef DUET_LD8
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+    asm volatile("tcgen05.wait::ld.sync.aligned;"
+                 : "+r"(r[i][0]), "+r"(r[i][1]), "+r"(r[i][2]), "+r"(r[i][3]), "+r"(r[i][4]), "+r"(r[i][5]),
+                   "+r"(r[i][6]), "+r"(r[i][7])
+                 :
+                 : "memory");  // the first waits, the rest pin the registers after it
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[i][j] = __uint_as_float(r[i][j]);
+}
 __device__ __forceinline__ void tmem_ld8(uint32_t taddr, float* v) {
   uint32_t r[8];
   asm volatile(

@@ -461,9 +461,9 @@ __global__ void __launch_bounds__(kRThreads, 1)
           // (bn = 256) reads chunk by chunk (128 live floats would spill) and releases at the end
           constexpr int CH = UH <= 16 ? UH / 8 : 1;
           float acc[UH / 8][4][8];
-          auto load_chunk = [&](int c) {
-#pragma unroll
-            for (int g = 0; g < 4; ++g) ptx::tmem_ld8(tq + g * U + half * UH + 8 * c, acc[c][g]);
+          auto load_chunk = [&](int c) {  // the four gate blocks of 8 units, one wait
+            const uint32_t a0 = tq + half * UH + 8 * c;
+            ptx::tmem_ld8x4(a0, a0 + U, a0 + 2 * U, a0 + 3 * U, acc[c]);
           };
           auto release = [&]() {
             ptx::tc_fence_before();
