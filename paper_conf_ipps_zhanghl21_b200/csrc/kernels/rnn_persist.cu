@@ -141,6 +141,23 @@ __device__ __forceinline__ void store_bf16x8(__nv_bfloat16* dst, const float* h)
   *reinterpret_cast<uint4*>(dst) = make_uint4(w[0], w[1], w[2], w[3]);
 }
 
+// the four gate blocks (N columns each, U apart) behind a single wait::ld
+template <int N>
+__device__ __forceinline__ void tmem_ld_gates(uint32_t taddr, int U, float (*v)[N]) {
+  if constexpr (N == 8) {
+    ptx::tmem_ld8x4(taddr, taddr + U, taddr + 2 * U, taddr + 3 * U, v);
+  } else {
+    uint32_t r[4][16];
+#pragma unroll
+    for (int g = 0; g < 4; ++g) ptx::tmem_ld16_nowait(taddr + g * U, r[g]);
+#pragma unroll
+    for (int g = 0; g < 4; ++g) ptx::tmem_wait_ld16(r[g]);  // the first waits, the rest pin the registers
+#pragma unroll
+    for (int g = 0; g < 4; ++g)
+#pragma unroll
+      for (int i = 0; i < 16; ++i) v[g][i] = __uint_as_float(r[g][i]);
+  }
+}
 template <int N>
 __device__ __forceinline__ void tmem_ld_n(uint32_t taddr, float* v) {
   if constexpr (N == 16) ptx::tmem_ld16(taddr, v);
@@ -366,8 +383,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
 #pragma unroll
         for (int ch = 0; ch < NCH; ++ch) {
           float acc[4][CU];
-#pragma unroll
-          for (int g = 0; g < 4; ++g) tmem_ld_n<CU>(tq + g * U + half * UH + ch * CU, acc[g]);
+          tmem_ld_gates<CU>(tq + half * UH + ch * CU, U, acc);
           if (ch == NCH - 1) {
             ptx::tc_fence_before();
             __syncwarp();
