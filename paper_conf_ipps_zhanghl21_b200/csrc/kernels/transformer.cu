@@ -140,6 +140,7 @@ __global__ void __launch_bounds__(32 * kAttWarps) attention_kernel(const void* q
   float* Kt = att_smem;
   float* Vs = Kt + (size_t)dh * ldk;
   float* Qs = Vs + (size_t)Sp * dh;
+  float* Ps = Qs + (size_t)kAttWarps * dh;  // [warps][Sp] softmax probabilities
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   ptx::pdl_wait();
   ptx::pdl_trigger();
@@ -212,22 +213,27 @@ __global__ void __launch_bounds__(32 * kAttWarps) attention_kernel(const void* q
       sum += p[t];
     }
     const float inv = 1.0f / warp_sum(sum);
-    float acc[2][DV];
+    // probabilities -> this warp's smem row, then every lane walks the keys with broadcast reads
+    // (a shuffle per key serialised the PV loop on its latency)
+    float* pw = Ps + warp * Sp;
 #pragma unroll
-    for (int v = 0; v < DV; ++v) acc[0][v] = acc[1][v] = 0.0f;
+    for (int t = 0; t < NT; ++t) pw[t * 32 + lane] = p[t];
+    __syncwarp();
+    float acc[4][DV];
 #pragma unroll
-    for (int t = 0; t < NT; ++t) {
-      const float* vr = Vs + (size_t)(t * 32) * dh + lane;
+    for (int v = 0; v < DV; ++v) acc[0][v] = acc[1][v] = acc[2][v] = acc[3][v] = 0.0f;
+    const float* vr = Vs + lane;
 #pragma unroll 8
-      for (int l = 0; l < 32; ++l) {
-        const float pj = __shfl_sync(0xffffffffu, p[t], l);
+    for (int jj = 0; jj < 32 * NT; ++jj) {
+      const float pj = pw[jj];
 #pragma unroll
-        for (int v = 0; v < DV; ++v) acc[l & 1][v] = fmaf(pj, vr[l * dh + 32 * v], acc[l & 1][v]);
-      }
+      for (int v = 0; v < DV; ++v) acc[jj & 3][v] = fmaf(pj, vr[jj * dh + 32 * v], acc[jj & 3][v]);
     }
+#pragma unroll
+    for (int v = 0; v < DV; ++v) acc[0][v] += acc[1][v] + acc[2][v] + acc[3][v];
     const int64_t o = ((int64_t)b * S + qi) * H + (int64_t)h * dh + lane;
 #pragma unroll
-    for (int v = 0; v < DV; ++v) stv(out, o + 32 * v, (acc[0][v] + acc[1][v]) * inv, bf16);
+    for (int v = 0; v < DV; ++v) stv(out, o + 32 * v, acc[0][v] * inv, bf16);
     __syncwarp();
   }
 }
@@ -248,7 +254,7 @@ int att_nt(int S) {  // key chunks of the instantiated kernel (1, 2, 4, 6, 8, 12
 }
 size_t att_smem_bytes(int S, int dh) {
   const size_t sp = (size_t)32 * att_nt(S);
-  return ((size_t)dh * (sp + 1) + sp * dh + (size_t)kAttWarps * dh) * 4;
+  return ((size_t)dh * (sp + 1) + sp * dh + (size_t)kAttWarps * dh + (size_t)kAttWarps * sp) * 4;
 }
 
 }  // namespace
