@@ -320,6 +320,24 @@ Schedule* make_schedule_with(const Partition* p, const Profile* pr, const duet_s
       }
     }
   }
+  // measured mode: the slots are identical in the model but not on the device (the home slot's
+  // stream has normal priority, the others high), so relabelling the slots
+  // of the chosen assignment can change its measured latency -- c2 measured 5% faster with the
+  // critical path off the home slot (profiles/r1c_fig13.md).  Step 3's `measure latency` therefore
+  // also tries every relabelling (D <= 4) and keeps the fastest.
+  if (measured && (opts.mode == 0 || opts.mode == 6) && m.D >= 2 && m.D <= 4) {
+    std::vector<int> perm(m.D);
+    for (int d = 0; d < m.D; ++d) perm[d] = d;
+    int64_t best = lat(a);
+    std::vector<int> best_a = a;
+    while (std::next_permutation(perm.begin(), perm.end())) {
+      std::vector<int> b(a.size());
+      for (size_t s = 0; s < a.size(); ++s) b[s] = perm[a[s]];
+      const int64_t v = lat(b);
+      if (v < best) best = v, best_a = b;
+    }
+    a = best_a;
+  }
   S->slot_of = a;
   for (int s = 0; s < m.n; ++s) S->order.push_back(s);
   S->makespan = m.makespan(a);
