@@ -52,6 +52,9 @@
  *                                                  (PyTorch r,z,n; b_hn inside r*(.))
  *     lstm / gru {seq=1}                           every h_t -> [S,B,H] (a lower layer of a stacked
  *                                                  RNN, Fig. 14)
+ *     lstm / gru {tile_n=64|128|256}               gate-tile width of the persistent recurrence
+ *                                                  (an SM budget when branches share the GPU;
+ *                                                  absent = automatic; other values DUET_EINVAL)
  *     conv2d_bn(%x[N,H,W,C], @W[Co,kh,kw,C], @gamma,@beta,@mean,@var f32[Co]) {stride,pad,act}
  *                                                  NHWC conv + inference BN (eps 1e-5) + act
  *     add(%a, %b) {act}   maxpool(%x) {k,stride,pad}   avgpool(%x[N,H,W,C]) -> [N,C]

@@ -356,7 +356,12 @@ void build_op(Program& P, const Node& n, Op& op) {
     // the SMs (two recurrent branches on two slots co-reside), else every SM with several tiles per
     // CTA (large batches).  DUET_RNN_PERSIST=0 forces the per-step kernels.
     static const int rp_env = getenv("DUET_RNN_PERSIST") ? atoi(getenv("DUET_RNN_PERSIST")) : 1;
-    static const int rp_bn_env = getenv("DUET_RNN_BN") ? atoi(getenv("DUET_RNN_BN")) : 0;
+    // gate-tile width: the node's tile_n attribute (a per-workload SM budget, DESIGN.md "SM sharing
+    // between concurrent branches"), else DUET_RNN_BN (experiments), else automatic
+    static const int rp_bn_env0 = getenv("DUET_RNN_BN") ? atoi(getenv("DUET_RNN_BN")) : 0;
+    const int rp_bn_env = (int)n.attr_int("tile_n", rp_bn_env0);
+    if (rp_bn_env != 0 && rp_bn_env != 64 && rp_bn_env != 128 && rp_bn_env != 256)
+      fail(DUET_EINVAL, "%" + n.name + ": tile_n must be 64, 128 or 256");
     int rp_bn = 0, rp_grid = 0;
     if (tc && rp_env) {
       const int mt = (B + 127) / 128;

@@ -106,8 +106,10 @@ class _Builder:
         return self.node(name, "mlp", args, out_dt or self.dt, (m, dims[-1]), act=act,
                          last_act=last_act)
 
-    def rnn(self, name, kind, x, e, h, s, b, seq=False):
-        """seq=True: output every h_t as [S, B, H] (a lower layer of a stacked RNN)."""
+    def rnn(self, name, kind, x, e, h, s, b, seq=False, tile_n=0):
+        """seq=True: output every h_t as [S, B, H] (a lower layer of a stacked RNN).  tile_n: the
+        persistent recurrence's gate-tile width (0 = automatic)."""
+        kw = {"tile_n": tile_n} if tile_n else {}
         g = 4 if kind == "lstm" else 3
         bd = 1.0 / math.sqrt(h)
         Wih = self.param(f"{name}_Wih", self.dt, (g * h, e), ("uniform", bd))
@@ -115,15 +117,16 @@ class _Builder:
         bih = self.param(f"{name}_bih", "f32", (g * h,), ("uniform", bd))
         bhh = self.param(f"{name}_bhh", "f32", (g * h,), ("uniform", bd))
         if seq:
-            return self.node(name, kind, [x, Wih, Whh, bih, bhh], self.dt, (s, b, h), seq=1)
-        return self.node(name, kind, [x, Wih, Whh, bih, bhh], self.dt, (b, h))
+            return self.node(name, kind, [x, Wih, Whh, bih, bhh], self.dt, (s, b, h), seq=1, **kw)
+        return self.node(name, kind, [x, Wih, Whh, bih, bhh], self.dt, (b, h), **kw)
 
-    def stacked_rnn(self, name, kind, x, e, h, s, b, layers=1):
+    def stacked_rnn(self, name, kind, x, e, h, s, b, layers=1, tile_n=0):
         """`layers` stacked RNNs (Fig. 14): layers 0..L-2 return their whole output
         sequence, the top layer h_S.  The top layer keeps the plain name (layers=1 is the plain RNN)."""
         for li in range(layers - 1):
-            x = self.rnn(f"{name}_l{li}", kind, x, e if li == 0 else h, h, s, b, seq=True)
-        return self.rnn(name, kind, x, e if layers == 1 else h, h, s, b)
+            x = self.rnn(f"{name}_l{li}", kind, x, e if li == 0 else h, h, s, b, seq=True,
+                         tile_n=tile_n)
+        return self.rnn(name, kind, x, e if layers == 1 else h, h, s, b, tile_n=tile_n)
 
     def conv_bn(self, name, x, n, h, w, cin, cout, k, stride, pad, act, gamma=(0.5, 1.5)):
         ho = (h + 2 * pad - k) // stride + 1
@@ -252,10 +255,13 @@ def c3_two_tower(batch=256, seq=64, vocab=32768, emb=256, hidden=512, dt="bf16")
 # Join sigma(w . concat[512, 1024, 256] + b).
 # ------------------------------------------------------------------------------------------
 def c4_hybrid(batch=64, image=224, seq=64, vocab=32768, emb=256, gru_hidden=1024, fields=8,
-              rows=100_000, mlp_out=256, rnn_layers=1, resnet=18, ffn_layers=1, dt="bf16") -> Workload:
+              rows=100_000, mlp_out=256, rnn_layers=1, resnet=18, ffn_layers=1, dt="bf16",
+              gru_tile_n=128) -> Workload:
     """`rnn_layers`, `resnet` and `ffn_layers` are the model variations of PAPER.md:89 (§VI-D,
     Figs. 14-16: stacked RNN 1/2/4/8, ResNet 18/34/50/101, FFN depth); `batch` is Fig. 17's.
-    The defaults are BASELINE.json:10's configuration."""
+    The defaults are BASELINE.json:10's configuration.  gru_tile_n=128: the GRU runs half as many
+    persistent CTAs as with 64-wide gate tiles and leaves the SMs to the co-running ResNet
+    (measured c4 p50 0.905 -> 0.867 ms)."""
     B = _Builder("c4_hybrid", 4, dt)
     img = B.input("image", dt, (batch, image, image, 3), ("normal", 1.0))
     cnn = B.resnet("cnn", img, batch, image, image, resnet)
@@ -263,7 +269,7 @@ def c4_hybrid(batch=64, image=224, seq=64, vocab=32768, emb=256, gru_hidden=1024
     tok = B.input("tok", "i32", (batch, seq), ("randint", vocab))
     E = B.param("tok_E", dt, (vocab, emb), ("normal", 1.0))
     x = B.node("tok_x", "embed_seq", [tok, E], dt, (seq, batch, emb))
-    rnn = B.stacked_rnn("gru", "gru", x, emb, gru_hidden, seq, batch, rnn_layers)
+    rnn = B.stacked_rnn("gru", "gru", x, emb, gru_hidden, seq, batch, rnn_layers, gru_tile_n)
     raw = B.input("raw", "i64", (batch, fields), ("randint", 1 << 31))
     ids = B.node("ids", "hash_mod", [raw], "i32", (batch, fields), V=rows)
     T = B.param("mlp_E", dt, (fields, rows, 64), ("normal", 1.0))

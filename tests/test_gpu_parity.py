@@ -384,6 +384,32 @@ def test_model_variation_parity(layers, resnet, ffn, batch, dt):
         assert err <= TOL[dt], (name, err)
 
 
+@pytest.mark.parametrize("tile_n,layers", [(64, 1), (256, 1), (128, 2)])
+def test_rnn_tile_n_parity(tile_n, layers):
+    """The persistent recurrence's gate-tile width as a node attribute (c4's GRU runs 128-wide
+    tiles by default): every width gives the oracle's answer."""
+    wl = W.build("c4", small=True, branch_outputs=True, rnn_layers=layers, gru_tile_n=tile_n)
+    assert f"tile_n={tile_n}" in wl.ir
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    want = _oracle_outputs(wl, sess.params, dict(zip(wl.inputs, inputs)))
+    outs = sess.outputs()
+    sess.run(sess.schedule(), inputs, outs)
+    torch.cuda.synchronize()
+    for (name, _, _), y in zip(wl.outputs, outs):
+        err = rel_err(y.float().cpu().numpy(), want[name])
+        print(f"[parity] c4 gru tile_n={tile_n} L{layers} {name}: rel err {err:.3e}")
+        assert err <= TOL["bf16"], (name, err)
+
+
+def test_rnn_tile_n_invalid():
+    wl = W.build("c4", small=True, gru_tile_n=96)
+    with pytest.raises(duet.DuetError) as e:
+        Session(wl, n_slots=2, profile=FAST_PROFILE)
+    assert e.value.name == "EINVAL"
+    assert "tile_n" in str(e.value)
+
+
 @pytest.mark.parametrize("layers,resnet,ffn", [(8, 18, 1), (1, 101, 1), (1, 18, 8)])
 def test_model_variation_full_size_sampled(layers, resnet, ffn):
     """The deepest Fig. 14-16 variations at c4's full size (bench launch configuration); the oracle
