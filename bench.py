@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--profile-samples", type=int, default=100)
     ap.add_argument("--sched", default="measured", choices=["measured", "model"],
                     help="Step 3's `measure latency`: device measurement (default) or the C3 model")
+    ap.add_argument("--rnn-tiles", type=int, default=1,
+                    help="1: choose the recurrences' gate-tile width by measured latency (harness.tuned_session)")
     ap.add_argument("--placement", default="batch", choices=["batch", "branch"],
                     help="N>1: 'batch' = every rank runs its own batch (weak scaling); 'branch' = one batch, "
                          "subgraphs placed on the GPUs by greedy-correction, cut edges over NCCL (strong)")
@@ -383,7 +385,7 @@ def main():
     from paper_conf_ipps_zhanghl21_b200 import duet
     from paper_conf_ipps_zhanghl21_b200 import multirank as MR
     from paper_conf_ipps_zhanghl21_b200 import workloads as W
-    from paper_conf_ipps_zhanghl21_b200.harness import Session, materialize
+    from paper_conf_ipps_zhanghl21_b200.harness import Session, materialize, tuned_session
 
     rank, world, local = MR.env()
     torch.cuda.set_device(local)
@@ -391,14 +393,23 @@ def main():
     dev = f"cuda:{local}"
 
     wl = W.build(args.config, dt=args.dtype)
-    sess = Session(wl, n_slots=args.slots, device=local,
-                   profile=dict(warmup=5, samples=args.profile_samples, reps=10, calibrate_comm=True))
+    prof_opts = dict(warmup=5, samples=args.profile_samples, reps=10, calibrate_comm=True)
+    tile_ns = None
+    if args.sched == "measured" and W.rnn_nodes(wl) and args.rnn_tiles:
+        # the recurrences' gate-tile width chosen by measured latency (harness.tuned_session); the
+        # serial baseline keeps the automatic width (tuned for a branch running alone)
+        sess, duet_s, tile_ns, base = tuned_session(wl, n_slots=args.slots, device=local, profile=prof_opts,
+                                                    tile_candidates=(0, 128))
+    else:
+        sess = base = Session(wl, n_slots=args.slots, device=local, profile=prof_opts)
+        duet_s = None
     inputs = list(materialize(wl.inputs, dev).values())
     outs = sess.outputs()
     torch.cuda.synchronize()
     model_s = sess.schedule(duet.GREEDY_CORRECTION)
-    duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=30) if args.sched == "measured" else model_s
-    serial_s = sess.schedule(duet.SERIAL)
+    if duet_s is None:
+        duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=30) if args.sched == "measured" else model_s
+    serial_s = base.schedule(duet.SERIAL)
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
     home = sess.home
 
@@ -408,10 +419,12 @@ def main():
         duet_s.run(sess.slots, inputs, outs)
 
     def step_serial():
-        serial_s.run(sess.slots, inputs, outs)
+        serial_s.run(base.slots, inputs, outs)
 
     # serial 1-stream reference of the same kernels (BASELINE.json:2)
-    t_serial = time_steps(torch, step_serial, home, args.steps, args.warmup, flush)
+    base.home.wait_stream(torch.cuda.current_stream())
+    t_serial = time_steps(torch, step_serial, base.home, args.steps, args.warmup, flush)
+    torch.cuda.synchronize()
     t_model = None
     if duet_s is not model_s and duet_s.export()["slot_of"] != model_s.export()["slot_of"]:
         t_model = time_steps(torch, lambda: model_s.run(sess.slots, inputs, outs), home, args.steps, args.warmup,
@@ -504,7 +517,9 @@ def main():
                      "measured_ns": getattr(duet_s, "measured_ns", None),
                      "evaluations": getattr(duet_s, "evaluations", None),
                      "model_mode_slot_of": model_s.export()["slot_of"],
-                     "model_mode_p50_ms": round(statistics.median(t_model), 5) if t_model else None},
+                     "model_mode_p50_ms": round(statistics.median(t_model), 5) if t_model else None,
+                     "rnn_tile_n": sess.wl.meta.get("rnn_tile_n"),
+                     "rnn_tile_measured_ns": tile_ns},
         "e2e": {"value": round(world * wl.batch * args.steps / (e2e_ms / 1e3), 1), "unit": "samples/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "p50_ms": round(statistics.median(t_e2e), 5)},

@@ -64,3 +64,36 @@ class Session:
     @property
     def home(self) -> torch.cuda.Stream:
         return self.streams[0]
+
+
+def tuned_session(wl: Workload, n_slots: int = 2, device: int = 0, profile: dict | None = None,
+                  tile_candidates=(0, 128), samples: int = 30, mode=duet.GREEDY_CORRECTION):
+    """Kernel-variant choice by measurement (the compiler-aware profiler's idea, §IV-B:
+    each compiled variant is profiled, and the correction's, :81 §IV-C: candidate schedules are
+    compared by measured latency).  The variant here is the persistent recurrence's gate-tile width,
+    an SM budget when branches share one GPU:
+    the workload is built with each width in `tile_candidates` (applied to every LSTM/GRU node;
+    0 = the automatic choice), scheduled with measured greedy-correction, and the session with the
+    lowest measured latency is kept.  The weights are materialised once and shared.
+
+    Returns (best session, its measured schedule, {tile_n: measured ns}, the automatic-width session
+    (the serial baseline's kernels: tuned for running alone), or the best one if it is that)."""
+    from .workloads import rnn_nodes, with_rnn_tile_n
+    base = Session(with_rnn_tile_n(wl, 0) if rnn_nodes(wl) else wl, n_slots=n_slots, device=device,
+                   profile=profile)
+    torch.cuda.synchronize(device)
+    s0 = base.schedule(mode, measured=True, samples=samples)
+    results = {0: int(s0.measured_ns)}
+    best, best_s, best_ns = base, s0, s0.measured_ns
+    if rnn_nodes(wl):
+        for t in tile_candidates:
+            if t == 0:
+                continue
+            sess = Session(with_rnn_tile_n(wl, t), n_slots=n_slots, device=device,
+                           params=base.params, profile=profile)
+            torch.cuda.synchronize(device)
+            s = sess.schedule(mode, measured=True, samples=samples)
+            results[t] = int(s.measured_ns)
+            if s.measured_ns < best_ns:
+                best, best_s, best_ns = sess, s, s.measured_ns
+    return best, best_s, results, base

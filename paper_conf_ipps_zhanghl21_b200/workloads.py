@@ -256,12 +256,11 @@ def c3_two_tower(batch=256, seq=64, vocab=32768, emb=256, hidden=512, dt="bf16")
 # ------------------------------------------------------------------------------------------
 def c4_hybrid(batch=64, image=224, seq=64, vocab=32768, emb=256, gru_hidden=1024, fields=8,
               rows=100_000, mlp_out=256, rnn_layers=1, resnet=18, ffn_layers=1, dt="bf16",
-              gru_tile_n=128) -> Workload:
+              gru_tile_n=0) -> Workload:
     """`rnn_layers`, `resnet` and `ffn_layers` are the model variations of PAPER.md:89 (§VI-D,
     Figs. 14-16: stacked RNN 1/2/4/8, ResNet 18/34/50/101, FFN depth); `batch` is Fig. 17's.
-    The defaults are BASELINE.json:10's configuration.  gru_tile_n=128: the GRU runs half as many
-    persistent CTAs as with 64-wide gate tiles and leaves the SMs to the co-running ResNet
-    (measured c4 p50 0.905 -> 0.867 ms)."""
+    The defaults are BASELINE.json:10's configuration.  gru_tile_n: the GRU's gate-tile width
+    (0 = automatic; `with_rnn_tile_n` / `harness.tuned_session` choose it by measurement)."""
     B = _Builder("c4_hybrid", 4, dt)
     img = B.input("image", dt, (batch, image, image, 3), ("normal", 1.0))
     cnn = B.resnet("cnn", img, batch, image, image, resnet)
@@ -429,6 +428,31 @@ def with_branch_outputs(wl: Workload) -> Workload:
     order = {nm: i for i, nm in enumerate(decl)}
     outs.sort(key=lambda o: order[o[0]])
     return Workload(wl.name, "\n".join(lines) + "\n", wl.params, wl.inputs, outs, wl.batch, dict(wl.meta))
+
+
+def rnn_nodes(wl: Workload) -> list:
+    import re
+    return [m.group(1) for m in (re.match(r"^%([\w.]+) = (?:lstm|gru)\(", ln) for ln in wl.ir.splitlines()) if m]
+
+
+def with_rnn_tile_n(wl: Workload, tile_n: int) -> Workload:
+    """Every LSTM/GRU node with gate-tile width `tile_n` (0 = automatic; include/duet.h `tile_n`).
+    The width is an SM budget when branches share the GPU (DESIGN.md "SM sharing between concurrent
+    branches"): fewer, wider tiles leave SMs to a co-running branch but lengthen the recurrence."""
+    import re
+    out = []
+    for ln in wl.ir.splitlines():
+        if re.match(r"^%[\w.]+ = (?:lstm|gru)\(", ln):
+            head, tail = ln.rsplit(" : ", 1)
+            m = re.search(r" \{(.*)\}$", head)
+            attrs = [a for a in (m.group(1).split(", ") if m else []) if not a.startswith("tile_n=")]
+            if tile_n:
+                attrs.append(f"tile_n={tile_n}")
+            head = head[:m.start()] if m else head
+            ln = head + (" {" + ", ".join(attrs) + "}" if attrs else "") + " : " + tail
+        out.append(ln)
+    meta = dict(wl.meta, rnn_tile_n=tile_n)
+    return Workload(wl.name, "\n".join(out) + "\n", wl.params, wl.inputs, list(wl.outputs), wl.batch, meta)
 
 
 def build(name: str, small: bool = False, dt: str | None = None, branch_outputs: bool = False,

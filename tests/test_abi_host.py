@@ -157,3 +157,25 @@ def test_state_errors():
     with pytest.raises(duet.DuetError) as e:
         s.launch_count()
     assert e.value.name == "ESTATE"
+
+
+@pytest.mark.parametrize("cfg", ["c3", "c4", "c5"])
+def test_rnn_tile_n_rewrite(cfg):
+    """with_rnn_tile_n sets / clears the tile_n attribute on exactly the LSTM/GRU nodes, keeps
+    their other attributes, and leaves the partition (the IR's structure) unchanged."""
+    wl = W.build(cfg, small=True, **({"rnn_layers": 2} if cfg == "c4" else {}))
+    rnn = W.rnn_nodes(wl)
+    assert rnn
+    w128 = W.with_rnn_tile_n(wl, 128)
+    lines0, lines1 = wl.ir.splitlines(), w128.ir.splitlines()
+    assert len(lines0) == len(lines1)
+    for a, b in zip(lines0, lines1):
+        if any(a.startswith(f"%{n} = ") for n in rnn):
+            assert "tile_n=128" in b and b.replace(", tile_n=128", "").replace(" {tile_n=128}", "") == a
+        else:
+            assert a == b
+    assert W.with_rnn_tile_n(w128, 0).ir == wl.ir
+    assert w128.meta["rnn_tile_n"] == 128
+    p0 = duet.Graph(wl.ir).partition("coarse").export()
+    p1 = duet.Graph(w128.ir).partition("coarse").export()
+    assert p0 == p1

@@ -402,6 +402,28 @@ def test_rnn_tile_n_parity(tile_n, layers):
         assert err <= TOL["bf16"], (name, err)
 
 
+@pytest.mark.parametrize("cfg", ["c3", "c4"])
+def test_tuned_session_parity(cfg):
+    """harness.tuned_session (bench.py's default for workloads with recurrences): both gate-tile
+    widths are measured, the kept session is the faster one, and its outputs match the oracle."""
+    from paper_conf_ipps_zhanghl21_b200.harness import tuned_session
+    wl = W.build(cfg, small=True, branch_outputs=True)
+    sess, s, tiles, base = tuned_session(wl, n_slots=2, profile=FAST_PROFILE, samples=5)
+    assert set(tiles) == {0, 128} and all(v > 0 for v in tiles.values())
+    assert tiles[sess.wl.meta["rnn_tile_n"]] == min(tiles.values())
+    assert base.wl.meta["rnn_tile_n"] == 0 and base.params is sess.params
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    want = _oracle_outputs(wl, sess.params, dict(zip(wl.inputs, inputs)))
+    for sch, ss in ((s, sess), (base.schedule(duet.SERIAL), base)):
+        outs = ss.outputs()
+        ss.run(sch, inputs, outs)
+        torch.cuda.synchronize()
+        for (name, _, _), y in zip(wl.outputs, outs):
+            err = rel_err(y.float().cpu().numpy(), want[name])
+            print(f"[parity] {cfg} tuned tile_n={ss.wl.meta['rnn_tile_n']} {name}: rel err {err:.3e}")
+            assert err <= TOL["bf16"], (name, err)
+
+
 def test_rnn_tile_n_invalid():
     wl = W.build("c4", small=True, gru_tile_n=96)
     with pytest.raises(duet.DuetError) as e:

@@ -36,13 +36,14 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--slots", type=int, default=2)
     ap.add_argument("--out", default="gpurun_out/sweeps.json")
+    ap.add_argument("--rnn-tiles", type=int, default=1)
     args = ap.parse_args()
     import torch
 
     import bench
     from paper_conf_ipps_zhanghl21_b200 import duet
     from paper_conf_ipps_zhanghl21_b200 import workloads as W
-    from paper_conf_ipps_zhanghl21_b200.harness import Session, materialize
+    from paper_conf_ipps_zhanghl21_b200.harness import Session, materialize, tuned_session
 
     flush = torch.empty(bench.L2_FLUSH_BYTES // 4, dtype=torch.float32, device="cuda")
     res = {}
@@ -52,14 +53,22 @@ def main():
         for var in variants:
             t0 = time.time()
             wl = W.build("c4", **var)
-            sess = Session(wl, n_slots=args.slots, profile=dict(warmup=3, samples=30, reps=5, calibrate_comm=True))
+            popts = dict(warmup=3, samples=30, reps=5, calibrate_comm=True)
+            if args.rnn_tiles:  # gate-tile width chosen by measured latency (bench.py's default)
+                sess, duet_s, tile_ns, base = tuned_session(wl, n_slots=args.slots, profile=popts, samples=20)
+            else:
+                sess = base = Session(wl, n_slots=args.slots, profile=popts)
+                tile_ns = None
             inputs = list(materialize(wl.inputs, "cuda").values())
             outs = sess.outputs()
             torch.cuda.synchronize()
-            duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=20)
-            serial_s = sess.schedule(duet.SERIAL)
-            t_ser = bench.time_steps(torch, lambda: serial_s.run(sess.slots, inputs, outs), sess.home, args.steps,
+            if not args.rnn_tiles:
+                duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=20)
+            serial_s = base.schedule(duet.SERIAL)
+            base.home.wait_stream(torch.cuda.current_stream())
+            t_ser = bench.time_steps(torch, lambda: serial_s.run(base.slots, inputs, outs), base.home, args.steps,
                                      args.warmup, flush)
+            torch.cuda.synchronize()
             t_duet = bench.time_steps(torch, lambda: duet_s.run(sess.slots, inputs, outs), sess.home, args.steps,
                                       args.warmup, flush)
             prof = sess.prof.export()["t_ns"][:, 0].tolist()
@@ -70,10 +79,11 @@ def main():
                  "speedup_vs_serial": round(p50s / p50, 3), "samples_per_s": round(wl.batch / p50 * 1e3, 1),
                  "slot_of": e["slot_of"], "fell_back": e["fell_back"], "model_makespan_ms": e["makespan"] / 1e6,
                  "profile_ms": [round(v / 1e6, 4) for v in prof], "launches": duet_s.launch_count(),
+                 "rnn_tile_n": sess.wl.meta.get("rnn_tile_n"), "rnn_tile_measured_ns": tile_ns,
                  "wall_s": round(time.time() - t0, 1)}
             print(json.dumps({key: r}), flush=True)
             rows.append(r)
-            del sess, inputs, outs, duet_s, serial_s
+            del sess, base, inputs, outs, duet_s, serial_s
             torch.cuda.empty_cache()
         res[key] = {"title": title, "rows": rows}
     os.makedirs(os.path.dirname(os.path.abspath(args.out)), exist_ok=True)
