@@ -30,6 +30,9 @@ def launches(path):
 
 def main():
     tag, launch_csv, full_csv = sys.argv[1:4]
+    # optional: a substring of "<kernel> grid<grid>" keys that are not c2 step kernels (e.g. bench.py's
+    # secondary roofline launches at B = 65536), listed separately and left out of the step shares
+    exclude = sys.argv[4] if len(sys.argv) > 4 else None
     per = launches(launch_csv)
     # the last 3 timed steps: take the launches after the profiler/warm-up (last 3*7 of the bench graph)
     items = list(per.items())
@@ -43,6 +46,7 @@ def main():
         a["rd"] += m.get("dram__bytes_read.sum", 0.0)
         a["wr"] += m.get("dram__bytes_write.sum", 0.0)
     # share of one step: each kernel once (bench.py also launches fc1 alone for the roofline timing)
+    extra = collections.OrderedDict((k, agg.pop(k)) for k in list(agg) if exclude and exclude in k)
     tot = sum(a["ns"] / a["n"] for a in agg.values())
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     with open(os.path.join(ROOT, "profiles", f"{tag}_launches.md"), "w") as f:
@@ -54,6 +58,10 @@ def main():
             n = a["n"]
             unit = 1e-3 if a["ns"] / n > 1000 else 1.0  # ncu reports ns or us depending on version
             f.write(f"| {k} | {n} | {a['ns'] / n * (1e-3 if unit == 1e-3 else 1):.2f} | {a['ns'] / n / tot:.1%} | "
+                    f"{a['rd'] / n / 1e6:.2f} | {a['wr'] / n / 1e6:.2f} |\n")
+        for k, a in extra.items():
+            n = a["n"]
+            f.write(f"| {k} (not a step kernel: bench.py secondary roofline) | {n} | {a['ns'] / n * (1e-3 if a['ns'] / n > 1000 else 1):.2f} | - | "
                     f"{a['rd'] / n / 1e6:.2f} | {a['wr'] / n / 1e6:.2f} |\n")
     # full capture of the dominant kernel
     r = list(csv.reader(open(full_csv)))
