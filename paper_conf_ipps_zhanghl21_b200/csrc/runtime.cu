@@ -1060,6 +1060,7 @@ struct HostCopy {
   const void* src;
   size_t bytes;
   cudaMemcpyKind kind;
+  int node = -1;  // H2D: the input node it fills (its copy is issued before its first consumer)
 };
 
 static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<cudaStream_t>& streams,
@@ -1082,11 +1083,32 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
   std::vector<std::vector<int>> preds(n);
   for (auto& kv : part.edges)
     if (kv.first.first >= 0 && kv.first.second >= 0) preds[kv.first.second].push_back(kv.first.first);
+  // H2D copies of pinned-host inputs go on the stream of their first consuming subgraph, just
+  // before it, so a branch that does not read a large input (c4's GRU vs the 19 MB image) starts
+  // while that input is still crossing PCIe; other consumers on other streams wait on its event.
+  const Graph& G = *part.g;
+  std::vector<std::vector<int>> copies_of(n);  // subgraph -> indices into h2d it consumes
+  std::vector<char> early(h2d.size(), 1);
+  for (size_t c = 0; c < h2d.size(); ++c) {
+    if (h2d[c].node < 0) continue;
+    for (int s = 0; s < n; ++s)
+      for (int v : part.sg_nodes[s]) {
+        const auto& an = G.nodes[v].arg_nodes;
+        if (std::find(an.begin(), an.end(), h2d[c].node) != an.end()) {
+          copies_of[s].push_back((int)c);
+          early[c] = 0;
+          break;
+        }
+      }
+  }
+  std::vector<cudaEvent_t> copied(h2d.size(), nullptr);
+  std::vector<cudaStream_t> copied_on(h2d.size(), nullptr);
   int64_t nk = 0;
   CK(cudaStreamBeginCapture(home, cudaStreamCaptureModeRelaxed));
   try {
     // pinned-host inputs/outputs are memcpy nodes of the same graph: one launch per inference
-    for (auto& c : h2d) CK(cudaMemcpyAsync(c.dst, c.src, c.bytes, c.kind, home));
+    for (size_t c = 0; c < h2d.size(); ++c)
+      if (early[c]) CK(cudaMemcpyAsync(h2d[c].dst, h2d[c].src, h2d[c].bytes, h2d[c].kind, home));
     CK(cudaEventRecord(fork, home));
     std::vector<char> forked(streams.size(), 0);
     std::vector<int> last_on(streams.size(), -1);
@@ -1106,6 +1128,16 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
       }
       for (int u : preds[s])
         if (streams[S.slot_of[u]] != st) CK(cudaStreamWaitEvent(st, done[u], 0));
+      for (int c : copies_of[s]) {
+        if (!copied[c]) {
+          CK(cudaMemcpyAsync(h2d[c].dst, h2d[c].src, h2d[c].bytes, h2d[c].kind, st));
+          copied[c] = mk();
+          copied_on[c] = st;
+          CK(cudaEventRecord(copied[c], st));
+        } else if (copied_on[c] != st) {
+          CK(cudaStreamWaitEvent(st, copied[c], 0));
+        }
+      }
       launch_subgraph(P, part, s, T, st);
       nk += subgraph_kernels(P, part, s);
       CK(cudaEventRecord(done[s], st));
@@ -1223,7 +1255,7 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
     } else if (void* dp = direct_input_ptr(*g, nd, in[i].data)) {
       T[nd.id] = dp;  // zero-copy: its only consumer streams it once over PCIe
     } else {
-      h2d.push_back({P->buf[nd.id], in[i].data, (size_t)nd.nbytes(), cudaMemcpyHostToDevice});
+      h2d.push_back({P->buf[nd.id], in[i].data, (size_t)nd.nbytes(), cudaMemcpyHostToDevice, nd.id});
     }
   }
   for (int i = 0; i < n_out; ++i) {
