@@ -209,8 +209,9 @@ def greedy(m: Model):
     return a
 
 
-def correct(m: Model, a, p, rounds: int = 1):
-    """Step 3 (Algorithm 1) on multi-path phase p, in model mode."""
+def correct(m: Model, a, p, rounds: int = 1, trace=None):
+    """Step 3 (Algorithm 1) on multi-path phase p, in model mode.  `trace` (a list, optional)
+    receives one (M, kind, i, d-or-j, accepted) tuple per inner iteration, in order."""
     a = list(a)
     t_old = m.makespan(a)
     ph = m.phases[p]
@@ -242,6 +243,8 @@ def correct(m: Model, a, p, rounds: int = 1):
                 break
             t_new, kind, i, y = best
             U = [s for s in U if s != i and not (kind == 1 and s == y)]
+            if trace is not None:
+                trace.append((t_new, kind, i, y, t_new < t_old))
             if t_new < t_old:
                 if kind == 0:
                     a[i] = y
@@ -267,7 +270,7 @@ def lowbias32(x: int) -> int:
 
 
 def schedule(part: Partition, T, slot_gpu, comm: Comm, mode: int = 0, correction_rounds: int = 1,
-             allow_fallback: bool = True, fixed=None, seed: int = 0) -> Schedule:
+             allow_fallback: bool = True, fixed=None, seed: int = 0, trace=None) -> Schedule:
     """mode 0 greedy-correction, 1 greedy only, 2 serial (home slot 0), 3 fixed; Fig. 13
     baselines: 4 random, 5 round-robin, 6 random + correction."""
     m = Model(part, T, slot_gpu, comm)
@@ -287,7 +290,7 @@ def schedule(part: Partition, T, slot_gpu, comm: Comm, mode: int = 0, correction
         if mode in (0, 6):
             for p in range(part.n_phase):
                 if part.phase_kind[p] == MULTI:
-                    a = correct(m, a, p, correction_rounds)
+                    a = correct(m, a, p, correction_rounds, trace)
         if allow_fallback:
             m_gc = m.makespan(a)
             singles = [(m.makespan([d] * n), d) for d in range(m.D)]
@@ -307,3 +310,54 @@ def brute_force(part: Partition, T, slot_gpu, comm: Comm):
         if best is None or ms < best[0]:
             best = (ms, list(a))
     return best
+
+
+def brute_force_symmetric(part: Partition, T, slot_gpu, comm: Comm):
+    """C5 for D interchangeable non-home slots (8 identical GPUs x 1 stream
+    over NVSwitch).  Only canonical assignments are evaluated: set partitions of the subgraphs
+    with one distinguished home block (slot 0, where graph inputs live and outputs must return,
+    C3) and at most D-1 unlabeled non-home blocks, labeled 1, 2, ... in order of first use
+    (restricted growth strings).  Valid only when relabeling slots 1..D-1 changes no cost: every
+    subgraph has equal T on those slots and they are all on distinct GPUs other than slot 0's, or
+    all on slot 0's GPU.  Returns (min makespan, first canonical assignment reaching it)."""
+    m = Model(part, T, slot_gpu, comm)
+    D, n = m.D, part.n_sg
+    for row in m.T:
+        if any(row[d] != row[1] for d in range(2, D)):
+            raise ValueError("non-home slots must have identical costs")
+    rest = m.slot_gpu[1:]
+    if not (all(g == m.slot_gpu[0] for g in rest)
+            or (len(set(rest)) == len(rest) and m.slot_gpu[0] not in rest)):
+        raise ValueError("non-home slots must all share slot 0's GPU or all sit on distinct other GPUs")
+    best = None
+    a = [0] * n
+
+    def rec(s, used):
+        nonlocal best
+        if s == n:
+            ms = m.makespan(a)
+            if best is None or ms < best[0]:
+                best = (ms, list(a))
+            return
+        for d in range(0, min(used + 1, D - 1) + 1):
+            a[s] = d
+            rec(s + 1, max(used, d))
+
+    rec(0, 0)
+    return best
+
+
+def canonical_count(n: int, D: int) -> int:
+    """Number of assignments brute_force_symmetric evaluates (the enumeration alone)."""
+    cnt = 0
+
+    def rec(s, used):
+        nonlocal cnt
+        if s == n:
+            cnt += 1
+            return
+        for d in range(0, min(used + 1, D - 1) + 1):
+            rec(s + 1, max(used, d))
+
+    rec(0, 0)
+    return cnt

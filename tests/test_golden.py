@@ -86,3 +86,49 @@ def test_toy_mlp_golden(dt):
     out = F.run(TOY.format(dt=dt), params, {"x": enc(g["x"], (1, 2))}, keep_all=True)
     np.testing.assert_array_equal(np.asarray(out["h"], dtype=np.float64).ravel(), g["expect_h"])
     assert out["y"][0, 0] == pytest.approx(g["expect_y"][0], rel=1e-15)
+
+
+def fig8_ir():
+    """The constructed Fig. 8 graph (tests/golden/fig8_swap.txt): head, branches b1..b6 (subgraph
+    ids 1..6 = the figure's), join; b6's output is 2000 B, every other tensor 4 B."""
+    lines = ["%x = input() : f32[1]", "%h = opaque(%x) : f32[1]"]
+    lines += [f"%b{k} = opaque(%h) : f32[{500 if k == 6 else 1}]" for k in range(1, 7)]
+    lines += ["%j = opaque(" + ", ".join(f"%b{k}" for k in range(1, 7)) + ") : f32[1]", "output %j"]
+    return "\n".join(lines) + "\n"
+
+
+def test_fig8_swap_golden():
+    """PAPER.md:81 §IV-C Step 3 / Fig. 8: initial GPU = {1,3,6}, CPU = {2,4,5}; the first accepted
+    correction is the pair (6, 5), avoiding b6's large output crossing devices."""
+    from oracle.schedule import Model
+    g = load("fig8_swap.txt")
+    ir = fig8_ir()
+    p = partition(ir)
+    assert p.n_sg == 8 and p.sg_phase == [0, 1, 1, 1, 1, 1, 1, 2]
+    assert p.edges[(6, 7)] == 2000 and p.edges[(5, 7)] == 4
+    T, slot_gpu = g["t_ns"], g["slot_gpu"]
+    comm = Comm(Link(0, 0), Link(g["comm_cross_alpha_ns"][0], g["comm_cross_ps_per_byte"][0]))
+    gr = schedule(p, T, slot_gpu, comm, mode=1, allow_fallback=False)
+    assert gr.slot_of == g["expect_greedy_slot_of"] and gr.makespan == g["expect_greedy_makespan_ns"][0]
+    gpu = {s for s in range(1, 7) if gr.slot_of[s] == 1}
+    cpu = {s for s in range(1, 7) if gr.slot_of[s] == 0}
+    assert gpu == {1, 3, 6} and cpu == {2, 4, 5}
+    trace = []
+    s = schedule(p, T, slot_gpu, comm, trace=trace)
+    m_first, kind, i, j, accepted = trace[0]
+    assert [m_first, kind, i, j] == g["expect_first_correction"] and accepted
+    assert [t for t in trace[1:] if t[4]] == []           # nothing else accepted
+    assert s.slot_of == g["expect_slot_of"] and s.makespan == g["expect_makespan_ns"][0]
+    assert s.fell_back == g["expect_fell_back"][0]
+    m = Model(p, T, slot_gpu, comm)
+    assert m.critical_path_lb() == g["expect_critical_path_lb_ns"][0]
+    assert [m.makespan([d] * 8) for d in (0, 1)] == g["expect_single_slot_ns"]
+    assert brute_force(p, T, slot_gpu, comm)[0] <= s.makespan
+    # the C++ scheduler through the C ABI
+    dp = duet.Graph(ir).partition()
+    cm = ((0, 0), (g["comm_cross_alpha_ns"][0], g["comm_cross_ps_per_byte"][0]))
+    pr = dp.profile_from_table(slot_gpu, T, comm=cm)
+    e = pr.schedule(mode=duet.GREEDY_ONLY, allow_fallback=False).export()
+    assert e["slot_of"] == g["expect_greedy_slot_of"]
+    e = pr.schedule().export()
+    assert e["slot_of"] == g["expect_slot_of"] and e["makespan"] == g["expect_makespan_ns"][0]

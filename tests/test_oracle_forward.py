@@ -345,3 +345,33 @@ def test_mtdnn_layer_vs_torch_encoder_layer():
     np.testing.assert_allclose(vals["L0_ln2"], want.reshape(B * S, H).numpy(), rtol=1e-10, atol=1e-10)
     # [CLS] rows feed the task heads
     np.testing.assert_allclose(vals["cls"], vals["L1_ln2"][::S])
+
+
+def test_reduce_sum_closed_form():
+    """c1/c2 wide part 'wide = reduce_sum(gathered weights) + b0' (Cheng et al.'s
+    wide model): row sums of integer rows.  Row r = [r, r+1, ..., r+F-1] sums to F*r + F(F-1)/2;
+    through the IR as well (op dispatch, bias parameter, [B, 1] shape)."""
+    B, F_ = 5, 26
+    x = np.arange(B)[:, None] + np.arange(F_)[None, :]
+    got = F.reduce_sum(x.astype(np.float64), np.array([0.5]))
+    assert got.shape == (B, 1)
+    assert got[:, 0].tolist() == [F_ * r + F_ * (F_ - 1) / 2 + 0.5 for r in range(B)]
+    ir = f"param @b : f32[1]\n%x = input() : f32[{B},{F_}]\n%y = reduce_sum(%x, @b) : f32[{B},1]\noutput %y\n"
+    y = F.run(ir, {"b": np.array([-3.0], np.float32)}, {"x": x.astype(np.float32)})["y"]
+    assert y[:, 0].tolist() == [F_ * r + 325 - 3 for r in range(B)]
+
+
+def test_select_rows_closed_form():
+    """MT-DNN's [CLS] select (Fig. 3; R-31): rows offset, offset + S, ... of a
+    [B*S, H] activation.  With x[i, k] = 1000 i + k the selected row b is 1000 (b S + offset) + k."""
+    B, S, H = 3, 7, 4
+    x = 1000.0 * np.arange(B * S)[:, None] + np.arange(H)[None, :]
+    for off in (0, 2, S - 1):
+        got = F.select_rows(x, S, off)
+        assert got.shape == (B, H)
+        want = [[1000 * (b * S + off) + k for k in range(H)] for b in range(B)]
+        assert got.tolist() == want
+    ir = (f"%x = input() : f32[{B * S},{H}]\n%c = select_rows(%x) {{stride={S}, offset=1}} : f32[{B},{H}]\n"
+          "output %c\n")
+    y = F.run(ir, {}, {"x": x.astype(np.float32)})["c"]
+    assert y[:, 0].tolist() == [1000 * (b * S + 1) for b in range(B)]

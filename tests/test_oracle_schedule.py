@@ -254,3 +254,134 @@ def test_fig13_baselines_definitions():
     gc = schedule(p, T, [0, 1], ZERO, mode=0, allow_fallback=False)
     assert gc.makespan <= g.makespan
     assert gc.makespan >= brute_force(p, T, [0, 1], ZERO)[0]
+
+
+# ---- Step 1's intra-phase critical path at op granularity (hand-traced) ---------------------------
+CHAIN_IR = """%x = input() : f32[1]
+%a = opaque(%x) : f32[1]
+%l = opaque(%a) : f32[1]
+%r0 = opaque(%a) : f32[1]
+%r1a = opaque(%r0) : f32[1]
+%r1b = opaque(%r0) : f32[1]
+%r2 = opaque(%r1a, %r1b) : f32[1]
+%r3 = opaque(%r2) : f32[1]
+%j = opaque(%l, %r3) : f32[1]
+output %j
+"""
+#           a      l      r0     r1a    r1b    r2     r3     j      (sg ids 0..7 = topological order)
+CHAIN_T = [[1000, 1000], [6000, 6000], [3000, 1000], [1000, 2000], [4000, 2000], [9000, 7000],
+           [2000, 1000], [1000, 1000]]
+
+
+def test_phase_chain_op_granularity():
+    """PAPER.md:81 Step 1 "add the subgraph that has maximum cost in that phase to the critical path"
+    (with intra-phase edges, the longest chain through s* by cost).  Hand trace:
+    cost = min_d T: l 6000, r0 1000, r1a 1000, r1b 2000, r2 7000, r3 1000 -> s* = r2 (sg 5).
+    Backwards r2's in-phase preds are r1a (dp_in 1000 + 1000 = 2000) and r1b (2000 + 1000 = 3000)
+    -> r1b, then r0; forwards r3.  Chain {r0, r1b, r2, r3} = sgs {2, 4, 5, 6}, each on its argmin
+    slot (slot 1).  Step 2 (Kahn, cost desc): l: slot 0 keeps the phase end at 12000 (d 0) vs 18000
+    on slot 1 -> slot 0; r1a: slot 0 delays r2 (phase end 16000, d 4000) vs slot 1 (14000, d 2000)
+    -> slot 1.  A chain that took r1a instead of r1b would put r1a on its argmin slot 0; a chain of
+    s* alone would leave r0/r1b/r3 to Step 2."""
+    from oracle.schedule import _phase_chain, greedy
+    p = partition(CHAIN_IR, "op")
+    assert p.n_sg == 8 and p.sg_phase == [0, 1, 1, 1, 1, 1, 1, 2] and p.phase_kind == [SEQ, MULTI, SEQ]
+    m = Model(p, CHAIN_T, [0, 0], ZERO)
+    cost = {s: min(CHAIN_T[s]) for s in m.phases[1]}
+    assert _phase_chain(m, 1, cost) == [2, 4, 5, 6]
+    assert greedy(m) == [0, 0, 1, 1, 1, 1, 1, 0]
+    g = schedule(p, CHAIN_T, [0, 0], ZERO, mode=1, allow_fallback=False)
+    assert g.makespan == 1000 + 13000 + 1000
+    # exact lower bounds (a -> r0 -> r1b -> r2 -> r3 -> j by min cost)
+    assert m.critical_path_lb() == 1000 + 1000 + 2000 + 7000 + 1000 + 1000
+    assert m.phase_cp_sum() == 1000 + 11000 + 1000
+    # the C++ scheduler agrees
+    from paper_conf_ipps_zhanghl21_b200 import duet
+    pr = duet.Graph(CHAIN_IR).partition("op").profile_from_table([0, 0], CHAIN_T)
+    assert pr.schedule(mode=duet.GREEDY_ONLY, allow_fallback=False).export()["slot_of"] == [0, 0, 1, 1, 1, 1, 1, 0]
+
+
+def test_critical_path_exact_values():
+    """C3's lower bounds as exact numbers on the diamond (not only the inequality chain): paths
+    a -> l -> j and a -> r1 -> r2 -> j with min-cost weights."""
+    ir = """%x = input() : f32[2,4]
+%a = opaque(%x) : f32[2,4]
+%l = opaque(%a) : f32[2,8]
+%r1 = opaque(%a) : f32[2,2]
+%r2 = opaque(%r1) : f32[2,2]
+%j = opaque(%l, %r2) : f32[2,1]
+output %j
+"""
+    p = partition(ir, "op")
+    T = [[500, 700], [9000, 4000], [3000, 2500], [1500, 2000], [100, 100]]
+    m = Model(p, T, [0, 0], ZERO)
+    assert m.critical_path_lb() == 500 + max(4000, 2500 + 1500) + 100
+    T2 = [[500, 700], [3000, 4000], [3000, 2500], [1500, 2000], [100, 100]]
+    assert Model(p, T2, [0, 0], ZERO).critical_path_lb() == 500 + 2500 + 1500 + 100
+    assert Model(p, T2, [0, 0], ZERO).phase_cp_sum() == 500 + 4000 + 100
+
+
+# ---- C5 symmetry-reduced brute force (D = 8 identical GPUs) ---------------------------------------
+def _stirling2(n, k):
+    S = [[0] * (k + 1) for _ in range(n + 1)]
+    S[0][0] = 1
+    for i in range(1, n + 1):
+        for j in range(1, k + 1):
+            S[i][j] = j * S[i - 1][j] + S[i - 1][j - 1]
+    return S[n][k]
+
+
+@pytest.mark.parametrize("n,D", [(3, 2), (5, 4), (10, 8), (10, 11)])
+def test_canonical_count(n, D):
+    """Canonical assignments = sum_j C(n, j) * sum_{i < D} S2(n - j, i) (j subgraphs at home, the
+    rest in at most D - 1 unlabeled blocks); with D > n this is Bell(n + 1) (678,570 at n = 10)."""
+    from math import comb
+
+    from oracle.schedule import canonical_count
+    want = sum(comb(n, j) * sum(_stirling2(n - j, i) for i in range(D)) for j in range(n + 1))
+    assert canonical_count(n, D) == want
+    if D > n:
+        assert want == {3: 15, 10: 678570}[n]
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_symmetric_brute_force_equals_full(seed):
+    """Symmetry reduction is exact: on fuzzed DAGs with identical non-home slots (D <= 4 distinct
+    GPUs, or stream slots of one GPU) its optimum equals the plain D^n enumeration."""
+    from oracle.schedule import brute_force_symmetric
+    rng = random.Random(100 + seed)
+    ir = random_dag_ir(rng, rng.randint(3, 7))
+    p = partition(ir, "op" if seed % 2 else "coarse")
+    D = 3 if p.n_sg > 6 else 4
+    slot_gpu = list(range(D)) if seed % 3 else [0] * D
+    T = []
+    for _ in range(p.n_sg):
+        h, o = rng.randint(1, 40) * 1000, rng.randint(1, 40) * 1000
+        T.append([h] + [o] * (D - 1))
+    comm = Comm(Link(rng.randint(0, 3000), rng.randint(0, 3)), Link(rng.randint(0, 9000), rng.randint(0, 900)))
+    ms, a = brute_force_symmetric(p, T, slot_gpu, comm)
+    full = brute_force(p, T, slot_gpu, comm)
+    assert ms == full[0]
+    assert Model(p, T, slot_gpu, comm).makespan(a) == ms
+
+
+def test_symmetric_brute_force_d8():
+    """D = 8 identical GPUs x 1 stream (the 8xB200 box): the 'Ideal' exists and bounds greedy-correction;
+    on 5 subgraphs it equals the full 8^5 enumeration."""
+    from oracle.schedule import brute_force_symmetric
+    p = partition(branches_ir(4, join=True))          # 5 subgraphs
+    T = [[t] * 8 for t in (9000, 7000, 6000, 5000, 300)]
+    comm = Comm(Link(0, 0), Link(2000, 10))
+    slot_gpu = list(range(8))
+    ms, a = brute_force_symmetric(p, T, slot_gpu, comm)
+    assert ms == brute_force(p, T, slot_gpu, comm)[0]
+    # hand check: a remote branch pays 2000 + ceil(64 B * 10 / 1000) = 2001 in and 2001 out.  The
+    # 9000 branch stays home (0-9000), the others each on their own GPU (the 7000 one ends at 9001,
+    # reaches the join at 11002), join 11002-11302.  Sending the 9000 branch away costs 13302;
+    # doubling up any two branches on one slot costs >= 14000.
+    assert (ms, a) == (11302, [0, 1, 2, 3, 0])
+    s = schedule(p, T, slot_gpu, comm)
+    assert ms <= s.makespan
+    p10 = partition(branches_ir(9, join=True))         # 10 subgraphs, ~677K canonical assignments
+    with pytest.raises(ValueError):
+        brute_force_symmetric(p10, [[1, 1, 2] + [1] * 5] * 10, slot_gpu, comm)
