@@ -35,6 +35,16 @@ def to_f64(a, dtype: str) -> np.ndarray:
     raise ValueError(dtype)
 
 
+def round_bf16(x) -> np.ndarray:
+    """float64 -> nearest bf16 value (via float32, round-to-nearest-even on the upper 16 bits).
+    Used only by run(..., round_storage=True): the diagnostic reading of DESIGN.md R-26 in which
+    every bf16-declared node output is stored rounded, as the GPU stores it."""
+    f = np.asarray(x, dtype=np.float64).astype(np.float32)
+    b = f.view(np.uint32)
+    b = (b + np.uint32(0x7FFF) + ((b >> np.uint32(16)) & np.uint32(1))) & np.uint32(0xFFFF0000)
+    return b.view(np.float32).astype(np.float64)
+
+
 def sigmoid(x):
     # 1 / (1 + e^-x), written to avoid overflow warnings for large |x|
     out = np.empty_like(x, dtype=np.float64)
@@ -279,10 +289,13 @@ def select_rows(x, stride, offset=0):
 
 
 # ---- graph evaluation -----------------------------------------------------------------------
-def run(ir, params: dict, inputs: dict, keep_all: bool = False) -> dict:
+def run(ir, params: dict, inputs: dict, keep_all: bool = False, round_storage: bool = False) -> dict:
     """Evaluate the graph in topological order.  Returns {output name: float64 array}
     (or every node value if keep_all).  Shapes come from the arrays, not the IR, so a batch
-    subset of the inputs evaluates exactly those rows (inference rows are independent)."""
+    subset of the inputs evaluates exactly those rows (inference rows are independent).
+    round_storage: round every bf16-declared node output to bf16 (the R-26 storage reading; a
+    diagnostic that separates activation-storage rounding from kernel error -- the parity bar
+    is always against the unrounded pass)."""
     g: Graph = parse(ir) if isinstance(ir, str) else ir
     val = {}
 
@@ -350,6 +363,8 @@ def run(ir, params: dict, inputs: dict, keep_all: bool = False) -> dict:
             v = select_rows(A[0], int(at["stride"]), int(at.get("offset", 0)))
         else:
             raise ValueError(f"oracle has no operator {op!r}")
+        if round_storage and n.dtype == "bf16" and op != "input":
+            v = round_bf16(v)
         val[n.name] = v
     if keep_all:
         return val

@@ -113,12 +113,11 @@ def partition(ir, granularity: str = "coarse") -> Partition:
     S, T = N, N + 1
     fwd = [list(s) for s in succs] + [[], []]
     bwd = [list(p) for p in preds] + [[], []]
-    outs = set(g.outputs)
     for v in range(N):
         if not preds[v]:
             fwd[S].append(v)
             bwd[v].append(S)
-        if not succs[v] or (v < n0 and v in outs):
+        if not succs[v]:        # only sinks; outputs with consumers keep just their boundary edge
             fwd[v].append(T)
             bwd[T].append(v)
     seps = [v for v in range(N) if not _reach(S, fwd, N + 2, blocked=v)[T]]

@@ -90,7 +90,6 @@ Partition* make_partition(const Graph* g, int granularity) {
   // step 2: virtual source S = N, sink T = N+1; separators
   const int S = N, T = N + 1;
   std::vector<std::vector<int>> fwd(N + 2), bwd(N + 2);
-  std::set<int> outs(g->outputs.begin(), g->outputs.end());
   for (int v = 0; v < N; ++v) {
     fwd[v] = succs[v];
     bwd[v] = preds[v];
@@ -100,7 +99,10 @@ Partition* make_partition(const Graph* g, int granularity) {
       fwd[S].push_back(v);
       bwd[v].push_back(S);
     }
-    if (succs[v].empty() || (v < n0 && outs.count(v))) {
+    // only nodes without successors reach the sink: an output that also feeds other nodes keeps
+    // its boundary edge (step 6) but must not bypass the join, or the join would stop being a
+    // separator and every branch concurrency behind it would be lost
+    if (succs[v].empty()) {
       fwd[v].push_back(T);
       bwd[T].push_back(v);
     }

@@ -1060,7 +1060,7 @@ struct HostCopy {
   const void* src;
   size_t bytes;
   cudaMemcpyKind kind;
-  int node = -1;  // H2D: the input node it fills (its copy is issued before its first consumer)
+  int node = -1;  // H2D: the input node it fills (its consumers wait on the copy's event)
 };
 
 static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<cudaStream_t>& streams,
@@ -1083,12 +1083,12 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
   std::vector<std::vector<int>> preds(n);
   for (auto& kv : part.edges)
     if (kv.first.first >= 0 && kv.first.second >= 0) preds[kv.first.second].push_back(kv.first.first);
-  // H2D copies of pinned-host inputs go on the stream of their first consuming subgraph, just
-  // before it, so a branch that does not read a large input (c4's GRU vs the 19 MB image) starts
-  // while that input is still crossing PCIe; other consumers on other streams wait on its event.
+  // H2D copies of pinned-host inputs start at the fork, each on its own side stream (one memcpy
+  // node + one event per input), so every copy overlaps all branch compute from t = 0 and a small
+  // input never queues behind a large one (c4's token ids vs its 19 MB image); each consuming
+  // subgraph waits only on the events of the inputs it reads.
   const Graph& G = *part.g;
   std::vector<std::vector<int>> copies_of(n);  // subgraph -> indices into h2d it consumes
-  std::vector<char> early(h2d.size(), 1);
   for (size_t c = 0; c < h2d.size(); ++c) {
     if (h2d[c].node < 0) continue;
     for (int s = 0; s < n; ++s)
@@ -1096,20 +1096,28 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
         const auto& an = G.nodes[v].arg_nodes;
         if (std::find(an.begin(), an.end(), h2d[c].node) != an.end()) {
           copies_of[s].push_back((int)c);
-          early[c] = 0;
           break;
         }
       }
   }
   std::vector<cudaEvent_t> copied(h2d.size(), nullptr);
-  std::vector<cudaStream_t> copied_on(h2d.size(), nullptr);
+  std::vector<cudaStream_t> side(h2d.size(), nullptr);
+  for (auto& st : side) CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+  auto free_side = [&]() {
+    for (auto st : side)
+      if (st) cudaStreamDestroy(st);
+  };
   int64_t nk = 0;
   CK(cudaStreamBeginCapture(home, cudaStreamCaptureModeRelaxed));
   try {
-    // pinned-host inputs/outputs are memcpy nodes of the same graph: one launch per inference
-    for (size_t c = 0; c < h2d.size(); ++c)
-      if (early[c]) CK(cudaMemcpyAsync(h2d[c].dst, h2d[c].src, h2d[c].bytes, h2d[c].kind, home));
     CK(cudaEventRecord(fork, home));
+    // pinned-host inputs/outputs are memcpy nodes of the same graph: one launch per inference
+    for (size_t c = 0; c < h2d.size(); ++c) {
+      CK(cudaStreamWaitEvent(side[c], fork, 0));
+      CK(cudaMemcpyAsync(h2d[c].dst, h2d[c].src, h2d[c].bytes, h2d[c].kind, side[c]));
+      copied[c] = mk();
+      CK(cudaEventRecord(copied[c], side[c]));
+    }
     std::vector<char> forked(streams.size(), 0);
     std::vector<int> last_on(streams.size(), -1);
     for (int s : S.order) {
@@ -1128,16 +1136,7 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
       }
       for (int u : preds[s])
         if (streams[S.slot_of[u]] != st) CK(cudaStreamWaitEvent(st, done[u], 0));
-      for (int c : copies_of[s]) {
-        if (!copied[c]) {
-          CK(cudaMemcpyAsync(h2d[c].dst, h2d[c].src, h2d[c].bytes, h2d[c].kind, st));
-          copied[c] = mk();
-          copied_on[c] = st;
-          CK(cudaEventRecord(copied[c], st));
-        } else if (copied_on[c] != st) {
-          CK(cudaStreamWaitEvent(st, copied[c], 0));
-        }
-      }
+      for (int c : copies_of[s]) CK(cudaStreamWaitEvent(st, copied[c], 0));
       launch_subgraph(P, part, s, T, st);
       nk += subgraph_kernels(P, part, s);
       CK(cudaEventRecord(done[s], st));
@@ -1145,6 +1144,7 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
     }
     for (size_t q = 0; q < streams.size(); ++q)
       if (last_on[q] >= 0 && streams[q] != home) CK(cudaStreamWaitEvent(home, done[last_on[q]], 0));
+    for (auto ev : copied) CK(cudaStreamWaitEvent(home, ev, 0));  // joins every side stream
     for (auto& c : d2h) CK(cudaMemcpyAsync(c.dst, c.src, c.bytes, c.kind, home));
   } catch (...) {
     cudaGraph_t junk = nullptr;
@@ -1152,9 +1152,11 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
     if (junk) cudaGraphDestroy(junk);
     cudaGetLastError();
     for (auto ev : E.events) cudaEventDestroy(ev);
+    free_side();
     throw;
   }
   CK(cudaStreamEndCapture(home, &E.graph));
+  free_side();
   static const bool log = getenv("DUET_MEASURE_LOG") != nullptr;
   auto t_inst = std::chrono::steady_clock::now();
   // per-node priorities: kernels captured from a higher-priority slot stream keep it inside the

@@ -158,6 +158,12 @@ class _Builder:
         ho, wo = (h + 2 - 3) // 2 + 1, (w + 2 - 3) // 2 + 1
         c = self.node(f"{prefix}_pool", "maxpool", [c], self.dt, (n, ho, wo, 64), k=3, stride=2, pad=1)
         h, w, cin = ho, wo, 64
+        # depth-scaled residual-branch gamma (R-28): the residual stream's variance grows
+        # with the number of blocks L, so the branch scale goes with sqrt(8 / L) (8 = ResNet-18's L,
+        # unchanged there; the 1/sqrt(L) residual scaling of Fixup / SkipInit) and the pooled
+        # features stay O(1) at every depth, as in a trained network
+        rs = math.sqrt(8.0 / sum(blocks))
+        rg = (0.1 * rs, 0.3 * rs)
         for li, width in enumerate([64, 128, 256, 512]):
             cout = width * exp
             for bi in range(blocks[li]):
@@ -169,12 +175,12 @@ class _Builder:
                 if kind == "basic":
                     y, h2, w2 = self.conv_bn(nm + "_c1", c, n, h, w, cin, cout, 3, stride, 1, "relu")
                     y, h2, w2 = self.conv_bn(nm + "_c2", y, n, h2, w2, cout, cout, 3, 1, 1, "none",
-                                             gamma=(0.1, 0.3))
+                                             gamma=rg)
                 else:
                     y, _, _ = self.conv_bn(nm + "_c1", c, n, h, w, cin, width, 1, 1, 0, "relu")
                     y, h2, w2 = self.conv_bn(nm + "_c2", y, n, h, w, width, width, 3, stride, 1, "relu")
                     y, h2, w2 = self.conv_bn(nm + "_c3", y, n, h2, w2, width, cout, 1, 1, 0, "none",
-                                             gamma=(0.1, 0.3))
+                                             gamma=rg)
                 if stride != 1 or cin != cout:
                     sc, _, _ = self.conv_bn(nm + "_ds", c, n, h, w, cin, cout, 1, stride, 0, "none")
                 else:

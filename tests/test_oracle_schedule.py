@@ -385,3 +385,19 @@ def test_symmetric_brute_force_d8():
     p10 = partition(branches_ir(9, join=True))         # 10 subgraphs, ~677K canonical assignments
     with pytest.raises(ValueError):
         brute_force_symmetric(p10, [[1, 1, 2] + [1] * 5] * 10, slot_gpu, comm)
+
+
+@pytest.mark.parametrize("cfg", ["c1", "c2", "c3", "c4", "c5", "c6"])
+def test_branch_outputs_do_not_change_partition(cfg):
+    """Exposing intermediate tensors as graph outputs (branch outputs, multi-task heads) adds
+    boundary edges only: the join stays a separator, so n_sg, sg_phase and the phase kinds are
+    those of the plain graph (only nodes without successors connect to C2's virtual sink)."""
+    from paper_conf_ipps_zhanghl21_b200 import duet
+    wl = W.build(cfg, small=True)
+    wb = W.build(cfg, small=True, branch_outputs=True)
+    for gran in ("coarse", "op"):
+        p, q = partition(wl.ir, gran), partition(wb.ir, gran)
+        assert (q.n_sg, q.sg_phase, q.phase_kind, q.node_to_sg) == (p.n_sg, p.sg_phase, p.phase_kind, p.node_to_sg)
+        assert set(p.edges) <= set(q.edges)
+        e = duet.Graph(wb.ir).partition(gran).export()
+        assert e["node_to_sg"] == q.node_to_sg and e["edges"] == q.edges

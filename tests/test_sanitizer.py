@@ -1,0 +1,28 @@
+"""compute-sanitizer over the hand-synchronised kernels (SURVEY.md §4/§5 race detection):
+memcheck (out-of-bounds / misaligned accesses), racecheck (shared-memory hazards) and synccheck
+(barrier misuse) on small launches of every tcgen05/TMA kernel family and a two-slot schedule
+(tools/sanitize_nodes.py).  Only libduet's kernels are instrumented (kernel-name filter)."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+def test_compute_sanitizer(tool):
+    cmd = [SAN, "--tool", tool, "--kernel-name", "kns=duet", "--error-exitcode", "99",
+           sys.executable, os.path.join(ROOT, "tools", "sanitize_nodes.py")]
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900)
+    out = r.stdout + r.stderr
+    print(out[-3000:])
+    assert r.returncode == 0, out[-4000:]
+    assert "ERROR SUMMARY: 0 errors" in out, out[-4000:]
+    for k in ("gemm", "rnn", "conv", "stem", "c2"):
+        assert f"{k} ok" in out
