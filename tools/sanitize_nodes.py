@@ -42,7 +42,7 @@ def main():
              {"Wih": r(3 * H, E, sc=H ** -0.5), "Whh": r(3 * H, H, sc=H ** -0.5), "bih": torch.zeros(3 * H),
               "bhh": torch.zeros(3 * H)}, [r(S, B, E)], (B, H))
         print("rnn ok", flush=True)
-    for key, (N_, H_, C, Co, k, s, p) in (("conv", (2, 14, 14, 64, 64, 3, 1, 1)), ("stem", (1, 64, 64, 3, 64, 7, 2, 3))):
+    for key, (N_, H_, C, Co, k, s, p) in (("conv", (2, 14, 64, 64, 3, 1, 1)), ("stem", (1, 64, 3, 64, 7, 2, 3))):
         if key not in which:
             continue
         Ho, Wo = (H_ + 2 * p - k) // s + 1, (H_ + 2 * p - k) // s + 1
