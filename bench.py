@@ -1,21 +1,28 @@
 """DUET on B200 — benchmark (driver contract: one JSON line on rank 0).
 
-Workload: BASELINE.json configs[1] (c2, wide&deep recommender, 26 tables x 64, MLP 1024-512-256,
-batch 2048) unless --config says otherwise.  A *step* = one inference of one batch through the
-whole hot path (hash -> {wide gather-sum || deep gather-concat -> 3 tcgen05 GEMMs} -> join),
-executed by libduet's greedy-correction schedule on CUDA-stream slots (one CUDA-graph replay).
+Headline workload: BASELINE.json configs[4] (c5, the 8-way heterogeneous ensemble, batch 4096), the
+largest configuration that fits one GPU; `per_config` adds c1-c4 (configs[0..3]) measured the same
+way in the same run (BASELINE.json:2 "per model").  A *step* = one inference of one batch through
+the whole hot path, executed by libduet's greedy-correction schedule on CUDA-stream slots (one
+CUDA-graph replay).
 
-  value        whole-job samples/s with inputs resident in HBM (N ranks x batch x K / max-rank time)
-  e2e          same, through duet_run with pinned HOST buffers (H2D + D2H inside the timed step)
-  p50/p99      per-step latency (CUDA events on the home stream, L2 flushed between steps)
+  value        whole-job samples/s with inputs resident in HBM (batch x K / max-rank time)
+  e2e          same, through duet_run with pinned HOST buffers (H2D + D2H inside the timed step);
+               also its host wall clock (duet_run + stream sync) per step
+  p50/p99      per-step latency (CUDA events on the home stream, L2 flushed between steps); p99 /
+               p99.9 from a separate tail pass of --tail-samples steps
   speedup      p50(serial 1-stream, same kernels) / p50(DUET)           (BASELINE.json:2)
-  roofline     dominant kernel, timed live with CUDA events on its stream
-  cpu_baseline float64 oracle on a bounded row sample (rank 0, N = 1)
+  roofline     dominant kernel, timed live and cold (L2 flushed before every launch; CUDA events
+               captured around the launch on its stream)
+  cpu_baseline float64 oracle on a bounded row sample (rank 0, N = 1), all host cores and 1 thread
 
-Multi-GPU (torchrun): one process per GPU, each runs its own batch (weak scaling, no data-path
-collective — inference rows are independent).  `--placement branch`
-instead runs ONE batch with its subgraphs placed on the GPUs by greedy-correction over one slot
-per GPU, cut-edge tensors over NCCL point-to-point (strong scaling; multigpu.py).
+Multi-GPU (torchrun, one process per GPU):
+  --placement shard (default for N > 1): ONE global batch per step, rows scattered from rank 0
+      over NCCL, every rank runs its row block through its own schedule, outputs gathered back to
+      rank 0 inside the timed step (strong scaling; multirank.ShardExecutor).
+  --placement replica: every rank runs its own full batch (weak scaling, no data-path collective).
+  --placement branch: ONE batch, subgraphs placed on the GPUs by greedy-correction over one slot
+      per GPU with a measured NVLink comm model, cut edges over NCCL point-to-point (multigpu.py).
 `--impl reference` times the oracle (the reference arm of this tier) on the host cores.
 """
 from __future__ import annotations
@@ -23,6 +30,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import re
 import statistics
 import sys
 import threading
@@ -33,6 +41,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "p50 inference latency (ms) & samples/sec per model; speedup vs serial 1-stream"
 L2_FLUSH_BYTES = 512 << 20  # > 126 MB L2
+BASELINE_IDX = {"c1": 0, "c2": 1, "c3": 2, "c4": 3, "c5": 4}
 
 
 def parse():
@@ -41,8 +50,11 @@ def parse():
     ap.add_argument("--steps", type=int, default=300)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="duet", choices=["duet", "reference"])
-    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5", "c6"],
+    ap.add_argument("--config", default="c5", choices=["c1", "c2", "c3", "c4", "c5", "c6"],
                     help="c1-c5 = BASELINE.json configs[0..4]; c6 = MT-DNN (SURVEY.md §8(f) N4(b), not a BASELINE config)")
+    ap.add_argument("--per-config", default="auto",
+                    help="comma list of extra configs measured in the same run ('auto': c1-c4 beside a c5 headline "
+                         "at N = 1; 'none')")
     ap.add_argument("--slots", type=int, default=2, help="CUDA-stream slots on the GPU")
     ap.add_argument("--dtype", default=None, choices=[None, "bf16", "f32"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -50,13 +62,14 @@ def parse():
     ap.add_argument("--ref-seconds", type=float, default=90.0,
                     help="--impl reference: timed oracle seconds over the whole --steps K --warmup W run")
     ap.add_argument("--profile-samples", type=int, default=100)
+    ap.add_argument("--tail-samples", type=int, default=1000, help="separate latency pass for p99 / p99.9")
     ap.add_argument("--sched", default="measured", choices=["measured", "model"],
                     help="Step 3's `measure latency`: device measurement (default) or the C3 model")
     ap.add_argument("--rnn-tiles", type=int, default=1,
                     help="1: choose the recurrences' gate-tile width by measured latency (harness.tuned_session)")
-    ap.add_argument("--placement", default="batch", choices=["batch", "branch"],
-                    help="N>1: 'batch' = every rank runs its own batch (weak scaling); 'branch' = one batch, "
-                         "subgraphs placed on the GPUs by greedy-correction, cut edges over NCCL (strong)")
+    ap.add_argument("--placement", default="auto", choices=["auto", "shard", "replica", "branch"],
+                    help="N>1: 'shard' (default) = one global batch, rows scattered / gathered over NCCL (strong); "
+                         "'replica' = every rank its own batch (weak); 'branch' = subgraphs placed on GPUs (strong)")
     return ap.parse_args()
 
 
@@ -124,88 +137,97 @@ def time_steps(torch, run_step, home, steps, warmup, flush):
     return [s.elapsed_time(e) for s, e in zip(starts, ends)]
 
 
-def dominant_kernel(wl, cfg):
-    """(node name, algorithmic FLOP or bytes per launch, bound) of the kernel that dominates a
-    step of this workload."""
-    if cfg == "c2":
-        return "fc1", 2 * wl.batch * 1664 * 1024, "tensor"
-    if cfg == "c1":
-        return None, None, None
-    return None, None, None
+def wall_steps(torch, run_step, home, steps, flush):
+    """Host wall clock of duet_run + stream synchronize per step (the user-visible end-to-end
+    latency including the launch path); L2 flushed and synchronised before each step, untimed."""
+    out = []
+    for _ in range(steps):
+        flush.zero_()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        run_step()
+        home.synchronize()
+        out.append((time.perf_counter() - t0) * 1e3)
+    return out
 
 
-def time_node(torch, graph, node, args, out, stream, iters=50, replays=20):
-    """Average device time of one launch of `node`'s kernel(s): `iters` launches captured in a CUDA
-    graph (no host overhead), replayed `replays` times between CUDA events on `stream`."""
-    graph.node_run(node, args, out, stream)
+def node_decl(wl, name):
+    """(op, %-args, dtype, shape) of node `name` in the workload's IR."""
+    for ln in wl.ir.splitlines():
+        m = re.match(r"^%([\w.]+) = (\w+)\((.*?)\).*: (\w+)\[([0-9,]*)\]$", ln)
+        if m and m.group(1) == name:
+            args = [a.strip()[1:] for a in m.group(3).split(",") if a.strip().startswith("%")]
+            return m.group(2), args, m.group(4), tuple(int(x) for x in m.group(5).split(","))
+    raise KeyError(name)
+
+
+DOMINANT = {  # config -> node whose single launch dominates a step (DESIGN.md "Roofline accounting")
+    "c2": "fc1",      # 2048x1024x1664 pair GEMM
+    "c3": "lstmA",    # one tower's persistent LSTM (S = 64)
+    "c4": "gru",      # persistent GRU 1024 (S = 64): the longest single launch; the CNN is 20 launches
+    "c5": "b4_gru",   # persistent GRU 1024 (S = 16, B = 4096): c5's longest single launch
+    "c6": None,
+    "c1": None,       # launch-bound at B = 1: no meaningful roofline
+}
+
+
+def node_work(wl, node):
+    """Algorithmic FLOP of one launch of `node` (2·M·N·K; RNN = 2·S·B·G·H·(E+H))."""
+    op, args, _, shape = node_decl(wl, node)
+    if op == "linear":
+        _, _, _, xs = node_decl(wl, args[0])
+        return 2 * xs[0] * xs[1] * shape[-1]
+    if op in ("lstm", "gru"):
+        _, _, _, xs = node_decl(wl, args[0])   # [S, B, E]
+        S, B, E = xs
+        H = shape[-1]
+        G = 4 if op == "lstm" else 3
+        return 2 * S * B * G * H * (E + H)
+    raise ValueError(op)
+
+
+def time_node_cold(torch, graph, wl, node, stream, flush, samples=15):
+    """Device time of one launch of `node`, L2 cold: a CUDA graph of [512 MB flush, event, the
+    launch, event] on `stream`, replayed `samples` times (synchronised each time); median.  Also the
+    warm back-to-back figure (20 launches in one graph) for reference."""
+    op, args, dt, shape = node_decl(wl, node)
+    tdt = {"bf16": torch.bfloat16, "f32": torch.float32}
+    ins = []
+    for a in args:
+        _, _, adt, ash = node_decl(wl, a)
+        ins.append((torch.randn(ash, device=stream.device) * 0.5).to(tdt[adt]))
+    out = torch.empty(shape, dtype=tdt[dt], device=stream.device)
+    graph.node_run(node, ins, out, stream)
     torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True, external=True)
+    e1 = torch.cuda.Event(enable_timing=True, external=True)
     cg = torch.cuda.CUDAGraph()
     with torch.cuda.graph(cg, stream=stream):
-        for _ in range(iters):
-            graph.node_run(node, args, out, stream)
-    for _ in range(3):
-        cg.replay()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with torch.cuda.stream(stream):
+        flush.zero_()
         e0.record(stream)
-        for _ in range(replays):
-            cg.replay()
+        graph.node_run(node, ins, out, stream)
         e1.record(stream)
+    ts = []
+    for i in range(samples + 2):
+        cg.replay()
+        torch.cuda.synchronize()
+        if i >= 2:
+            ts.append(e0.elapsed_time(e1))
+    cold = statistics.median(ts)
+    warm_g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(warm_g, stream=stream):
+        for _ in range(20):
+            graph.node_run(node, ins, out, stream)
+    warm_g.replay()
     torch.cuda.synchronize()
-    return e0.elapsed_time(e1) / (iters * replays)  # ms
-
-
-def secondary_rooflines(torch, sess, wl, inputs, cfg, stream, dev, hbm_peak, bf16_peak):
-    """c2's other kernels against their own roofline: the hash, the two gathers
-    (HBM bytes: ids + rows + output) and fc2 / fc3 (tensor), each timed like the dominant kernel
-    (CUDA graph of back-to-back launches, events on `stream`); plus the deep gather at the
-    capability size B = 65536 (c2's 13.6 MB gather is too small to saturate HBM)."""
-    if cfg != "c2":
-        return None
-    from paper_conf_ipps_zhanghl21_b200 import duet
-    g = sess.graph
-    B, F, D = wl.batch, 26, 64
-    raw = inputs[0]
-    ids = torch.empty(B, F, dtype=torch.int32, device=dev)
-    g.node_run("ids", [raw], ids, stream)
-    out = {}
-
-    def hbm(name, node, args, y, nbytes, what):
-        ms = time_node(torch, g, node, args, y, stream)
-        gbs = nbytes / (ms / 1e3) / 1e9
-        out[name] = {"bound": "hbm", "kernel": what, "achieved": round(gbs, 1), "peak": hbm_peak, "unit": "GB/s",
-                     "frac": round(gbs / hbm_peak, 4), "bytes_per_launch": nbytes, "ms_per_launch": round(ms, 5)}
-
-    def tensor(name, node, M, N, K, what):
-        x = torch.randn(M, K, device=dev).to(torch.bfloat16)
-        y = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
-        ms = time_node(torch, g, node, [x], y, stream)
-        tf = 2 * M * N * K / (ms / 1e3) / 1e12
-        out[name] = {"bound": "tensor", "kernel": what, "achieved": round(tf, 1), "peak": bf16_peak,
-                     "unit": "TFLOP/s", "frac": round(tf / bf16_peak, 4), "ms_per_launch": round(ms, 5)}
-
-    hbm("hash", "ids", [raw], ids, B * F * (8 + 4), "hash_mod_kernel: int64 raw -> int32 ids")
-    X = torch.empty(B, F * D, dtype=torch.bfloat16, device=dev)
-    hbm("deep_gather", "deep_x", [ids], X, B * F * (4 + 2 * D * 2), "gather_rows16p2_kernel (B=2048; repeated launches: rows L2-warm)")
-    w = torch.empty(B, 1, dtype=torch.float32, device=dev)
-    hbm("wide_gather", "wide", [ids], w, B * F * (4 + 2) + 4 * B, "gather_sum_kernel (algorithmic; 32-B sectors)")
-    tensor("fc2", "fc2", B, 512, 1024, "gemm2_kernel 2048x512x1024")
-    tensor("fc3", "fc3", B, 256, 512, "gemm2_kernel 2048x256x512")
-    # capability size: the same table and kernel, 65536 rows
-    Bc = 65536
-    ir = (f"param @E : bf16[{F},1000000,{D}]\n%ids = input() : i32[{Bc},{F}]\n"
-          f"%x = gather_concat(%ids, @E) : bf16[{Bc},{F * D}]\noutput %x\n")
-    gc = duet.Graph(ir)
-    gc.bind_all({"E": sess.params["deep_E"]})
-    idc = torch.randint(0, 1000000, (Bc, F), dtype=torch.int32, device=dev)
-    Xc = torch.empty(Bc, F * D, dtype=torch.bfloat16, device=dev)
-    ms = time_node(torch, gc, "x", [idc], Xc, stream, iters=10, replays=10)
-    nb = Bc * F * (4 + 2 * D * 2)
-    gbs = nb / (ms / 1e3) / 1e9
-    out["deep_gather_B65536"] = {"bound": "hbm", "kernel": "gather_rows16p2_kernel at the capability size",
-                                 "achieved": round(gbs, 1), "peak": hbm_peak, "unit": "GB/s",
-                                 "frac": round(gbs / hbm_peak, 4), "bytes_per_launch": nb, "ms_per_launch": round(ms, 5)}
-    return out
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with torch.cuda.stream(stream):
+        a.record(stream)
+        for _ in range(5):
+            warm_g.replay()
+        b.record(stream)
+    torch.cuda.synchronize()
+    return cold, a.elapsed_time(b) / 100
 
 
 def load_traffic(node):
@@ -222,17 +244,41 @@ def load_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             d = json.load(f)
-        return d["hbm_gbs"], d["bf16_tflops"], "measured"
+        return d["hbm_gbs"], d["bf16_tflops"], d.get("bf16_tflops_sustained", d["bf16_tflops"]), "measured"
     except Exception:  # noqa: BLE001
-        return 6650.0, 1590.0, "fallback"
+        return 6650.0, 1590.0, 1590.0, "fallback"
+
+
+def roofline(torch, cfg, wl, sess, flush):
+    node = DOMINANT.get(cfg)
+    if node is None:
+        return None
+    hbm, burst, sustained, src = load_peaks()
+    work = node_work(wl, node)
+    cold_ms, warm_ms = time_node_cold(torch, sess.graph, wl, node, sess.home, flush)
+    op = node_decl(wl, node)[0]
+    long_kernel = cold_ms > 0.1
+    # a kernel timed alone: the burst peak; the long recurrences run for 0.3-0.7 ms at full power,
+    # so the sustained figure is the honest denominator there (MEASURED_PEAKS.json)
+    peak = sustained if long_kernel else burst
+    achieved = work / (cold_ms / 1e3) / 1e12
+    kname = {"linear": "gemm2_kernel (tcgen05 cta_group::2, TMA, TMEM)",
+             "lstm": "rnn_persist_kernel (persistent LSTM: tcgen05 per step, fused gates)",
+             "gru": "rnn_persist_kernel (persistent GRU: tcgen05 per step, fused gates)"}[op]
+    return {"bound": "tensor", "kernel": f"{node}: {kname}", "achieved": round(achieved, 1), "peak": peak,
+            "unit": "TFLOP/s", "frac": round(achieved / peak, 4), "traffic": load_traffic(f"{cfg}:{node}"),
+            "peak_source": f"{src} MEASURED_PEAKS.json bf16_tflops{'_sustained' if long_kernel else ''}",
+            "algorithmic_per_launch": work, "ms_per_launch": round(cold_ms, 5), "timing": "cold (L2 flushed)",
+            "warm_ms_per_launch": round(warm_ms, 5),
+            "warm_frac": round(work / (warm_ms / 1e3) / 1e12 / burst, 4)}
 
 
 # ---------------------------------------------------------------------------------------------
-def cpu_oracle_baseline(wl, params_host, inputs_host, seconds, sample_rows=128):
+def cpu_oracle_baseline(wl, params_host, inputs_host, seconds, sample_rows=128, threads=None):
     """Oracle (float64 NumPy, as it stands) on bounded row samples of the same workload."""
     import numpy as np
     import torch
-    from threadpoolctl import threadpool_info
+    from threadpoolctl import threadpool_info, threadpool_limits
 
     from oracle import forward as OF
 
@@ -262,16 +308,34 @@ def cpu_oracle_baseline(wl, params_host, inputs_host, seconds, sample_rows=128):
         oparams[k] = lazy(spec, k) if spec.numel > 10_000_000 else params_host[k]
     OF.run(wl.ir, oparams, oin)  # warm the row cache (untimed)
     done_rows, elapsed, reps = 0, 0.0, 0
-    while elapsed < seconds or reps == 0:
-        t0 = time.perf_counter()
-        OF.run(wl.ir, oparams, oin)
-        elapsed += time.perf_counter() - t0
-        done_rows += len(rows)
-        reps += 1
-    threads = max([p.get("num_threads", 1) for p in threadpool_info()] or [1])
-    return {"value": done_rows / elapsed, "unit": "samples/s", "cores": threads, "kind": "oracle",
+    with threadpool_limits(limits=threads):
+        n_threads = max([p.get("num_threads", 1) for p in threadpool_info()] or [1])
+        while elapsed < seconds or reps == 0:
+            t0 = time.perf_counter()
+            OF.run(wl.ir, oparams, oin)
+            elapsed += time.perf_counter() - t0
+            done_rows += len(rows)
+            reps += 1
+    return {"value": done_rows / elapsed, "unit": "samples/s", "cores": n_threads, "kind": "oracle",
             "sample": f"{reps} timed passes over {len(rows)} random batch rows of {wl.name} (float64 NumPy "
                       f"oracle; the table rows they touch generated before timing)", "seconds": round(elapsed, 2)}
+
+
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
+def host_params(torch, wl):
+    import numpy as np
+    small = {k: s.materialize("cpu") for k, s in wl.params.items() if s.numel <= 10_000_000}
+    return {k: (v.view(torch.int16).numpy().view(np.uint16) if v.dtype == torch.bfloat16 else v.numpy())
+            for k, v in small.items()}
 
 
 def reference_arm(args):
@@ -279,14 +343,11 @@ def reference_arm(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    import numpy as np
     import torch
 
     from paper_conf_ipps_zhanghl21_b200 import workloads as W
     wl = W.build(args.config, dt=args.dtype)
-    small_params = {k: s.materialize("cpu") for k, s in wl.params.items() if s.numel <= 10_000_000}
-    params_host = {k: (v.view(torch.int16).numpy().view(np.uint16) if v.dtype == torch.bfloat16 else v.numpy())
-                   for k, v in small_params.items()}
+    params_host = host_params(torch, wl)
     inputs = {k: s.materialize("cpu") for k, s in wl.inputs.items()}
     # the whole --steps K --warmup W run: ~ref_seconds of timed oracle work (each step >= one pass)
     per_step = max(0.02, min(20.0, args.ref_seconds / max(1, args.steps + args.warmup)))
@@ -302,16 +363,309 @@ def reference_arm(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": wl.name, "global_batch": wl.batch, "parallelism": "cpu"},
             "cpu_baseline": {k: times[0][k] for k in ("cores", "kind", "sample")} | {"value": val,
-                                                                                     "unit": "samples/s"},
+                                                                                     "unit": "samples/s",
+                                                                                     "cpu_model": cpu_model()},
             "e2e": {"value": val, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 # ---------------------------------------------------------------------------------------------
+def make_session(args, cfg, local, batch=None):
+    """Load, bind, partition, profile and schedule one workload on this GPU: the measured
+    greedy-correction schedule (with the recurrences' gate-tile width chosen by measurement), the
+    model-mode schedule and the serial 1-stream baseline of the same kernels."""
+    import torch
+
+    from paper_conf_ipps_zhanghl21_b200 import duet
+    from paper_conf_ipps_zhanghl21_b200 import workloads as W
+    from paper_conf_ipps_zhanghl21_b200.harness import Session, tuned_session
+    kw = {"batch": batch} if batch else {}
+    wl = W.build(cfg, dt=args.dtype, **kw)
+    prof_opts = dict(warmup=5, samples=args.profile_samples, reps=10, calibrate_comm=True)
+    tile_ns = None
+    if args.sched == "measured" and W.rnn_nodes(wl) and args.rnn_tiles:
+        sess, duet_s, tile_ns, base = tuned_session(wl, n_slots=args.slots, device=local, profile=prof_opts,
+                                                    tile_candidates=(0, 128))
+    else:
+        sess = base = Session(wl, n_slots=args.slots, device=local, profile=prof_opts)
+        duet_s = None
+    torch.cuda.synchronize()
+    model_s = sess.schedule(duet.GREEDY_CORRECTION)
+    if duet_s is None:
+        duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=30) if args.sched == "measured" else model_s
+    serial_s = base.schedule(duet.SERIAL)
+    return dict(wl=wl, sess=sess, base=base, duet_s=duet_s, model_s=model_s, serial_s=serial_s, tile_ns=tile_ns)
+
+
+def measure(args, cfg, local, dev, flush, steps, warmup, headline=False):
+    """Everything bench.py reports for one configuration on one GPU."""
+    import torch
+
+    from paper_conf_ipps_zhanghl21_b200 import multirank as MR
+    from paper_conf_ipps_zhanghl21_b200.harness import materialize
+    S = make_session(args, cfg, local)
+    wl, sess, base, duet_s, model_s, serial_s = (S[k] for k in ("wl", "sess", "base", "duet_s", "model_s",
+                                                                "serial_s"))
+    inputs = list(materialize(wl.inputs, dev).values())
+    outs = sess.outputs()
+    torch.cuda.synchronize()  # inputs were generated on the default stream; duet_run uses `home`
+    home = sess.home
+
+    def step_duet():
+        duet_s.run(sess.slots, inputs, outs)
+
+    base.home.wait_stream(torch.cuda.current_stream())
+    t_serial = time_steps(torch, lambda: serial_s.run(base.slots, inputs, outs), base.home, steps, warmup, flush)
+    t_model = None
+    if duet_s is not model_s and duet_s.export()["slot_of"] != model_s.export()["slot_of"]:
+        t_model = time_steps(torch, lambda: model_s.run(sess.slots, inputs, outs), home, steps, warmup, flush)
+
+    # --- timed region (DUET) ---
+    MR.barrier()
+    torch.cuda.synchronize()
+    finish_clocks, _, clk_err = clock_sampler(local) if headline else (None, None, None)
+    t_duet = time_steps(torch, step_duet, home, steps, warmup, flush)
+    clocks = finish_clocks() if finish_clocks else clk_err
+    torch.cuda.synchronize()
+    total_ms = MR.max_over_ranks(sum(t_duet))
+    MR.barrier()
+    # tail pass (p99 / p99.9 need many samples)
+    t_tail = time_steps(torch, step_duet, home, max(args.tail_samples, steps), 0, flush)
+
+    # --- end to end through the C ABI with pinned host buffers ---
+    host_in = [t.cpu().pin_memory() for t in inputs]
+    host_out = sess.outputs(device=False)
+
+    def step_e2e():
+        duet_s.run(sess.slots, host_in, host_out)
+
+    t_e2e = time_steps(torch, step_e2e, home, steps, warmup, flush)
+    e2e_ms = MR.max_over_ranks(sum(t_e2e))
+    t_wall = wall_steps(torch, step_e2e, home, min(steps, 200), flush)
+
+    roof = roofline(torch, cfg, wl, sess, flush) if MR.env()[0] == 0 else None
+    sched = duet_s.export()
+    prof = sess.prof.export()
+    p50 = statistics.median(t_duet)
+    h2d = sum(t.numel() * t.element_size() for t in host_in)
+    d2h = sum(t.numel() * t.element_size() for t in host_out)
+    r = {
+        "workload": wl.name, "baseline_config": BASELINE_IDX.get(cfg), "batch": wl.batch,
+        "total_ms": total_ms, "steps": steps,
+        "p50_ms": round(p50, 5), "p99_ms": round(percentile(t_tail, 99), 5),
+        "p999_ms": round(percentile(t_tail, 99.9), 5), "tail_samples": len(t_tail),
+        "mean_ms": round(statistics.mean(t_duet), 5),
+        "serial_p50_ms": round(statistics.median(t_serial), 5),
+        "speedup_vs_serial": round(statistics.median(t_serial) / p50, 4),
+        "samples_per_s_p50": round(wl.batch / p50 * 1e3, 1),
+        "schedule": {"step3": args.sched, "slot_of": sched["slot_of"], "fell_back": sched["fell_back"],
+                     "model_makespan_ns": sched["makespan"], "profile_t_ns": prof["t_ns"][:, 0].tolist(),
+                     "comm_alpha_same_ns": prof["comm"][0][0],
+                     "measured_ns": getattr(duet_s, "measured_ns", None),
+                     "evaluations": getattr(duet_s, "evaluations", None),
+                     "model_mode_slot_of": model_s.export()["slot_of"],
+                     "model_mode_p50_ms": round(statistics.median(t_model), 5) if t_model else None,
+                     "rnn_tile_n": sess.wl.meta.get("rnn_tile_n"), "rnn_tile_measured_ns": S["tile_ns"]},
+        "e2e": {"value": round(wl.batch * steps / (e2e_ms / 1e3), 1), "unit": "samples/s",
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                "p50_ms": round(statistics.median(t_e2e), 5),
+                "host_wall_p50_ms": round(statistics.median(t_wall), 5),
+                "host_wall_note": "time.perf_counter around duet_run + home-stream synchronize, L2 flushed before"},
+        "launches_per_step": duet_s.launch_count(),
+        "roofline": roof,
+        "clocks": clocks,
+    }
+    r["_keep"] = (wl, inputs)
+    del S, sess, base, duet_s, model_s, serial_s, outs, host_in, host_out
+    return r
+
+
+def bench_single(args):
+    import torch
+
+    from paper_conf_ipps_zhanghl21_b200 import multirank as MR
+    rank, world, local = MR.env()
+    torch.cuda.set_device(local)
+    MR.init("nccl", torch.device(f"cuda:{local}"))
+    dev = f"cuda:{local}"
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
+    head = measure(args, args.config, local, dev, flush, args.steps, args.warmup, headline=True)
+    wl, inputs = head.pop("_keep")
+
+    extra = {}
+    pcs = args.per_config
+    if pcs == "auto":
+        pcs = "c1,c2,c3,c4" if (args.config == "c5" and world == 1) else "none"
+    if pcs != "none" and rank == 0:
+        for c in [c for c in pcs.split(",") if c and c != args.config]:
+            torch.cuda.empty_cache()
+            r = measure(args, c, local, dev, flush, min(args.steps, 200), max(args.warmup, 3))
+            r.pop("_keep")
+            for k in ("total_ms", "steps", "clocks"):
+                r.pop(k)
+            extra[c] = r
+
+    if rank != 0:
+        MR.finalize()
+        return
+    cpu_baseline = None
+    if world == 1 and not args.no_cpu_baseline:
+        ph = host_params(torch, wl)
+        ih = dict(zip(wl.inputs, [t.cpu() for t in inputs]))
+        cpu_baseline = cpu_oracle_baseline(wl, ph, ih, args.cpu_seconds)
+        one = cpu_oracle_baseline(wl, ph, ih, max(2.0, args.cpu_seconds / 3), threads=1)
+        cpu_baseline.update({"cpu_model": cpu_model(), "value_1thread": round(one["value"], 2),
+                             "sample_1thread": one["sample"]})
+
+    total_ms = head.pop("total_ms")
+    line = {
+        "metric": METRIC,
+        "value": round(world * wl.batch * args.steps / (total_ms / 1e3), 1),
+        "unit": "samples/s",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(total_ms / args.steps, 5),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": wl.params[next(iter(wl.params))].dtype if args.dtype is None else args.dtype,
+        "data": "synthetic (seeded counter-based generator; random-init weights)",
+        "config": {"workload": head["workload"], "baseline_config": head["baseline_config"],
+                   "global_batch": wl.batch * world, "per_gpu_batch": wl.batch, "slots": args.slots,
+                   "parallelism": f"dp{world} (independent batches per rank) x {args.slots} stream slots",
+                   "l2": "flushed (512 MB write) before every timed step"},
+        "p50_ms": head["p50_ms"], "p99_ms": head["p99_ms"], "p999_ms": head["p999_ms"],
+        "tail_samples": head["tail_samples"],
+        "serial_p50_ms": head["serial_p50_ms"], "speedup_vs_serial": head["speedup_vs_serial"],
+        "schedule": head["schedule"],
+        "e2e": head["e2e"],
+        "gpu_launches": head["launches_per_step"] * args.steps,
+        "gpu_launches_per_step": head["launches_per_step"],
+        "roofline": head["roofline"],
+        "per_config": extra or None,
+        "cpu_baseline": cpu_baseline,
+        "clocks": head["clocks"],
+    }
+    print(json.dumps(line), flush=True)
+    MR.finalize()
+
+
+# ---------------------------------------------------------------------------------------------
+def bench_shard(args):
+    """--placement shard (N > 1 default): ONE global batch per step (BASELINE.json:11 "batch 4096
+    across 1/2/4/8"); rank 0 holds the inputs in HBM, the rows are scattered over NCCL, every rank
+    runs its B/N rows through its own measured DUET schedule, the outputs are gathered back to rank 0
+    -- all inside the timed step (multirank.ShardExecutor)."""
+    import torch
+
+    from paper_conf_ipps_zhanghl21_b200 import multirank as MR
+    from paper_conf_ipps_zhanghl21_b200 import workloads as W
+    from paper_conf_ipps_zhanghl21_b200.harness import materialize
+    rank, world, local = MR.env()
+    torch.cuda.set_device(local)
+    MR.init("nccl", torch.device(f"cuda:{local}"))
+    dev = torch.device(f"cuda:{local}")
+    full = W.build(args.config, dt=args.dtype)
+    B = full.batch
+    link = MR.calibrate_link()
+    S = make_session(args, args.config, local, batch=B // world)
+    sess, duet_s = S["sess"], S["duet_s"]
+    tdt = {"f32": torch.float32, "bf16": torch.bfloat16}
+    inputs = list(materialize(full.inputs, dev).values()) if rank == 0 else None
+    in_meta = [(s.shape[1:], {"f32": torch.float32, "bf16": torch.bfloat16, "i32": torch.int32,
+                              "i64": torch.int64}[s.dtype]) for s in full.inputs.values()]
+    out_meta = [(tuple(shape[1:]), tdt[dt]) for _, dt, shape in full.outputs]
+    ex = MR.ShardExecutor(B, in_meta, out_meta, dev)
+    outs = [torch.empty((B,) + m[0], dtype=m[1], device=dev) for m in out_meta] if rank == 0 else None
+    cur = torch.cuda.current_stream()
+
+    def runner(si, so):
+        sess.run(duet_s, si, so)                  # home waits on the current stream (the scatter)
+        cur.wait_stream(sess.home)                # the gather sees the shard's outputs
+
+    def step():
+        ex.step(inputs, outs, runner)
+
+    torch.cuda.synchronize()
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    MR.barrier()
+    finish_clocks, _, clk_err = clock_sampler(local)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(args.steps):
+        step()
+    e1.record()
+    torch.cuda.synchronize()
+    clocks = finish_clocks() if finish_clocks else clk_err
+    ms = MR.max_over_ranks(e0.elapsed_time(e1))
+    MR.barrier()
+    # per-step latency (max over ranks per step is bounded by the rank-0 gather: rank 0 waits for all)
+    lat = []
+    for _ in range(min(args.steps, 100)):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        step()
+        b.record()
+        b.synchronize()
+        lat.append(a.elapsed_time(b))
+    # end to end: rank 0's pinned host inputs copied in, scattered, run, gathered, copied out
+    host_in = [t.cpu().pin_memory() for t in inputs] if rank == 0 else None
+    host_out = [torch.empty(o.shape, dtype=o.dtype).pin_memory() for o in outs] if rank == 0 else None
+    dev_in = [torch.empty_like(t) for t in inputs] if rank == 0 else None
+
+    def step_e2e():
+        if rank == 0:
+            for d, h in zip(dev_in, host_in):
+                d.copy_(h, non_blocking=True)
+        ex.step(dev_in, outs, runner)
+        if rank == 0:
+            for h, o in zip(host_out, outs):
+                h.copy_(o, non_blocking=True)
+
+    for _ in range(3):
+        step_e2e()
+    torch.cuda.synchronize()
+    MR.barrier()
+    e0.record()
+    for _ in range(args.steps):
+        step_e2e()
+    e1.record()
+    torch.cuda.synchronize()
+    e2e_ms = MR.max_over_ranks(e0.elapsed_time(e1))
+    sc, ga = ex.bytes_moved()
+    n_launch = duet_s.launch_count()
+    if rank == 0:
+        line = {"metric": METRIC, "value": round(B * args.steps / (ms / 1e3), 1), "unit": "samples/s",
+                "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": round(ms / args.steps, 5), "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": args.dtype or "bf16",
+                "data": "synthetic (seeded counter-based generator; random-init weights)",
+                "config": {"workload": full.name, "baseline_config": BASELINE_IDX.get(args.config),
+                           "global_batch": B, "per_gpu_batch": B // world, "slots": args.slots,
+                           "parallelism": f"batch shards over {world} GPUs (NCCL scatter / gather of one global "
+                                          f"batch inside the step) x {args.slots} stream slots",
+                           "l2": "not flushed (inputs 33 MB on rank 0; every step re-scatters them)"},
+                "p50_ms": round(statistics.median(lat), 5), "p99_ms": round(percentile(lat, 99), 5),
+                "schedule": {"slot_of": duet_s.export()["slot_of"], "per_rank_batch": B // world},
+                "collective_bytes_per_step": {"scatter_from_rank0": sc, "gather_to_rank0": ga},
+                "nvlink_calibration": link,
+                "e2e": {"value": round(B * args.steps / (e2e_ms / 1e3), 1), "unit": "samples/s",
+                        "h2d_bytes_per_step": sum(t.numel() * t.element_size() for t in host_in),
+                        "d2h_bytes_per_step": sum(t.numel() * t.element_size() for t in host_out)},
+                "gpu_launches": n_launch * args.steps, "gpu_launches_per_step_per_rank": n_launch,
+                "roofline": None, "cpu_baseline": None, "clocks": clocks}
+        print(json.dumps(line), flush=True)
+    MR.finalize()
+
+
 def bench_branch(args):
     """--placement branch: ONE batch per step; the greedy-correction schedule over one slot per GPU
     places the subgraphs, each rank runs its (GPU, phase) pieces through libduet, cut-edge tensors
-    move over NCCL point-to-point (paper_conf_ipps_zhanghl21_b200/multigpu.py)."""
+    move over NCCL point-to-point (paper_conf_ipps_zhanghl21_b200/multigpu.py).
+    The cross-GPU link in the comm model is measured (multirank.calibrate_link)."""
     import torch
     import torch.distributed as dist
 
@@ -325,6 +679,7 @@ def bench_branch(args):
     torch.cuda.set_device(local)
     MR.init("nccl", torch.device(f"cuda:{local}"))
     dev = f"cuda:{local}"
+    link = MR.calibrate_link()
     wl = W.build(args.config, dt=args.dtype)
     params = materialize(wl.params, dev)
     g = duet.Graph(wl.ir)
@@ -340,7 +695,8 @@ def bench_branch(args):
         obj = [t_one]
         dist.broadcast_object_list(obj, src=0)
         t_one = obj[0]
-    sg_gpu, sched = MG.place_branches(ex, t_one, world, graph=g)
+    kw = {"cross_alpha_ns": link["alpha_ns"], "cross_ps_per_byte": link["ps_per_byte"]} if link else {}
+    sg_gpu, sched = MG.place_branches(ex, t_one, world, graph=g, **kw)
     pl = MG.plan(wl.ir, ex["node_to_sg"], ex["sg_phase"], sg_gpu)
     runner = MG.DuetPieces(pl, rank, params, local, n_slots=args.slots,
                            profile=dict(warmup=3, samples=max(5, args.profile_samples // 4), reps=5))
@@ -373,8 +729,11 @@ def bench_branch(args):
                            "l2": "not flushed (multi-rank step)"},
                 "placement": {"sg_gpu": sg_gpu, "model_makespan_ns": sched["makespan"],
                               "fell_back": sched["fell_back"], "profile_t_ns": t_one,
+                              "comm_cross": kw or "nominal (single GPU: no link to measure)",
                               "transfers": [(t.tensor, t.src, t.dst) for t in pl.transfers]},
-                "gpu_launches_per_step_rank0": n_launch, "clocks": clocks}
+                "nvlink_calibration": link,
+                "gpu_launches": n_launch * args.steps,
+                "gpu_launches_per_step_rank0": n_launch, "roofline": None, "cpu_baseline": None, "clocks": clocks}
         print(json.dumps(line), flush=True)
     MR.finalize()
 
@@ -383,160 +742,13 @@ def main():
     args = parse()
     if args.impl == "reference":
         return reference_arm(args)
-    if args.placement == "branch":
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    placement = args.placement if args.placement != "auto" else ("shard" if world > 1 else "replica")
+    if placement == "branch":
         return bench_branch(args)
-    import torch
-
-    from paper_conf_ipps_zhanghl21_b200 import duet
-    from paper_conf_ipps_zhanghl21_b200 import multirank as MR
-    from paper_conf_ipps_zhanghl21_b200 import workloads as W
-    from paper_conf_ipps_zhanghl21_b200.harness import Session, materialize, tuned_session
-
-    rank, world, local = MR.env()
-    torch.cuda.set_device(local)
-    MR.init("nccl", torch.device(f"cuda:{local}"))
-    dev = f"cuda:{local}"
-
-    wl = W.build(args.config, dt=args.dtype)
-    prof_opts = dict(warmup=5, samples=args.profile_samples, reps=10, calibrate_comm=True)
-    tile_ns = None
-    if args.sched == "measured" and W.rnn_nodes(wl) and args.rnn_tiles:
-        # the recurrences' gate-tile width chosen by measured latency (harness.tuned_session); the
-        # serial baseline keeps the automatic width (tuned for a branch running alone)
-        sess, duet_s, tile_ns, base = tuned_session(wl, n_slots=args.slots, device=local, profile=prof_opts,
-                                                    tile_candidates=(0, 128))
-    else:
-        sess = base = Session(wl, n_slots=args.slots, device=local, profile=prof_opts)
-        duet_s = None
-    inputs = list(materialize(wl.inputs, dev).values())
-    outs = sess.outputs()
-    torch.cuda.synchronize()
-    model_s = sess.schedule(duet.GREEDY_CORRECTION)
-    if duet_s is None:
-        duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=30) if args.sched == "measured" else model_s
-    serial_s = base.schedule(duet.SERIAL)
-    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
-    home = sess.home
-
-    torch.cuda.synchronize()  # inputs were generated on the default stream; duet_run uses `home`
-
-    def step_duet():
-        duet_s.run(sess.slots, inputs, outs)
-
-    def step_serial():
-        serial_s.run(base.slots, inputs, outs)
-
-    # serial 1-stream reference of the same kernels (BASELINE.json:2)
-    base.home.wait_stream(torch.cuda.current_stream())
-    t_serial = time_steps(torch, step_serial, base.home, args.steps, args.warmup, flush)
-    torch.cuda.synchronize()
-    t_model = None
-    if duet_s is not model_s and duet_s.export()["slot_of"] != model_s.export()["slot_of"]:
-        t_model = time_steps(torch, lambda: model_s.run(sess.slots, inputs, outs), home, args.steps, args.warmup,
-                             flush)
-
-    # --- timed region (DUET) ---
-    MR.barrier()
-    torch.cuda.synchronize()
-    finish_clocks, _, clk_err = clock_sampler(local)
-    t_duet = time_steps(torch, step_duet, home, args.steps, args.warmup, flush)
-    clocks = finish_clocks() if finish_clocks else clk_err
-    torch.cuda.synchronize()
-    total_ms = MR.max_over_ranks(sum(t_duet))
-    MR.barrier()
-
-    # --- end to end through the C ABI with pinned host buffers ---
-    host_in = [t.cpu().pin_memory() for t in inputs]
-    host_out = sess.outputs(device=False)
-
-    def step_e2e():
-        duet_s.run(sess.slots, host_in, host_out)
-
-    t_e2e = time_steps(torch, step_e2e, home, args.steps, args.warmup, flush)
-    e2e_ms = MR.max_over_ranks(sum(t_e2e))
-
-    if rank != 0:
-        MR.finalize()
-        return
-
-    n_launch = duet_s.launch_count()
-    p50 = statistics.median(t_duet)
-    p50_serial = statistics.median(t_serial)
-    value = world * wl.batch * args.steps / (total_ms / 1e3)
-    hbm_peak, bf16_peak, peak_src = load_peaks()
-
-    roof = None
-    node, work, bound = dominant_kernel(wl, args.config)
-    if node:
-        g = sess.graph
-        if args.config == "c2":
-            x = torch.randn(wl.batch, 1664, device=dev).to(torch.bfloat16)
-            y = torch.empty(wl.batch, 1024, device=dev, dtype=torch.bfloat16)
-            ms = time_node(torch, g, node, [x], y, home)
-            achieved = work / (ms / 1e3) / 1e12
-            roof = {"bound": bound, "kernel": f"linear {node} (gemm2_kernel: tcgen05 cta_group::2, 256xBN tile)",
-                    "achieved": round(achieved, 1), "peak": bf16_peak, "unit": "TFLOP/s",
-                    "frac": round(achieved / bf16_peak, 4), "traffic": load_traffic(node),
-                    "peak_source": f"{peak_src} (MEASURED_PEAKS.json bf16_tflops, burst)",
-                    "algorithmic_per_launch": work, "ms_per_launch": round(ms, 5)}
-
-    kernels = secondary_rooflines(torch, sess, wl, inputs, args.config, home, dev, hbm_peak, bf16_peak)
-
-    cpu_baseline = None
-    if world == 1 and not args.no_cpu_baseline:
-        import numpy as np
-        small = {k: s.materialize("cpu") for k, s in wl.params.items() if s.numel <= 10_000_000}
-        ph = {k: (v.view(torch.int16).numpy().view(np.uint16) if v.dtype == torch.bfloat16 else v.numpy())
-              for k, v in small.items()}
-        cpu_baseline = cpu_oracle_baseline(wl, ph, dict(zip(wl.inputs, [t.cpu() for t in inputs])),
-                                           args.cpu_seconds)
-
-    h2d = sum(t.numel() * t.element_size() for t in host_in)
-    d2h = sum(t.numel() * t.element_size() for t in host_out)
-    sched = duet_s.export()
-    prof = sess.prof.export()
-    line = {
-        "metric": METRIC,
-        "value": round(value, 1),
-        "unit": "samples/s",
-        "n_gpus": world,
-        "steps": args.steps,
-        "warmup": args.warmup,
-        "ms_per_step": round(total_ms / args.steps, 5),
-        "higher_is_better": True,
-        "scaling": "weak",
-        "vs_baseline": None,
-        "dtype": wl.params[next(iter(wl.params))].dtype if args.dtype is None else args.dtype,
-        "data": "synthetic (seeded counter-based generator; random-init weights)",
-        "config": {"workload": wl.name, "baseline_config": {"c1": 0, "c2": 1, "c3": 2, "c4": 3, "c5": 4}.get(args.config),
-                   "global_batch": wl.batch * world, "per_gpu_batch": wl.batch, "slots": args.slots,
-                   "parallelism": f"dp{world} (independent batches per rank) x {args.slots} stream slots",
-                   "l2": "flushed (512 MB write) before every timed step"},
-        "p50_ms": round(p50, 5), "p99_ms": round(percentile(t_duet, 99), 5),
-        "p999_ms": round(percentile(t_duet, 99.9), 5),
-        "serial_p50_ms": round(p50_serial, 5),
-        "speedup_vs_serial": round(p50_serial / p50, 4),
-        "schedule": {"step3": args.sched, "slot_of": sched["slot_of"], "fell_back": sched["fell_back"],
-                     "model_makespan_ns": sched["makespan"], "profile_t_ns": prof["t_ns"][:, 0].tolist(),
-                     "comm_alpha_same_ns": prof["comm"][0][0],
-                     "measured_ns": getattr(duet_s, "measured_ns", None),
-                     "evaluations": getattr(duet_s, "evaluations", None),
-                     "model_mode_slot_of": model_s.export()["slot_of"],
-                     "model_mode_p50_ms": round(statistics.median(t_model), 5) if t_model else None,
-                     "rnn_tile_n": sess.wl.meta.get("rnn_tile_n"),
-                     "rnn_tile_measured_ns": tile_ns},
-        "e2e": {"value": round(world * wl.batch * args.steps / (e2e_ms / 1e3), 1), "unit": "samples/s",
-                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                "p50_ms": round(statistics.median(t_e2e), 5)},
-        "gpu_launches": n_launch * args.steps,
-        "gpu_launches_per_step": n_launch,
-        "roofline": roof,
-        "kernels": kernels,
-        "cpu_baseline": cpu_baseline,
-        "clocks": clocks,
-    }
-    print(json.dumps(line), flush=True)
-    MR.finalize()
+    if placement == "shard" and world > 1:
+        return bench_shard(args)
+    return bench_single(args)
 
 
 if __name__ == "__main__":

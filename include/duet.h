@@ -141,7 +141,12 @@ typedef struct {
 
 typedef struct {
   int granularity;   /* 0 = coarse, 1 = one subgraph per operator node    */
-  int batch_shards;  /* 1 = off. >1 is DUET_EUNSUPPORTED in this build       */
+  int batch_shards;  /* 1 = off; k in [2, 64]: every multi-path subgraph becomes k row shards
+                      * (duet_partition_shards).  A sharded
+                      * partition is a scheduling model for multi-GPU placement: it schedules
+                      * from duet_profile_from_table; duet_profile / duet_schedule_measured /
+                      * duet_run reject it with DUET_EUNSUPPORTED (the shards of one subgraph
+                      * run on different ranks, paper_conf_ipps_zhanghl21_b200/multirank.py). */
 } duet_partition_opts;
 
 typedef struct {
@@ -197,6 +202,15 @@ duet_status duet_partition_export(const duet_partition_t* p, int32_t* node_to_sg
                                   uint8_t* phase_kind, int32_t* edge_src, int32_t* edge_dst,
                                   int64_t* edge_bytes, int32_t* n_sg, int32_t* n_phase,
                                   int32_t* n_edge);
+/* Row shards of a batch_shards = k partition (PAPER.md:79 phases with
+ * the paper's subgraphs split by rows for more devices than branches).  sg_shard[n_sg]: shard
+ * index j of each subgraph (rows [j B / k, (j+1) B / k)), -1 if unsharded (sequential phases, or
+ * k = 1); sg_origin[n_sg]: the id the subgraph has in the k = 1 partition.  Shards of one subgraph
+ * have consecutive ids; node_to_sg maps a sharded node to its shard 0.  A boundary tensor of b
+ * bytes entering or leaving shard j carries floor(b (j+1) / k) - floor(b j / k) bytes.  NULL
+ * arrays allowed (counts only). */
+duet_status duet_partition_shards(const duet_partition_t* p, int32_t* sg_shard, int32_t* sg_origin,
+                                  int32_t* n_sg);
 void duet_partition_destroy(duet_partition_t* p);
 
 /* ---- profile (§IV-B; 500 runs PAPER.md:87) -------------------------------------- */

@@ -16,8 +16,14 @@ R-C2), step by step:
   4. a region with >= 2 components is a multi-path phase; separators and regions with <= 1
      component are merged into maximal sequential phases;
   5. granularity: coarse = one subgraph per sequential phase / per component; op = one per node;
-  6. subgraph ids sorted by (phase, smallest topological rank); boundary tensors and bytes.
-Input nodes are not compute and belong to no subgraph (node_to_sg = -1).
+  6. subgraph ids sorted by (phase, smallest topological rank); boundary tensors and bytes;
+  7. batch_shards = k > 1 (multi-GPU): every subgraph of a multi-path
+     phase becomes k row-shard subgraphs (ids consecutive, shard j = rows [j B / k, (j+1) B / k)),
+     each priced separately by the profile; a tensor crossing into or out of shard j carries
+     share_j(b) = floor(b (j+1) / k) - floor(b j / k) of its b bytes (the shares sum to b);
+     shard-to-shard edges connect equal shard indices only (rows are independent).
+Input nodes are not compute and belong to no subgraph (node_to_sg = -1; a sharded node maps to
+its shard 0).
 """
 from __future__ import annotations
 
@@ -38,6 +44,8 @@ class Partition:
     phase_kind: list        # SEQ / MULTI
     edges: dict             # (src_sg, dst_sg) -> bytes; -1 = graph input / output
     n_placeholders: int
+    sg_shard: list = None   # per subgraph: row-shard index, -1 = unsharded (batch_shards = 1 or seq phase)
+    sg_origin: list = None  # per subgraph: id of the unsharded subgraph it is a shard of
 
     @property
     def n_sg(self):
@@ -82,7 +90,12 @@ def _reach(start, adj, n_total, blocked=None):
     return seen
 
 
-def partition(ir, granularity: str = "coarse") -> Partition:
+def share(b: int, j: int, k: int) -> int:
+    """Bytes of a b-byte row-major tensor that fall in row shard j of k (step 7)."""
+    return b * (j + 1) // k - b * j // k
+
+
+def partition(ir, granularity: str = "coarse", batch_shards: int = 1) -> Partition:
     g: Graph = parse(ir) if isinstance(ir, str) else ir
     n0 = len(g.nodes)
     is_input = [nd.op == "input" for nd in g.nodes]
@@ -194,7 +207,33 @@ def partition(ir, granularity: str = "coarse") -> Partition:
     for s, (_, nodes) in enumerate(sgs):
         for v in nodes:
             sg_of[v] = s
-    tensors = {}
+    # ---- step 7: row shards of the multi-path subgraphs ----
+    k = int(batch_shards)
+    if k < 1:
+        raise ValueError("batch_shards must be >= 1")
+    ids = []                      # unsharded subgraph -> its new ids (k of them if sharded)
+    sg_shard, sg_origin = [], []
+    for s, (p, _) in enumerate(sgs):
+        shard = k > 1 and phases[p][0] == MULTI
+        ids.append([])
+        for j in range(k if shard else 1):
+            ids[s].append(len(sg_shard))
+            sg_shard.append(j if shard else -1)
+            sg_origin.append(s)
+
+    def pairs(src, dst):
+        """(new src, new dst, shard index of the bytes or -1) for an edge between two unsharded ids."""
+        S = ids[src] if src >= 0 else [-1]
+        D = ids[dst] if dst >= 0 else [-1]
+        if len(S) > 1 and len(D) > 1:
+            return [(S[j], D[j], j) for j in range(k)]
+        if len(D) > 1:
+            return [(S[0], D[j], j) for j in range(k)]
+        if len(S) > 1:
+            return [(S[i], D[0], i) for i in range(k)]
+        return [(S[0], D[0], -1)]
+
+    tensors = {}                  # (new src, new dst) -> (shard index, {tensor ids})
     for v in range(N):
         if not compute[v]:
             continue
@@ -202,17 +241,26 @@ def partition(ir, granularity: str = "coarse") -> Partition:
             src = sg_of[u] if compute[u] else -1
             if src == sg_of[v]:
                 continue
-            tensors.setdefault((src, sg_of[v]), set()).add(alias[u])
+            for a, b, j in pairs(src, sg_of[v]):
+                tensors.setdefault((a, b), (j, set()))[1].add(alias[u])
     for o in g.outputs:
         if compute[o]:
-            tensors.setdefault((sg_of[o], -1), set()).add(o)
-    edges = {k: sum(g.nodes[t].nbytes for t in ts) for k, ts in tensors.items()}
+            for a, b, j in pairs(sg_of[o], -1):
+                tensors.setdefault((a, b), (j, set()))[1].add(o)
+    edges = {key: sum(g.nodes[t].nbytes if j < 0 else share(g.nodes[t].nbytes, j, k) for t in ts)
+             for key, (j, ts) in tensors.items()}
+    sg_nodes, sg_phase = [], []
+    for s_new, s in enumerate(sg_origin):
+        sg_nodes.append(sgs[s][1])
+        sg_phase.append(sgs[s][0])
     return Partition(
         n_nodes=n0,
-        node_to_sg=[sg_of[v] for v in range(n0)],
-        sg_nodes=[nodes for _, nodes in sgs],
-        sg_phase=[p for p, _ in sgs],
-        phase_kind=[k for k, _ in phases],
+        node_to_sg=[ids[sg_of[v]][0] if sg_of[v] >= 0 else -1 for v in range(n0)],
+        sg_nodes=sg_nodes,
+        sg_phase=sg_phase,
+        phase_kind=[kk for kk, _ in phases],
         edges=edges,
         n_placeholders=n_ph,
+        sg_shard=sg_shard,
+        sg_origin=sg_origin,
     )

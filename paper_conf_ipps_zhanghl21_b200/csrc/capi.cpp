@@ -108,10 +108,8 @@ duet_status duet_partition(const duet_graph_t* g, const duet_partition_opts* o, 
     need(out, "out");
     duet_partition_opts opts{0, 1};
     if (o) opts = *o;
-    if (opts.batch_shards != 1)
-      fail(DUET_EUNSUPPORTED, "batch_shards > 1: multi-GPU runs shard the batch across ranks (DESIGN.md)");
     std::unique_ptr<duet_partition_t> h(new duet_partition_t());
-    h->p.reset(make_partition(g->g.get(), opts.granularity));
+    h->p.reset(make_partition(g->g.get(), opts.granularity, opts.batch_shards));
     *out = h.release();
   });
 }
@@ -141,7 +139,26 @@ duet_status duet_partition_export(const duet_partition_t* p, int32_t* node_to_sg
   });
 }
 
+duet_status duet_partition_shards(const duet_partition_t* p, int32_t* sg_shard, int32_t* sg_origin, int32_t* n_sg) {
+  return guard([&] {
+    need(p, "partition");
+    const Partition& P = *p->p;
+    if (n_sg) *n_sg = P.n_sg();
+    for (int s = 0; s < P.n_sg(); ++s) {
+      if (sg_shard) sg_shard[s] = P.sg_shard[s];
+      if (sg_origin) sg_origin[s] = P.sg_origin[s];
+    }
+  });
+}
+
 void duet_partition_destroy(duet_partition_t* p) { delete p; }
+
+static void no_shards(const Partition& P, const char* what) {
+  if (P.sharded())
+    fail(DUET_EUNSUPPORTED, std::string(what) +
+                                ": a batch_shards > 1 partition is a scheduling model (its row shards run on "
+                                "different ranks, multirank.ShardExecutor); profile it from a table");
+}
 
 duet_status duet_profile(const duet_partition_t* p, const duet_slot* slots, int n_slots, const duet_profile_opts* o,
                          duet_profile_t** out) {
@@ -151,6 +168,7 @@ duet_status duet_profile(const duet_partition_t* p, const duet_slot* slots, int 
     need(out, "out");
     need(slots, "slots");
     if (n_slots < 1) fail(DUET_EINVAL, "n_slots < 1");
+    no_shards(*p->p, "duet_profile");
     std::unique_ptr<duet_profile_t> h(new duet_profile_t());
     h->pr.reset(profile_on_device(p->p.get(), slots, n_slots, o));
     *out = h.release();
@@ -220,6 +238,7 @@ duet_status duet_schedule_measured(const duet_partition_t* p, const duet_profile
     need(pr, "profile");
     need(slots, "slots");
     need(out, "out");
+    no_shards(*p->p, "duet_schedule_measured");
     std::unique_ptr<duet_schedule_t> h(new duet_schedule_t());
     h->s.reset(schedule_measured(p->p.get(), pr->pr.get(), o, slots, n_slots, mo));
     *out = h.release();
@@ -249,6 +268,7 @@ duet_status duet_run(duet_schedule_t* s, const duet_slot* slots, int n_slots, co
     need(slots, "slots");
     if (n_in && !inputs) fail(DUET_EINVAL, "inputs is NULL");
     if (n_out && !outputs) fail(DUET_EINVAL, "outputs is NULL");
+    no_shards(*s->s->p, "duet_run");
     run_schedule(s->s.get(), slots, n_slots, inputs, n_in, outputs, n_out);
   });
 }

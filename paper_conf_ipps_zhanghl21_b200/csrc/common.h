@@ -86,10 +86,14 @@ struct Partition {
   std::vector<int> phase_kind;
   std::map<std::pair<int, int>, int64_t> edges;  // (src,dst) -> bytes; -1 = graph in/out
   int n_placeholders = 0;
+  int batch_shards = 1;
+  std::vector<int> sg_shard;   // row-shard index of each subgraph, -1 = unsharded
+  std::vector<int> sg_origin;  // the unsharded subgraph a shard comes from
   int n_sg() const { return (int)sg_nodes.size(); }
+  bool sharded() const { return batch_shards > 1; }
 };
 
-Partition* make_partition(const Graph* g, int granularity);
+Partition* make_partition(const Graph* g, int granularity, int batch_shards = 1);
 
 struct Profile {
   const Partition* p = nullptr;

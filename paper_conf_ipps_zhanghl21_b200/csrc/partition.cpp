@@ -32,8 +32,13 @@ std::vector<char> reach(int start, const std::vector<std::vector<int>>& adj, int
 
 }  // namespace
 
-Partition* make_partition(const Graph* g, int granularity) {
+// Bytes of a b-byte row-major tensor in row shard j of k: the k shares
+// floor(b (j+1) / k) - floor(b j / k) sum to b.
+static int64_t share(int64_t b, int j, int k) { return b * (j + 1) / k - b * j / k; }
+
+Partition* make_partition(const Graph* g, int granularity, int batch_shards) {
   if (granularity != 0 && granularity != 1) fail(DUET_EINVAL, "granularity must be 0 or 1");
+  if (batch_shards < 1 || batch_shards > 64) fail(DUET_EINVAL, "batch_shards must be in [1, 64]");
   const int n0 = (int)g->nodes.size();
   std::vector<std::vector<int>> preds(n0), succs(n0);
   std::vector<char> is_input(n0);
@@ -222,24 +227,67 @@ Partition* make_partition(const Graph* g, int granularity) {
   std::vector<int> sg_of(N, -1);
   for (int s = 0; s < (int)sgs.size(); ++s)
     for (int v : sgs[s].second) sg_of[v] = s;
-  std::map<std::pair<int, int>, std::set<int>> tensors;
+  // step 7 (batch_shards = k > 1): every multi-path subgraph becomes k row-shard subgraphs with
+  // consecutive ids; boundary bytes split by share(); shard-to-shard edges pair equal indices
+  const int k = batch_shards;
+  std::vector<std::vector<int>> ids(sgs.size());
+  for (int s = 0; s < (int)sgs.size(); ++s) {
+    const bool shard = k > 1 && phases[sgs[s].first].first == kMulti;
+    for (int j = 0; j < (shard ? k : 1); ++j) {
+      ids[s].push_back((int)P->sg_shard.size());
+      P->sg_shard.push_back(shard ? j : -1);
+      P->sg_origin.push_back(s);
+    }
+  }
+  struct Pair { int a, b, j; };
+  auto pairs = [&](int src, int dst) {
+    std::vector<int> S = src >= 0 ? ids[src] : std::vector<int>{-1};
+    std::vector<int> D = dst >= 0 ? ids[dst] : std::vector<int>{-1};
+    std::vector<Pair> out;
+    if (S.size() > 1 && D.size() > 1) {
+      for (int j = 0; j < k; ++j) out.push_back({S[j], D[j], j});
+    } else if (D.size() > 1) {
+      for (int j = 0; j < k; ++j) out.push_back({S[0], D[j], j});
+    } else if (S.size() > 1) {
+      for (int i = 0; i < k; ++i) out.push_back({S[i], D[0], i});
+    } else {
+      out.push_back({S[0], D[0], -1});
+    }
+    return out;
+  };
+  std::map<std::pair<int, int>, std::pair<int, std::set<int>>> tensors;  // -> (shard index, tensors)
   for (int v = 0; v < N; ++v) {
     if (!compute(v)) continue;
     for (int u : preds[v]) {
       int src = compute(u) ? sg_of[u] : -1;
       if (src == sg_of[v]) continue;
-      tensors[{src, sg_of[v]}].insert(alias[u]);
+      for (const Pair& e : pairs(src, sg_of[v])) {
+        auto& t = tensors[{e.a, e.b}];
+        t.first = e.j;
+        t.second.insert(alias[u]);
+      }
     }
   }
   for (int o : g->outputs)
-    if (compute(o)) tensors[{sg_of[o], -1}].insert(o);
+    if (compute(o))
+      for (const Pair& e : pairs(sg_of[o], -1)) {
+        auto& t = tensors[{e.a, e.b}];
+        t.first = e.j;
+        t.second.insert(o);
+      }
   for (auto& kv : tensors) {
     int64_t b = 0;
-    for (int t : kv.second) b += g->nodes[t].nbytes();
+    for (int t : kv.second.second) {
+      const int64_t nb = g->nodes[t].nbytes();
+      b += kv.second.first < 0 ? nb : share(nb, kv.second.first, k);
+    }
     P->edges[kv.first] = b;
   }
-  P->node_to_sg.assign(sg_of.begin(), sg_of.begin() + n0);
-  for (auto& s : sgs) {
+  P->batch_shards = k;
+  P->node_to_sg.resize(n0);
+  for (int v = 0; v < n0; ++v) P->node_to_sg[v] = sg_of[v] >= 0 ? ids[sg_of[v]][0] : -1;
+  for (int s_new = 0; s_new < (int)P->sg_origin.size(); ++s_new) {
+    const auto& s = sgs[P->sg_origin[s_new]];
     P->sg_nodes.push_back(s.second);
     P->sg_phase.push_back(s.first);
   }

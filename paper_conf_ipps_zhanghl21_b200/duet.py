@@ -84,6 +84,7 @@ _sig = {
                                         C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.POINTER(C.c_int64),
                                         C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.POINTER(C.c_int32)]),
     "duet_partition_destroy": (None, [_P]),
+    "duet_partition_shards": (C.c_int, [_P, C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.POINTER(C.c_int32)]),
     "duet_profile": (C.c_int, [_P, C.POINTER(Slot), C.c_int, C.POINTER(ProfileOpts), C.POINTER(_P)]),
     "duet_profile_from_table": (C.c_int, [_P, C.c_int, C.POINTER(C.c_int32), C.POINTER(C.c_int64),
                                           C.POINTER(CommModel), C.POINTER(_P)]),
@@ -235,6 +236,14 @@ class Partition:
             "phase_kind": kind[:n_ph.value].tolist(),
             "edges": {(int(a), int(b)): int(c) for a, b, c in zip(es[:n_e.value], ed[:n_e.value], eb[:n_e.value])},
         }
+
+    def shards(self) -> dict:
+        """Row shards of a batch_shards > 1 partition (duet_partition_shards)."""
+        n = C.c_int32()
+        _check(_lib.duet_partition_shards(self._h, None, None, C.byref(n)))
+        sh, org = np.zeros(max(1, n.value), np.int32), np.zeros(max(1, n.value), np.int32)
+        _check(_lib.duet_partition_shards(self._h, _np_ptr(sh, C.c_int32), _np_ptr(org, C.c_int32), None))
+        return {"sg_shard": sh[:n.value].tolist(), "sg_origin": org[:n.value].tolist()}
 
     @property
     def n_sg(self) -> int:

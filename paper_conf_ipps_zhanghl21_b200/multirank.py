@@ -87,3 +87,115 @@ def barrier():
 def finalize():
     if dist.is_initialized():
         dist.destroy_process_group()
+
+
+class ShardExecutor:
+    """One global batch per step with its rows sharded over the ranks (SURVEY.md §8(e) item 1,
+    strong scaling): rank 0 holds the step's inputs, every input is scattered in contiguous row
+    blocks (one collective per input), each rank runs `runner(shard_inputs, shard_outputs)` on
+    its rows, and every output is gathered back to rank 0 in rank order.  Rows are independent
+    (BN folded; the only cross-row operators are per-row joins), so the result equals the
+    single-GPU run of the whole batch.  With NCCL everything is enqueued on the current stream
+    (no host synchronisation inside a step); with gloo device tensors are staged through host
+    memory (the one-GPU test of the multi-rank flow).
+
+    in_meta / out_meta: [(trailing shape, torch dtype)] per input / output; n_rows must divide by
+    the world size (NCCL scatter/gather move equal blocks)."""
+
+    def __init__(self, n_rows: int, in_meta, out_meta, device: torch.device):
+        self.world = dist.get_world_size() if dist.is_initialized() else 1
+        self.rank = dist.get_rank() if dist.is_initialized() else 0
+        if n_rows % self.world:
+            raise ValueError(f"batch {n_rows} does not split evenly over {self.world} ranks")
+        self.n_rows, self.rows = n_rows, n_rows // self.world
+        self.device = device
+        self.staged = dist.is_initialized() and dist.get_backend() == "gloo" and device.type == "cuda"
+        mk = lambda shape, dt: torch.empty((self.rows,) + tuple(shape), dtype=dt, device=device)  # noqa: E731
+        self.shard_in = [mk(s, d) for s, d in in_meta]
+        self.shard_out = [mk(s, d) for s, d in out_meta]
+        self.out_meta = out_meta
+
+    def bytes_moved(self):
+        """(scatter bytes leaving rank 0, gather bytes arriving at rank 0) per step."""
+        ob = (self.world - 1) * self.rows
+        sc = sum(t[0].numel() * t.element_size() * ob for t in self.shard_in)
+        ga = sum(t[0].numel() * t.element_size() * ob for t in self.shard_out)
+        return sc, ga
+
+    def _scatter(self, full, shard):
+        if self.world == 1:
+            shard.copy_(full)
+            return
+        if self.staged:
+            tmp = torch.empty(shard.shape, dtype=shard.dtype)
+            chunks = list(full.cpu().chunk(self.world)) if self.rank == 0 else None
+            dist.scatter(tmp, chunks, src=0)
+            shard.copy_(tmp)
+            return
+        dist.scatter(shard, list(full.chunk(self.world)) if self.rank == 0 else None, src=0)
+
+    def _gather(self, shard, full):
+        if self.world == 1:
+            full.copy_(shard)
+            return
+        if self.staged:
+            bufs = [torch.empty(shard.shape, dtype=shard.dtype) for _ in range(self.world)] if self.rank == 0 else None
+            dist.gather(shard.cpu(), bufs, dst=0)
+            if self.rank == 0:
+                full.copy_(torch.cat(bufs))
+            return
+        dist.gather(shard, list(full.chunk(self.world)) if self.rank == 0 else None, dst=0)
+
+    def step(self, inputs, outputs, runner):
+        """inputs / outputs: full-batch tensors on rank 0 (ignored elsewhere).  runner(shard_in,
+        shard_out) computes this rank's rows in place."""
+        for i, s in enumerate(self.shard_in):
+            self._scatter(inputs[i] if self.rank == 0 else None, s)
+        runner(self.shard_in, self.shard_out)
+        for i, s in enumerate(self.shard_out):
+            self._gather(s, outputs[i] if self.rank == 0 else None)
+
+
+def calibrate_link(sizes=(1 << 12, 1 << 16, 1 << 20, 1 << 24), reps: int = 20, peer: int = 1):
+    """Measured NVLink cut-edge cost for the comm model (§III-B, Fig. 5: transfer
+    latency is linear in the message size): rank 0 <-> `peer` NCCL send/recv ping-pong per size,
+    timed with CUDA events on rank 0; one-way time = half the round trip.  A least-squares line
+    t = alpha + bytes * ps_per_byte / 1000 gives the comm model's cross-GPU link (integer ns and
+    ps per byte, include/duet.h duet_link).  Every rank must call it; returns the same dict on
+    every rank, or None without a second GPU (single rank)."""
+    if not dist.is_initialized() or dist.get_world_size() < 2 or dist.get_backend() != "nccl":
+        return None
+    rank = dist.get_rank()
+    dev = torch.device("cuda", torch.cuda.current_device())
+    pts = []
+    for nb in sizes:
+        buf = torch.empty(nb, dtype=torch.uint8, device=dev)
+        ms = None
+        for it in range(reps + 3):
+            if rank == 0:
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                dist.send(buf, peer)
+                dist.recv(buf, peer)
+                e1.record()
+                e1.synchronize()
+                if it >= 3:
+                    t = e0.elapsed_time(e1) / 2
+                    ms = t if ms is None else min(ms, t)
+            elif rank == peer:
+                dist.recv(buf, 0)
+                dist.send(buf, 0)
+        if rank == 0:
+            pts.append((nb, ms * 1e6))
+    res = [None]
+    if rank == 0:
+        xs = [p[0] for p in pts]
+        ys = [p[1] for p in pts]
+        n = len(xs)
+        mx, my = sum(xs) / n, sum(ys) / n
+        slope = sum((x - mx) * (y - my) for x, y in zip(xs, ys)) / max(sum((x - mx) ** 2 for x in xs), 1e-30)
+        alpha = my - slope * mx
+        res[0] = {"alpha_ns": max(0, int(round(alpha))), "ps_per_byte": max(0, int(round(slope * 1000))),
+                  "points_ns": [(int(b), round(t, 1)) for b, t in pts], "peer": peer}
+    dist.broadcast_object_list(res, src=0)
+    return res[0]

@@ -179,3 +179,77 @@ def test_rnn_tile_n_rewrite(cfg):
     p0 = duet.Graph(wl.ir).partition("coarse").export()
     p1 = duet.Graph(w128.ir).partition("coarse").export()
     assert p0 == p1
+
+
+# ---- batch_shards = k ---------------------------------------------------
+def _same_sharded(ir, gran, k):
+    dp = duet.Graph(ir).partition(gran, batch_shards=k)
+    p = dp.export()
+    o = o_partition(ir, gran, batch_shards=k)
+    assert p["node_to_sg"] == o.node_to_sg and p["sg_phase"] == o.sg_phase
+    assert p["phase_kind"] == o.phase_kind and p["edges"] == o.edges
+    sh = dp.shards()
+    assert sh["sg_shard"] == o.sg_shard and sh["sg_origin"] == o.sg_origin
+    return dp, o
+
+
+@pytest.mark.parametrize("cfg", ["c1", "c2", "c3", "c4", "c5", "c6"])
+@pytest.mark.parametrize("k", [2, 3, 8])
+def test_batch_shards_bit_exact_configs(cfg, k):
+    """libduet's row-shard transform == the oracle's, on every config; c5 at k = 8 has the 8k + 1 = 65
+    subgraphs of SURVEY.md §8(a) A0."""
+    ir = W.build(cfg, small=not (cfg == "c5" and k == 8)).ir
+    dp, o = _same_sharded(ir, "coarse", k)
+    base = o_partition(ir)
+    n_multi = sum(1 for s in range(base.n_sg) if base.phase_kind[base.sg_phase[s]] == 1)
+    assert o.n_sg == base.n_sg + (k - 1) * n_multi
+    if cfg == "c5":
+        assert o.n_sg == 8 * k + 1
+    # the shares of every boundary tensor add back up to the unsharded bytes
+    agg = {}
+    for (a, b), nb in o.edges.items():
+        key = (o.sg_origin[a] if a >= 0 else -1, o.sg_origin[b] if b >= 0 else -1)
+        agg[key] = agg.get(key, 0) + nb
+    # (an edge between a sharded and an unsharded subgraph splits into k shares; shard-to-shard
+    # edges pair equal indices: either way the parts sum to the unsharded bytes)
+    assert agg == base.edges
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_batch_shards_bit_exact_fuzz(seed):
+    rng = random.Random(5000 + seed)
+    ir = random_dag_ir(rng, rng.randint(2, 14), rng.randint(1, 3))
+    gran = rng.choice(["coarse", "op"])
+    k = rng.choice([2, 3, 4, 7])
+    dp, o = _same_sharded(ir, gran, k)
+    if o.n_sg > 24:   # the Python greedy-correction is O(n^3) model evaluations: partition only
+        return
+    D = rng.choice([2, 3, 4])
+    slot_gpu = list(range(D))
+    T = [[rng.randint(1, 40) * 1000 for _ in range(D)] for _ in range(o.n_sg)]
+    comm = Comm(Link(rng.randint(0, 3000), rng.randint(0, 3)), Link(rng.randint(0, 9000), rng.randint(0, 500)))
+    os_ = o_schedule(o, T, slot_gpu, comm)
+    e = dp.profile_from_table(slot_gpu, T, ((comm.same_gpu.alpha_ns, comm.same_gpu.ps_per_byte),
+                                            (comm.cross_gpu.alpha_ns, comm.cross_gpu.ps_per_byte))).schedule().export()
+    assert e["slot_of"] == os_.slot_of and e["makespan"] == os_.makespan and e["fell_back"] == os_.fell_back
+
+
+def test_batch_shards_hand_case():
+    """x -> {a, b} -> j with k = 3: a and b become shards 0..2 (ids 0-2 and 3-5), j is 6.
+    x is f32[6,4] (96 B): each shard of a reads 32 B; a's output f32[6,2] (48 B) reaches j as
+    16 B per shard; the unsharded output j f32[6,1] leaves whole (24 B).  Shares of 10 B over
+    k = 3 are 3, 3, 4 (floor(10 (j+1) / 3) - floor(10 j / 3))."""
+    from oracle.partition import share
+    ir = ("%x = input() : f32[6,4]\n%a = opaque(%x) : f32[6,2]\n%b = opaque(%x) : f32[6,3]\n"
+          "%j = opaque(%a, %b) : f32[6,1]\noutput %j\n")
+    dp, o = _same_sharded(ir, "coarse", 3)
+    assert o.n_sg == 7 and o.sg_shard == [0, 1, 2, 0, 1, 2, -1] and o.sg_origin == [0, 0, 0, 1, 1, 1, 2]
+    assert o.node_to_sg == [-1, 0, 3, 6]
+    assert o.edges[(-1, 0)] == 32 and o.edges[(-1, 5)] == 32
+    assert o.edges[(1, 6)] == 16 and o.edges[(4, 6)] == 24 and o.edges[(6, -1)] == 24
+    assert [share(10, j, 3) for j in range(3)] == [3, 3, 4]
+    with pytest.raises(duet.DuetError) as e:
+        dp.profile([(0, 0)])
+    assert e.value.name == "EUNSUPPORTED"
+    with pytest.raises(duet.DuetError):
+        duet.Graph(ir).partition(batch_shards=0)

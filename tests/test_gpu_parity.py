@@ -690,24 +690,33 @@ def test_branch_placement_pieces_on_device():
 
 def test_bench_contract_keys():
     """`python bench.py` (the driver's default N=1 run, shortened): one JSON line with the contract's
-    keys, the roofline of the dominant kernel measured live, the CPU-oracle baseline and the e2e leg."""
+    keys for the c5 headline, the cold roofline of its dominant kernel, a per-config block, the
+    CPU-oracle baseline and the e2e leg (device-event and host wall clock)."""
     import json
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     r = subprocess.run([sys.executable, "bench.py", "--steps", "10", "--warmup", "3", "--cpu-seconds", "1",
-                        "--profile-samples", "5"], cwd=root, capture_output=True, text=True, timeout=900)
+                        "--profile-samples", "5", "--tail-samples", "30", "--per-config", "c2"],
+                       cwd=root, capture_output=True, text=True, timeout=1500)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
     for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
-              "vs_baseline", "dtype", "data", "config", "e2e", "gpu_launches", "roofline", "cpu_baseline", "clocks"):
+              "vs_baseline", "dtype", "data", "config", "e2e", "gpu_launches", "roofline", "cpu_baseline", "clocks",
+              "per_config", "p99_ms", "p999_ms"):
         assert k in d, k
     assert d["steps"] == 10 and d["warmup"] == 3 and d["n_gpus"] == 1 and d["value"] > 0
-    assert d["config"]["workload"] == "c2_wide_deep"
+    assert d["config"]["workload"] == "c5_ensemble" and d["tail_samples"] == 30
     assert d["roofline"]["bound"] == "tensor" and 0 < d["roofline"]["frac"] < 1
+    assert d["roofline"]["timing"].startswith("cold")
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["value"] > 0
-    assert d["e2e"]["h2d_bytes_per_step"] == 2048 * 26 * 8 and d["e2e"]["d2h_bytes_per_step"] == 2048 * 4
+    assert d["cpu_baseline"]["value_1thread"] > 0
+    assert d["e2e"]["h2d_bytes_per_step"] > 30e6 and d["e2e"]["d2h_bytes_per_step"] == 4096 * 4
+    assert d["e2e"]["host_wall_p50_ms"] >= d["e2e"]["p50_ms"] * 0.9
     assert d["gpu_launches"] >= d["steps"]
+    c2 = d["per_config"]["c2"]
+    assert c2["workload"] == "c2_wide_deep" and c2["roofline"]["frac"] > 0 and c2["speedup_vs_serial"] > 0
+    assert c2["e2e"]["h2d_bytes_per_step"] == 2048 * 26 * 8
