@@ -11,6 +11,12 @@
 // continuous stage ring (2 k-blocks per stage) and a double-buffered TMEM accumulator; 4 epilogue
 // warps add the folded BN bias and the optional residual, apply ReLU and store bf16 NHWC.
 // Layers with C % 64 != 0 (the 3-channel stem) use im2col_kernel + the CTA-pair GEMM instead.
+//
+// Tap rectangle (round 2): filter taps whose window lies in the zero padding for EVERY output pixel
+// are skipped (their products are exact zeros).  A 3x3 / pad 1 conv on a 1x1 map (c5's ResNet
+// layer 4 at 32x32 input) keeps only the centre tap: K drops 9x (57 -> 24 us).  (A split-K variant
+// for the under-filled layer-3/4 grids -- fp32 partial tiles + last-arriver reduction -- was built
+// and measured slower at every ResNet shape, 1.1-3x.)
 #include <cudaTypedefs.h>
 
 #include "../common.h"
@@ -43,8 +49,10 @@ struct ConvArgs {
   const __nv_bfloat16* res;
   __nv_bfloat16* y;
   ConvShape s;
-  int K;   // kh * kw * C (true reduction length)
+  int K;   // kh * kw * C (true reduction length; also the first fully out-of-bounds weight column)
   int act;
+  int nkb;             // effective 64-wide k-blocks: taps in the rectangle x C / 64
+  int r0, s0, ns;      // tap rectangle: rows r0.., columns s0 .. s0 + ns - 1
 };
 
 // TMA-im2col variant (C % 64 == 0): one thread streams both operands; A tile = 128 consecutive
@@ -68,10 +76,14 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   const int warp = ptx::warp_id();
   const int lane = threadIdx.x & 31;
   const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
-  const int nk = (a.K + KB * CBK - 1) / (KB * CBK);
   const int tiles_n = (s.Co + BN - 1) / BN;
   const int64_t n_tiles = ((M + CBM - 1) / CBM) * tiles_n;
+  const int64_t n_units = n_tiles;
   const int cb = s.C / 64;
+  auto krange = [&](int64_t, int& kb0, int& kb1) {
+    kb0 = 0;
+    kb1 = a.nkb;
+  };
 
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tmX);
@@ -103,7 +115,8 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   if (warp == 0) {
     if (lane == 0) {
       int64_t g = 0;
-      for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+      for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x) {
+        const int64_t tile = u;
         const int n0 = (int)(tile % tiles_n) * BN;
         const int64_t m0 = (tile / tiles_n) * CBM;
         const int wo = (int)(m0 % s.Wo);
@@ -111,20 +124,25 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
         const int ho = (int)(q0 % s.Ho);
         const int nn = (int)(q0 / s.Ho);
         const int wb = wo * s.stride - s.pad, hb = ho * s.stride - s.pad;
-        int kb = 0;
+        int kb0, kb1;
+        krange(u, kb0, kb1);
+        const int nk = (kb1 - kb0 + KB - 1) / KB;
         for (int it = 0; it < nk; ++it, ++g) {
           const int st = (int)(g % C::STAGES);
           const int64_t use = g / C::STAGES;
           if (use >= 1) ptx::mbar_wait(&empty[st], (uint32_t)((use - 1) & 1));
           ptx::mbar_arrive_expect_tx(&full[st], C::STAGE);
 #pragma unroll
-          for (int h = 0; h < KB; ++h, ++kb) {
-            const int kbc = kb < a.K / CBK ? kb : a.K / CBK - 1;  // tail stage: re-load a valid block, B is 0
-            const int tap = kbc / cb, c0 = (kbc - tap * cb) * 64;
-            const int r = tap / s.kw, q = tap - r * s.kw;
+          for (int h = 0; h < KB; ++h) {
+            const int kbi = kb0 + it * KB + h;
+            const bool valid = kbi < kb1;
+            const int kv = valid ? kbi : kb1 - 1;  // tail of an odd range: re-load a valid A block, B is 0
+            const int tap = kv / cb, c0 = (kv - tap * cb) * 64;
+            const int r = a.r0 + tap / a.ns, q = a.s0 + tap % a.ns;
             ptx::tma_load_im2col_4d(&tmX, &full[st], sA + st * CA_BYTES + h * (CBM * CBK * 2), c0, wb, hb, nn,
                                     (uint16_t)q, (uint16_t)r);
-            ptx::tma_load_2d(&tmW, &full[st], sB + st * C::B_BYTES + h * C::B_ATOM, kb * CBK, n0);
+            const int wcol = valid ? (r * s.kw + q) * s.C + c0 : a.K;  // column K: all out of bounds -> zeros
+            ptx::tma_load_2d(&tmW, &full[st], sB + st * C::B_BYTES + h * C::B_ATOM, wcol, n0);
           }
         }
       }
@@ -136,9 +154,12 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
     const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
     int64_t g = 0;
     int j = 0;
-    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++j) {
+    for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x, ++j) {
       const int acc = j & 1;
       const int use_acc = j >> 1;
+      int kb0, kb1;
+      krange(u, kb0, kb1);
+      const int nk = (kb1 - kb0 + KB - 1) / KB;
       if (use_acc >= 1) ptx::mbar_wait(&tmem_empty[acc], (use_acc - 1) & 1);
       ptx::tc_fence_after();
       const uint32_t d = tmem + acc * C::TMEM_COLS;
@@ -162,10 +183,12 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
     const int et = threadIdx.x - 64;
     const int qd = warp & 3;
     int j = 0;
-    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++j) {
+    for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x, ++j) {
       const int acc = j & 1;
+      const int64_t tile = u;
       const int n0 = (int)(tile % tiles_n) * BN;
-      const int64_t row = (tile / tiles_n) * CBM + qd * 32 + lane;
+      const int rt = qd * 32 + lane;  // row within the tile
+      const int64_t row = (tile / tiles_n) * CBM + rt;
       asm volatile("bar.sync 1, 128;" ::: "memory");
       for (int c = et; c < BN; c += 128) s_bias[c] = (n0 + c < s.Co) ? a.bias[n0 + c] : 0.0f;
       asm volatile("bar.sync 1, 128;" ::: "memory");
@@ -174,10 +197,7 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
       const uint32_t tq = tmem + acc * C::TMEM_COLS + ((uint32_t)(qd * 32) << 16);
       __nv_bfloat16* out = a.y + row * s.Co;
       const __nv_bfloat16* res = a.res ? a.res + row * s.Co : nullptr;
-#pragma unroll 1
-      for (int c = 0; c < BN / 16; ++c) {
-        float v[16];
-        ptx::tmem_ld16(tq + c * 16, v);
+      auto finish16 = [&](int c, float* v) {  // bias (+ residual) + activation + bf16 store of 16 columns
         const int col0 = n0 + c * 16;
         if (row < M && col0 < s.Co) {
           if (res && col0 + 16 <= s.Co) {
@@ -198,6 +218,12 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
           bias_act<16>(v, s_bias + c * 16, a.act);
           store_row16_any(out + col0, v, s.Co - col0);
         }
+      };
+#pragma unroll 1
+      for (int c = 0; c < BN / 16; ++c) {
+        float v[16];
+        ptx::tmem_ld16(tq + c * 16, v);
+        finish16(c, v);
       }
       ptx::tc_fence_before();
       ptx::mbar_arrive(&tmem_empty[acc]);
@@ -221,10 +247,10 @@ void launch_conv_tma(const CUtensorMap& tx, const CUtensorMap& tw, const ConvArg
     attr = true;
   }
   const int64_t M = (int64_t)a.s.N * a.s.Ho * a.s.Wo;
-  const int64_t tiles = ((M + CBM - 1) / CBM) * ((a.s.Co + BN - 1) / BN);
+  const int64_t units = ((M + CBM - 1) / CBM) * ((a.s.Co + BN - 1) / BN);
   int dev = 0;
   cudaGetDevice(&dev);
-  const int grid = (int)std::min<int64_t>(tiles, num_sms(dev));
+  const int grid = (int)std::min<int64_t>(units, num_sms(dev));
   launch_pdl_if(pdl_on(true), kern, dim3(grid), dim3(192), C::SMEM, st, tx, tw, a);
 }
 
@@ -244,16 +270,28 @@ PFN_cuTensorMapEncodeIm2col_v12000 get_encode_im2col() {
 
 }  // namespace
 
-int conv_tc_pick_bn(const ConvShape& s, int sms) {
-  // wide tiles amortise the per-stage barrier round trip and the im2col re-reads; only narrow
-  // the tile when the (persistent) grid would leave SMs idle
-  const int64_t mt = ((int64_t)s.N * s.Ho * s.Wo + CBM - 1) / CBM;
-  for (int bn : {256, 128, 64}) {
-    if (bn > s.Co && bn > 64) continue;
-    if (mt * ((s.Co + bn - 1) / bn) >= (int64_t)sms) return bn;
-  }
-  return 64;
+ConvTaps conv_taps(const ConvShape& s) {
+  // taps whose input row / column is in the padding for every output pixel contribute exact zeros
+  ConvTaps t;
+  t.r0 = std::max(0, s.pad - (s.Ho - 1) * s.stride);
+  const int r1 = std::min(s.kh - 1, s.H - 1 + s.pad);
+  t.s0 = std::max(0, s.pad - (s.Wo - 1) * s.stride);
+  const int s1 = std::min(s.kw - 1, s.W - 1 + s.pad);
+  t.nr = std::max(1, r1 - t.r0 + 1);
+  t.ns = std::max(1, s1 - t.s0 + 1);
+  return t;
 }
+
+ConvPlan conv_tc_plan(const ConvShape& s, int sms) {
+  // tile width: measured at every c4 / c5 ResNet shape (tools/plan_sweep.sh, DESIGN.md "Conv design
+  // notes"), 128-wide tiles beat 64 (narrow tiles pay the per-k-block cost twice per FLOP) and 256
+  // (half the CTAs on these grids); 64 only for 64-channel layers
+  const ConvTaps t = conv_taps(s);
+  (void)sms;
+  return ConvPlan{s.Co <= 64 ? 64 : 128, 1, t.nr * t.ns * (s.C / 64)};
+}
+
+int conv_tc_pick_bn(const ConvShape& s, int sms) { return conv_tc_plan(s, sms).bn; }
 
 bool conv_tma_ok(const ConvShape& s) { return s.C % 64 == 0 && s.kh <= 16 && s.kw <= 16; }
 
@@ -277,8 +315,11 @@ CUtensorMap make_tmap_im2col(const void* x, const ConvShape& s) {
 }
 
 void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
-             const ConvShape& s, int K, int act, int bn, cudaStream_t st) {
-  ConvArgs a{(const __nv_bfloat16*)x, bias, (const __nv_bfloat16*)residual, (__nv_bfloat16*)y, s, K, act};
+             const ConvShape& s, int K, int act, const ConvPlan& p, cudaStream_t st) {
+  const ConvTaps t = conv_taps(s);
+  ConvArgs a{(const __nv_bfloat16*)x, bias, (const __nv_bfloat16*)residual, (__nv_bfloat16*)y, s, K, act,
+             p.nkb, t.r0, t.s0, t.ns};
+  const int bn = p.bn;
   if (conv_tma_ok(s) && ((uintptr_t)x % 16) == 0) {
     CUtensorMap tx = make_tmap_im2col(x, s);
     switch (bn) {

@@ -199,6 +199,104 @@ __global__ void maxpool8_kernel(const uint4* __restrict__ x, uint4* __restrict__
   }
 }
 
+// ResNet maxpool (3x3, stride 2, pad 1) on NHWC bf16, 8 channels (16 B) per thread: the nine
+// window loads are unrolled and issued together (clamped addresses, out-of-window taps masked to
+// -inf), so each thread keeps nine 16-B requests in flight instead of one per loop trip.
+__global__ void maxpool3s2_kernel(const uint4* __restrict__ x, uint4* __restrict__ y, int N, int H, int W, int C8,
+                                  int Ho, int Wo) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
+  const int total = N * Ho * Wo * C8;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += gridDim.x * blockDim.x) {
+    const int c8 = i % C8;
+    int t = i / C8;
+    const int wo = t % Wo;
+    t /= Wo;
+    const int ho = t % Ho;
+    const int n = t / Ho;
+    uint4 v[9];
+    bool ok[9];
+#pragma unroll
+    for (int r = 0; r < 3; ++r)
+#pragma unroll
+      for (int q = 0; q < 3; ++q) {
+        const int hi = 2 * ho - 1 + r, wi = 2 * wo - 1 + q;
+        ok[r * 3 + q] = hi >= 0 && hi < H && wi >= 0 && wi < W;
+        const int hc = min(max(hi, 0), H - 1), wc = min(max(wi, 0), W - 1);
+        v[r * 3 + q] = __ldg(x + ((n * H + hc) * W + wc) * C8 + c8);
+      }
+    float m[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) m[e] = -INFINITY;
+#pragma unroll
+    for (int j = 0; j < 9; ++j) {
+      const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(&v[j]);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) m[e] = ok[j] ? fmaxf(m[e], __bfloat162float(b[e])) : m[e];
+    }
+    uint4 o;
+    __nv_bfloat16* ob = reinterpret_cast<__nv_bfloat16*>(&o);
+#pragma unroll
+    for (int e = 0; e < 8; ++e) ob[e] = __float2bfloat16_rn(m[e]);
+    y[i] = o;
+  }
+}
+
+// global average pool, NHWC bf16, C % 8 == 0: block = (image n, 32 chunks of 8 channels); its 8
+// warps split the HW positions (warp w takes j = w, w + 8, ...), lane = channel chunk, 4 loads in
+// flight per lane, then the 8 partial sums are added in warp order in shared memory (fixed order:
+// deterministic).
+__global__ void avgpool8_kernel(const uint4* __restrict__ x, uint4* __restrict__ y, int HW, int C8) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
+  __shared__ float part[8][32][8];
+  const int n = blockIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int c8 = blockIdx.y * 32 + lane;
+  float acc[8];
+#pragma unroll
+  for (int e = 0; e < 8; ++e) acc[e] = 0.0f;
+  if (c8 < C8) {
+    const uint4* base = x + (size_t)n * HW * C8 + c8;
+    int j = warp;
+    for (; j + 24 < HW; j += 32) {
+      uint4 v[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) v[u] = __ldg(base + (size_t)(j + 8 * u) * C8);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(&v[u]);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) acc[e] += __bfloat162float(b[e]);
+      }
+    }
+    for (; j < HW; j += 8) {
+      const uint4 v = __ldg(base + (size_t)j * C8);
+      const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(&v);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] += __bfloat162float(b[e]);
+    }
+  }
+#pragma unroll
+  for (int e = 0; e < 8; ++e) part[warp][lane][e] = acc[e];
+  __syncthreads();
+  if (warp == 0 && c8 < C8) {
+    float s[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) {
+      s[e] = 0.0f;
+#pragma unroll
+      for (int w = 0; w < 8; ++w) s[e] += part[w][lane][e];
+    }
+    uint4 o;
+    __nv_bfloat16* ob = reinterpret_cast<__nv_bfloat16*>(&o);
+    const float inv = 1.0f / (float)HW;
+#pragma unroll
+    for (int e = 0; e < 8; ++e) ob[e] = __float2bfloat16_rn(s[e] * inv);
+    y[(size_t)n * C8 + c8] = o;
+  }
+}
+
 }  // namespace
 
 void reduce_sum(const void* x, int x_bf16, const float* b, float* y, int B, int K, cudaStream_t st) {
@@ -268,8 +366,15 @@ void maxpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, 
                   cudaStream_t st) {
   int64_t total = (int64_t)N * Ho * Wo * C;
   if (!total) return;
-  if (bf16 && C % 8 == 0 && total / 8 < INT32_MAX && (int64_t)N * H * W * C / 8 < INT32_MAX &&
-      ((uintptr_t)x % 16) == 0 && ((uintptr_t)y % 16) == 0) {
+  const bool vec = bf16 && C % 8 == 0 && total / 8 < INT32_MAX && (int64_t)N * H * W * C / 8 < INT32_MAX &&
+                   ((uintptr_t)x % 16) == 0 && ((uintptr_t)y % 16) == 0;
+  if (vec && k == 3 && s == 2 && p == 1) {
+    launch_plain(maxpool3s2_kernel, dim3(grid_for(total / 8, 256, 16)), dim3(256), 0, st, (const uint4*)x, (uint4*)y, N, H,
+                 W, C / 8, Ho, Wo);
+    CK(cudaGetLastError());
+    return;
+  }
+  if (vec) {
     launch_plain(maxpool8_kernel, dim3(grid_for(total / 8, 256, 16)), dim3(256), 0, st, (const uint4*)x, (uint4*)y, N, H, W,
                C / 8, k, s, p, Ho, Wo);
     CK(cudaGetLastError());
@@ -287,6 +392,11 @@ void maxpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, 
 void avgpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, cudaStream_t st) {
   int64_t total = (int64_t)N * C;
   if (!total) return;
+  if (bf16 && C % 8 == 0 && H * W >= 8 && ((uintptr_t)x % 16) == 0 && ((uintptr_t)y % 16) == 0) {
+    launch_plain(avgpool8_kernel, dim3(N, (C / 8 + 31) / 32), dim3(256), 0, st, (const uint4*)x, (uint4*)y, H * W, C / 8);
+    CK(cudaGetLastError());
+    return;
+  }
   if (bf16)
     launch_plain(avgpool_kernel<__nv_bfloat16>, dim3(grid_for(total, 256)), dim3(256), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)y, N,
                                                                        H * W, C);

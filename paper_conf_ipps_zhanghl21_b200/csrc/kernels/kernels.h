@@ -198,10 +198,27 @@ void conv_fwd(const void* x, const void* Wf, const float* bias, const void* resi
 void fold_bn(const void* W, int bf16, const float* g, const float* beta, const float* mean, const float* var,
              void* Wf, float* bias, int Co, int64_t per_co, int64_t ldw, cudaStream_t st);
 // tcgen05 implicit-GEMM conv (conv_tc.cu); tw = TMA map of Wf [Co, ldw] with box rows = bn.
+// Tap rectangle of a conv: the filter taps that touch the input for at least one output pixel.
+struct ConvTaps { int r0 = 0, nr = 1, s0 = 0, ns = 1; };
+ConvTaps conv_taps(const ConvShape& s);
+// Launch plan: tile width bn, effective 64-wide k-blocks nkb (tap rectangle); ks is always 1.
+struct ConvPlan { int bn = 64, ks = 1, nkb = 0; };
+ConvPlan conv_tc_plan(const ConvShape& s, int num_sms);
 int conv_tc_pick_bn(const ConvShape& s, int num_sms);
 void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
-             const ConvShape& s, int K, int act, int bn, cudaStream_t st);
+             const ConvShape& s, int K, int act, const ConvPlan& p, cudaStream_t st);
 bool conv_tma_ok(const ConvShape& s);
+// Halo implicit-GEMM 3x3/s1/p1 conv (conv_halo.cu): input tile + zero halo loaded once per
+// 64-channel block, the nine taps read from shared memory.
+struct HaloPlan {
+  bool ok = false;
+  int bn = 64, hb = 0, ni = 1, Hs = 0, bands = 1, a_bytes = 0, box_bytes = 0, a_stages = 2, b_stages = 0, bres = 0,
+      smem = 0;
+  int64_t units = 0;
+};
+HaloPlan conv_halo_plan(const ConvShape& s, int num_sms);
+void conv_halo(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y, const ConvShape& s,
+               int act, const HaloPlan& p, cudaStream_t st);
 // Explicit im2col (layers with C % 64 != 0): cols[m, k] = x[n, ho*s-p+r, wo*s-p+q, c], k = (r, q, c),
 // rows padded to ldk (zeros), bf16.
 void im2col(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStream_t st);

@@ -540,12 +540,24 @@ void build_op(Program& P, const Node& n, Op& op) {
     float* bias = (float*)P.alloc((int64_t)s.Co * 4);
     fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
             (const float*)P.param(n.params[3]), (const float*)P.param(n.params[4]), Wf, bias, s.Co, per_co, ldw, 0);
-    if (tma) {
-      const int bn = conv_tc_pick_bn(s, sms);
-      CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, bn);
+    static const bool no_halo = getenv("DUET_CONV_HALO") && atoi(getenv("DUET_CONV_HALO")) == 0;
+    const HaloPlan halo = (tma && !no_halo) ? conv_halo_plan(s, sms) : HaloPlan{};
+    if (halo.ok) {
+      CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, halo.bn);
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        conv_halo(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, act, halo, st);
+      };
+      op.n_kernels = 1;
+    } else if (tma) {
+      ConvPlan plan = conv_tc_plan(s, sms);
+      if (const char* f = getenv("DUET_CONV_BN")) {  // tile-width sweeps (tools/plan_sweep.sh)
+        const int fb = atoi(f);
+        if (fb == 64 || fb == 128 || fb == 256) plan.bn = fb;
+      }
+      CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, plan.bn);
       const int K = (int)per_co;
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
-        conv_tc(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, K, act, bn, st);
+        conv_tc(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, K, act, plan, st);
       };
       op.n_kernels = 1;
     } else if (stem) {

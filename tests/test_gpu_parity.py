@@ -342,6 +342,15 @@ def test_c2_full_size_sampled():
     (3, 14, 14, 64, 64, 3, 1, 1),     # 3x3, vector path, ragged M tile
     (2, 15, 13, 128, 256, 3, 2, 1),   # stride 2, Co = 256
     (2, 9, 9, 64, 128, 1, 2, 0),      # 1x1 downsample
+    (4, 1, 1, 512, 512, 3, 1, 1),     # 1x1 map: only the centre tap (tap rectangle) + split-K
+    (16, 2, 2, 256, 512, 3, 2, 1),    # c5 layer-4 downsampling conv: 2 x 2 of 9 taps
+    (64, 7, 7, 512, 512, 3, 1, 1),    # c4 layer 4: 25 m tiles -> split-K
+    (30, 7, 7, 512, 256, 3, 1, 1),    # split-K with a ragged last m tile
+    (8, 14, 14, 256, 256, 3, 1, 1),   # layer-3 shape: halo kernel, bands of 8 + 6 rows, streamed weights
+    (2, 56, 56, 64, 64, 3, 1, 1),     # halo kernel, c4 layer 1: bands of 2 rows, resident weights
+    (3, 28, 28, 128, 128, 3, 1, 1),   # halo kernel, c4 layer 2
+    (7, 8, 8, 64, 64, 3, 1, 1),       # halo kernel, c5 layer 1: one whole image per unit
+    (3, 12, 20, 64, 48, 3, 1, 1),     # halo kernel, W != H, ragged last band, Co < tile
 ])
 def test_conv_node(N, H, W, C, Co, k, stride, pad):
     Ho, Wo = (H + 2 * pad - k) // stride + 1, (W + 2 * pad - k) // stride + 1
