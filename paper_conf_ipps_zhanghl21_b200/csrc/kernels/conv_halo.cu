@@ -260,7 +260,7 @@ __global__ void __launch_bounds__(192, 1) conv_halo_kernel(const __grid_constant
 
 }  // namespace
 
-HaloPlan conv_halo_plan(const ConvShape& s, int sms) {
+HaloPlan conv_halo_plan(const ConvShape& s, int sms, bool force) {
   HaloPlan p;
   if (s.stride != 1 || s.kh != 3 || s.kw != 3 || s.pad != 1 || s.C % 64 || s.Co % 16 || s.C > 512) return p;
   const int Wp = s.W + 2;
@@ -280,7 +280,7 @@ HaloPlan conv_halo_plan(const ConvShape& s, int sms) {
   const int bands = ni == 1 ? (s.H + hb - 1) / hb : 1;
   const int64_t groups = ni == 1 ? (int64_t)s.N * bands : ((int64_t)s.N + ni - 1) / ni;
   const double valid = (double)s.N * s.H * s.W / ((double)groups * HBM_ROWS);
-  if (valid < 0.45) return p;
+  if (valid < 0.45 && !force) return p;
   int bn = s.Co <= 64 ? 64 : s.Co <= 128 ? 128 : 256;
   if (bn == 256 && groups * 2 >= sms) bn = 128;  // narrower tiles when there is enough work
   const int box_rows = ni * Hs * Wp;
@@ -299,6 +299,13 @@ HaloPlan conv_halo_plan(const ConvShape& s, int sms) {
   }
   if (a_st < 2 || (!bres && b_st < 3)) return p;
   p.ok = true;
+  // measured (ncu, profiles/r2_conv.md): the halo kernel wins where the weights stay resident and
+  // the band holds >= 2 image rows of >= 16 pixels (c4 layer 1: 40 -> 33 us); with streamed
+  // weights (128-256 channels) or 8 x 8 maps (50% valid rows) the im2col-TMA kernel is faster
+  if ((!bres || s.W < 16) && !force) {
+    p.ok = false;
+    return p;
+  }
   p.bn = bn;
   p.hb = hb;
   p.ni = ni;

@@ -216,7 +216,7 @@ struct HaloPlan {
       smem = 0;
   int64_t units = 0;
 };
-HaloPlan conv_halo_plan(const ConvShape& s, int num_sms);
+HaloPlan conv_halo_plan(const ConvShape& s, int num_sms, bool force = false);
 void conv_halo(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y, const ConvShape& s,
                int act, const HaloPlan& p, cudaStream_t st);
 // Explicit im2col (layers with C % 64 != 0): cols[m, k] = x[n, ho*s-p+r, wo*s-p+q, c], k = (r, q, c),

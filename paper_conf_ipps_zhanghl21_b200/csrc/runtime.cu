@@ -540,8 +540,9 @@ void build_op(Program& P, const Node& n, Op& op) {
     float* bias = (float*)P.alloc((int64_t)s.Co * 4);
     fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
             (const float*)P.param(n.params[3]), (const float*)P.param(n.params[4]), Wf, bias, s.Co, per_co, ldw, 0);
-    static const bool no_halo = getenv("DUET_CONV_HALO") && atoi(getenv("DUET_CONV_HALO")) == 0;
-    const HaloPlan halo = (tma && !no_halo) ? conv_halo_plan(s, sms) : HaloPlan{};
+    // DUET_CONV_HALO: 0 = never, 2 = wherever eligible (tests), default = where measured faster
+    static const int halo_mode = getenv("DUET_CONV_HALO") ? atoi(getenv("DUET_CONV_HALO")) : 1;
+    const HaloPlan halo = (tma && halo_mode) ? conv_halo_plan(s, sms, halo_mode == 2) : HaloPlan{};
     if (halo.ok) {
       CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, halo.bn);
       op.launch = [=](const Ptrs& T, cudaStream_t st) {

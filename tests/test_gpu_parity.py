@@ -342,16 +342,17 @@ def test_c2_full_size_sampled():
     (3, 14, 14, 64, 64, 3, 1, 1),     # 3x3, vector path, ragged M tile
     (2, 15, 13, 128, 256, 3, 2, 1),   # stride 2, Co = 256
     (2, 9, 9, 64, 128, 1, 2, 0),      # 1x1 downsample
-    (4, 1, 1, 512, 512, 3, 1, 1),     # 1x1 map: only the centre tap (tap rectangle) + split-K
+    (4, 1, 1, 512, 512, 3, 1, 1),     # 1x1 map: only the centre tap (tap rectangle)
     (16, 2, 2, 256, 512, 3, 2, 1),    # c5 layer-4 downsampling conv: 2 x 2 of 9 taps
-    (64, 7, 7, 512, 512, 3, 1, 1),    # c4 layer 4: 25 m tiles -> split-K
-    (30, 7, 7, 512, 256, 3, 1, 1),    # split-K with a ragged last m tile
-    (8, 14, 14, 256, 256, 3, 1, 1),   # layer-3 shape: halo kernel, bands of 8 + 6 rows, streamed weights
+    (64, 7, 7, 512, 512, 3, 1, 1),    # c4 layer 4: 25 m tiles
+    (30, 7, 7, 512, 256, 3, 1, 1),    # ragged last m tile
+    (8, 14, 14, 256, 256, 3, 1, 1),   # layer-3 shape
     (2, 56, 56, 64, 64, 3, 1, 1),     # halo kernel, c4 layer 1: bands of 2 rows, resident weights
-    (3, 28, 28, 128, 128, 3, 1, 1),   # halo kernel, c4 layer 2
-    (7, 8, 8, 64, 64, 3, 1, 1),       # halo kernel, c5 layer 1: one whole image per unit
+    (3, 28, 28, 128, 128, 3, 1, 1),   # layer-2 shape
+    (7, 8, 8, 64, 64, 3, 1, 1),       # c5 layer-1 shape
     (3, 12, 20, 64, 48, 3, 1, 1),     # halo kernel, W != H, ragged last band, Co < tile
 ])
+
 def test_conv_node(N, H, W, C, Co, k, stride, pad):
     Ho, Wo = (H + 2 * pad - k) // stride + 1, (W + 2 * pad - k) // stride + 1
     ir = _single_node_graph(
@@ -375,6 +376,30 @@ def test_conv_node(N, H, W, C, Co, k, stride, pad):
     err = rel_err(y.float().cpu().numpy(), want)
     print(f"[parity] conv {N}x{H}x{W}x{C}->{Co} k{k}s{stride}: rel err {err:.3e}")
     assert err <= TOL["bf16"], err
+
+_HALO_SCRIPT = r'''
+import os, sys
+sys.path.insert(0, os.environ["REPO"])
+from tests.test_gpu_parity import test_conv_node
+for case in [(3, 14, 14, 64, 64, 3, 1, 1), (8, 14, 14, 256, 256, 3, 1, 1), (3, 28, 28, 128, 128, 3, 1, 1),
+             (7, 8, 8, 64, 64, 3, 1, 1), (2, 5, 6, 64, 64, 3, 1, 1)]:
+    test_conv_node(*case)
+    print("ok", case)
+'''
+
+
+def test_conv_halo_all_shapes_forced():
+    """The halo kernel on every eligible shape, including those the planner routes to the im2col
+    kernel (streamed weights, 8 x 8 and smaller maps, several whole images per unit): DUET_CONV_HALO=2
+    forces it; a subprocess because the switch is read once."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, DUET_CONV_HALO="2", REPO=root)
+    r = subprocess.run([sys.executable, "-c", _HALO_SCRIPT], env=env, capture_output=True, text=True, timeout=300,
+                       cwd=root)
+    assert r.returncode == 0 and r.stdout.count("ok") == 5, r.stdout[-3000:] + r.stderr[-3000:]
 
 
 @pytest.mark.parametrize("kind,S,B,E,H,dt", [
