@@ -153,6 +153,9 @@ void add_layernorm(const void* a, const void* b, const float* g, const float* be
 // qkv [B*S, 3H] (Q | K | V, head h = columns h*dh..) -> out [B*S, H], softmax(Q K^T / sqrt dh) V per
 // (b, head); S <= 512, dh in {32, 64, 128}, K^T and V (fp32) within 227 KB of shared memory
 bool attention_ok(int S, int dh);
+// tcgen05 attention (attention_tc.cu): bf16, dh = 64, S <= 128; one CTA per (sequence, head)
+bool attention_tc_ok(int S, int dh, int bf16);
+void attention_tc(const void* qkv, void* out, int B, int S, int heads, cudaStream_t st);
 void attention(const void* qkv, void* out, int bf16, int B, int S, int heads, int dh, cudaStream_t st);
 // y[i] = x[offset + i * stride] (rows of `cols` elements of `esize` bytes)
 void select_rows(const void* x, void* y, int esize, int64_t rows, int64_t cols, int64_t stride, int64_t offset,

@@ -644,7 +644,11 @@ void build_op(Program& P, const Node& n, Op& op) {
     const int B = (int)(x.shape[0] / S), dh = (int)(x.shape[1] / 3 / heads);
     if (!attention_ok(S, dh)) fail(DUET_EUNSUPPORTED, "%" + n.name + ": attention needs S <= 512, dh in {32, 64, 128}, K and V in shared memory");
     const int a = n.arg_nodes[0], bf = n.dtype == kBF16;
-    op.launch = [=](const Ptrs& T, cudaStream_t st) { attention(T[a], T[me], bf, B, S, heads, dh, st); };
+    static const bool no_att_tc = getenv("DUET_ATT_TC") && atoi(getenv("DUET_ATT_TC")) == 0;
+    if (attention_tc_ok(S, dh, bf) && !no_att_tc)
+      op.launch = [=](const Ptrs& T, cudaStream_t st) { attention_tc(T[a], T[me], B, S, heads, st); };
+    else
+      op.launch = [=](const Ptrs& T, cudaStream_t st) { attention(T[a], T[me], bf, B, S, heads, dh, st); };
     op.n_kernels = 1;
   } else if (n.op == "add_layernorm") {
     nargs(2, 2);

@@ -556,9 +556,12 @@ def test_model_variation_full_size_sampled(layers, resnet, ffn):
 
 @pytest.mark.parametrize("B,S,heads,dh,dt", [(2, 40, 2, 64, "bf16"), (1, 128, 12, 64, "bf16"), (3, 77, 3, 32, "f32"),
                                               (2, 300, 2, 64, "bf16"), (1, 5, 4, 32, "f32"),
-                                              (2, 128, 2, 128, "bf16"), (1, 512, 1, 32, "f32")])
+                                              (2, 128, 2, 128, "bf16"), (1, 512, 1, 32, "f32"),
+                                              (4, 128, 12, 64, "bf16"), (3, 1, 2, 64, "bf16"), (5, 100, 3, 64, "bf16")])
 def test_attention_node(B, S, heads, dh, dt):
-    """MT-DNN self-attention against the float64 oracle."""
+    """MT-DNN self-attention against the float64 oracle.  bf16 / dh = 64 /
+    S <= 128 runs the tcgen05 kernel (attention_tc.cu; S = 1, 40, 100, 128, several sequences per
+    launch), the rest the CUDA-core kernel."""
     H = heads * dh
     ir = _single_node_graph(f"%y = attention(%x) {{heads={heads}, seq={S}}} : {dt}[{B * S},{H}]", {},
                             {"x": (dt, (B * S, 3 * H))})
