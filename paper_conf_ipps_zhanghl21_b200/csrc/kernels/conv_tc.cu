@@ -53,6 +53,8 @@ struct ConvArgs {
   int act;
   int nkb;             // effective 64-wide k-blocks: taps in the rectangle x C / 64
   int r0, s0, ns;      // tap rectangle: rows r0.., columns s0 .. s0 + ns - 1
+  unsigned* ctr;       // [2] dynamic tile counter + exit count (zero between launches; the last
+                       // CTA to finish fetching resets both), or null: static tile = block + j grid
 };
 
 // TMA-im2col variant (C % 64 == 0): one thread streams both operands; A tile = 128 consecutive
@@ -69,7 +71,10 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   uint64_t* empty = full + C::STAGES;
   uint64_t* tmem_full = empty + C::STAGES;
   uint64_t* tmem_empty = tmem_full + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_empty + 2);
+  uint64_t* tile_full = tmem_empty + 2;   // [4] producer -> MMA / epilogue: s_tile[slot] is set
+  uint64_t* tile_empty = tile_full + 4;   // [4] MMA + epilogue have read it
+  int* s_tile = reinterpret_cast<int*>(tile_empty + 4);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(s_tile + 4);
   float* s_bias = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(full) + 512);
 
   const ConvShape& s = a.s;
@@ -78,12 +83,8 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
   const int tiles_n = (s.Co + BN - 1) / BN;
   const int64_t n_tiles = ((M + CBM - 1) / CBM) * tiles_n;
-  const int64_t n_units = n_tiles;
   const int cb = s.C / 64;
-  auto krange = [&](int64_t, int& kb0, int& kb1) {
-    kb0 = 0;
-    kb1 = a.nkb;
-  };
+  const int nk = (a.nkb + KB - 1) / KB;
 
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tmX);
@@ -95,6 +96,10 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
     for (int i = 0; i < 2; ++i) {
       ptx::mbar_init(&tmem_full[i], 1);
       ptx::mbar_init(&tmem_empty[i], 128);
+    }
+    for (int i = 0; i < 4; ++i) {
+      ptx::mbar_init(&tile_full[i], 1);
+      ptx::mbar_init(&tile_empty[i], 2);
     }
     ptx::fence_mbar_init();
   }
@@ -112,10 +117,27 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   const uint32_t tmem = *tmem_slot;
   ptx::pdl_trigger();
 
+  // Tiles are handed out dynamically when a.ctr is set: a CTA that finds its SM free early (the
+  // other stream slot's persistent recurrence holds most SMs) keeps taking
+  // tiles instead of owning a fixed share that waits for the late CTAs' SMs.  The producer fetches
+  // tile j into s_tile[j % 4]; the MMA warp and the epilogue read it from there.
   if (warp == 0) {
     if (lane == 0) {
       int64_t g = 0;
-      for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x) {
+      for (int j = 0;; ++j) {
+        int64_t u = a.ctr ? (int64_t)atomicAdd(a.ctr, 1u) : (int64_t)blockIdx.x + (int64_t)j * gridDim.x;
+        const int slot = j & 3;
+        if (j >= 4) ptx::mbar_wait(&tile_empty[slot], (uint32_t)(((j >> 2) - 1) & 1));
+        s_tile[slot] = u < n_tiles ? (int)u : -1;
+        ptx::mbar_arrive(&tile_full[slot]);
+        if (u >= n_tiles) {
+          // the last CTA to stop fetching resets the counters for the next launch
+          if (a.ctr && atomicAdd(a.ctr + 1, 1u) == gridDim.x - 1) {
+            a.ctr[0] = 0;
+            a.ctr[1] = 0;
+          }
+          break;
+        }
         const int64_t tile = u;
         const int n0 = (int)(tile % tiles_n) * BN;
         const int64_t m0 = (tile / tiles_n) * CBM;
@@ -124,9 +146,6 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
         const int ho = (int)(q0 % s.Ho);
         const int nn = (int)(q0 / s.Ho);
         const int wb = wo * s.stride - s.pad, hb = ho * s.stride - s.pad;
-        int kb0, kb1;
-        krange(u, kb0, kb1);
-        const int nk = (kb1 - kb0 + KB - 1) / KB;
         for (int it = 0; it < nk; ++it, ++g) {
           const int st = (int)(g % C::STAGES);
           const int64_t use = g / C::STAGES;
@@ -134,9 +153,9 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
           ptx::mbar_arrive_expect_tx(&full[st], C::STAGE);
 #pragma unroll
           for (int h = 0; h < KB; ++h) {
-            const int kbi = kb0 + it * KB + h;
-            const bool valid = kbi < kb1;
-            const int kv = valid ? kbi : kb1 - 1;  // tail of an odd range: re-load a valid A block, B is 0
+            const int kbi = it * KB + h;
+            const bool valid = kbi < a.nkb;
+            const int kv = valid ? kbi : a.nkb - 1;  // tail of an odd range: re-load a valid A block, B is 0
             const int tap = kv / cb, c0 = (kv - tap * cb) * 64;
             const int r = a.r0 + tap / a.ns, q = a.s0 + tap % a.ns;
             ptx::tma_load_im2col_4d(&tmX, &full[st], sA + st * CA_BYTES + h * (CBM * CBK * 2), c0, wb, hb, nn,
@@ -153,13 +172,15 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
     const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
     const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
     int64_t g = 0;
-    int j = 0;
-    for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x, ++j) {
+    for (int j = 0;; ++j) {
+      const int slot = j & 3;
+      ptx::mbar_wait(&tile_full[slot], (uint32_t)((j >> 2) & 1));
+      const int u = s_tile[slot];
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&tile_empty[slot]);
+      if (u < 0) break;
       const int acc = j & 1;
       const int use_acc = j >> 1;
-      int kb0, kb1;
-      krange(u, kb0, kb1);
-      const int nk = (kb1 - kb0 + KB - 1) / KB;
       if (use_acc >= 1) ptx::mbar_wait(&tmem_empty[acc], (use_acc - 1) & 1);
       ptx::tc_fence_after();
       const uint32_t d = tmem + acc * C::TMEM_COLS;
@@ -182,14 +203,18 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   } else {
     const int et = threadIdx.x - 64;
     const int qd = warp & 3;
-    int j = 0;
-    for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x, ++j) {
+    for (int j = 0;; ++j) {
+      const int slot = j & 3;
+      ptx::mbar_wait(&tile_full[slot], (uint32_t)((j >> 2) & 1));
+      const int u = s_tile[slot];
+      asm volatile("bar.sync 1, 128;" ::: "memory");  // every epilogue thread has read s_tile[slot]
+      if (et == 0) ptx::mbar_arrive(&tile_empty[slot]);
+      if (u < 0) break;
       const int acc = j & 1;
       const int64_t tile = u;
       const int n0 = (int)(tile % tiles_n) * BN;
       const int rt = qd * 32 + lane;  // row within the tile
       const int64_t row = (tile / tiles_n) * CBM + rt;
-      asm volatile("bar.sync 1, 128;" ::: "memory");
       for (int c = et; c < BN; c += 128) s_bias[c] = (n0 + c < s.Co) ? a.bias[n0 + c] : 0.0f;
       asm volatile("bar.sync 1, 128;" ::: "memory");
       ptx::mbar_wait(&tmem_full[acc], (j >> 1) & 1);
@@ -315,10 +340,10 @@ CUtensorMap make_tmap_im2col(const void* x, const ConvShape& s) {
 }
 
 void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
-             const ConvShape& s, int K, int act, const ConvPlan& p, cudaStream_t st) {
+             const ConvShape& s, int K, int act, const ConvPlan& p, unsigned* ctr, cudaStream_t st) {
   const ConvTaps t = conv_taps(s);
   ConvArgs a{(const __nv_bfloat16*)x, bias, (const __nv_bfloat16*)residual, (__nv_bfloat16*)y, s, K, act,
-             p.nkb, t.r0, t.s0, t.ns};
+             p.nkb, t.r0, t.s0, t.ns, ctr};
   const int bn = p.bn;
   if (conv_tma_ok(s) && ((uintptr_t)x % 16) == 0) {
     CUtensorMap tx = make_tmap_im2col(x, s);

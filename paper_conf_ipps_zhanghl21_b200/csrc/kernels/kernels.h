@@ -208,8 +208,9 @@ ConvTaps conv_taps(const ConvShape& s);
 struct ConvPlan { int bn = 64, ks = 1, nkb = 0; };
 ConvPlan conv_tc_plan(const ConvShape& s, int num_sms);
 int conv_tc_pick_bn(const ConvShape& s, int num_sms);
+// ctr: [2] zeroed unsigned counters for dynamic tile scheduling (null: static persistent tiles)
 void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
-             const ConvShape& s, int K, int act, const ConvPlan& p, cudaStream_t st);
+             const ConvShape& s, int K, int act, const ConvPlan& p, unsigned* ctr, cudaStream_t st);
 bool conv_tma_ok(const ConvShape& s);
 // Halo implicit-GEMM 3x3/s1/p1 conv (conv_halo.cu): input tile + zero halo loaded once per
 // 64-channel block, the nine taps read from shared memory.
