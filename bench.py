@@ -637,6 +637,10 @@ def bench_shard(args):
     e2e_ms = MR.max_over_ranks(e0.elapsed_time(e1))
     sc, ga = ex.bytes_moved()
     n_launch = duet_s.launch_count()
+    roof = None
+    if rank == 0:  # the dominant kernel at this rank's B / N rows, timed alone and cold
+        flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
+        roof = roofline(torch, args.config, S["wl"], sess, flush)
     if rank == 0:
         line = {"metric": METRIC, "value": round(B * args.steps / (ms / 1e3), 1), "unit": "samples/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -656,7 +660,7 @@ def bench_shard(args):
                         "h2d_bytes_per_step": sum(t.numel() * t.element_size() for t in host_in),
                         "d2h_bytes_per_step": sum(t.numel() * t.element_size() for t in host_out)},
                 "gpu_launches": n_launch * args.steps, "gpu_launches_per_step_per_rank": n_launch,
-                "roofline": None, "cpu_baseline": None, "clocks": clocks}
+                "roofline": roof, "cpu_baseline": None, "clocks": clocks}
         print(json.dumps(line), flush=True)
     MR.finalize()
 

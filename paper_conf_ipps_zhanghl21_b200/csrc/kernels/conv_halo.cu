@@ -48,6 +48,7 @@ struct HaloArgs {
   int box_bytes;   // bytes the halo TMA delivers (zero-filled halo included)
   int a_stages, b_stages;
   int bres;        // weights resident in SMEM
+  unsigned* ctr;   // [2] dynamic unit counter + exit count (null: static units block + j grid)
 };
 
 // SWIZZLE_128B K-major descriptor whose start sits at any 128-B row of a 1024-B aligned buffer the
@@ -76,7 +77,10 @@ __global__ void __launch_bounds__(192, 1) conv_halo_kernel(const __grid_constant
   uint64_t* tmem_full = b_empty + 8;
   uint64_t* tmem_empty = tmem_full + 2;
   uint64_t* w_full = tmem_empty + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(w_full + 1);
+  uint64_t* u_full = w_full + 1;   // [4] unit ring (dynamic scheduling, as conv_tc.cu)
+  uint64_t* u_empty = u_full + 4;  // [4]
+  int* s_unit = reinterpret_cast<int*>(u_empty + 4);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(s_unit + 4);
   float* s_bias = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(a_full) + 512);
 
   const int warp = ptx::warp_id();
@@ -113,6 +117,10 @@ __global__ void __launch_bounds__(192, 1) conv_halo_kernel(const __grid_constant
       ptx::mbar_init(&tmem_empty[i], 128);
     }
     ptx::mbar_init(w_full, 1);
+    for (int i = 0; i < 4; ++i) {
+      ptx::mbar_init(&u_full[i], 1);
+      ptx::mbar_init(&u_empty[i], 2);
+    }
     ptx::fence_mbar_init();
   }
   ptx::pdl_wait();  // before tensor memory is taken
@@ -133,7 +141,19 @@ __global__ void __launch_bounds__(192, 1) conv_halo_kernel(const __grid_constant
         for (int j = 0; j < nkw; ++j) ptx::tma_load_2d(&tmW, w_full, sB + j * B_BLOCK, j * 64, 0);
       }
       int64_t ga = 0, gb = 0;
-      for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x) {
+      for (int j = 0;; ++j) {
+        int64_t u = a.ctr ? (int64_t)atomicAdd(a.ctr, 1u) : (int64_t)blockIdx.x + (int64_t)j * gridDim.x;
+        const int slot = j & 3;
+        if (j >= 4) ptx::mbar_wait(&u_empty[slot], (uint32_t)(((j >> 2) - 1) & 1));
+        s_unit[slot] = u < n_units ? (int)u : -1;
+        ptx::mbar_arrive(&u_full[slot]);
+        if (u >= n_units) {
+          if (a.ctr && atomicAdd(a.ctr + 1, 1u) == gridDim.x - 1) {  // last CTA done fetching: reset
+            a.ctr[0] = 0;
+            a.ctr[1] = 0;
+          }
+          break;
+        }
         int n0, y0, nt;
         unit_geo(u, n0, y0, nt);
         for (int c = 0; c < cb; ++c, ++ga) {
@@ -165,8 +185,12 @@ __global__ void __launch_bounds__(192, 1) conv_halo_kernel(const __grid_constant
     const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
     if (a.bres) ptx::mbar_wait(w_full, 0);
     int64_t ga = 0, gb = 0;
-    int j = 0;
-    for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x, ++j) {
+    for (int j = 0;; ++j) {
+      ptx::mbar_wait(&u_full[j & 3], (uint32_t)((j >> 2) & 1));
+      const int u = s_unit[j & 3];
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&u_empty[j & 3]);
+      if (u < 0) break;
       const int acc = j & 1;
       if ((j >> 1) >= 1) ptx::mbar_wait(&tmem_empty[acc], ((j >> 1) - 1) & 1);
       ptx::tc_fence_after();
@@ -205,13 +229,16 @@ __global__ void __launch_bounds__(192, 1) conv_halo_kernel(const __grid_constant
     const int img = m / img_rows;
     const int yy = (m - img * img_rows) / a.Wp;
     const int xx = m - img * img_rows - yy * a.Wp;
-    int j = 0;
-    for (int64_t u = blockIdx.x; u < n_units; u += gridDim.x, ++j) {
+    for (int j = 0;; ++j) {
+      ptx::mbar_wait(&u_full[j & 3], (uint32_t)((j >> 2) & 1));
+      const int u = s_unit[j & 3];
+      asm volatile("bar.sync 1, 128;" ::: "memory");  // every epilogue thread has read the unit
+      if (et == 0) ptx::mbar_arrive(&u_empty[j & 3]);
+      if (u < 0) break;
       const int acc = j & 1;
       int n0, y0, nt;
       unit_geo(u, n0, y0, nt);
       const int nb = nt * BN;
-      asm volatile("bar.sync 1, 128;" ::: "memory");
       for (int c = et; c < BN; c += 128) s_bias[c] = (nb + c < s.Co) ? a.bias[nb + c] : 0.0f;
       asm volatile("bar.sync 1, 128;" ::: "memory");
       ptx::mbar_wait(&tmem_full[acc], (j >> 1) & 1);
@@ -322,7 +349,7 @@ HaloPlan conv_halo_plan(const ConvShape& s, int sms, bool force) {
 }
 
 void conv_halo(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y, const ConvShape& s,
-               int act, const HaloPlan& p, cudaStream_t st) {
+               int act, const HaloPlan& p, unsigned* ctr, cudaStream_t st) {
   if (!p.ok) fail(DUET_EINVAL, "conv_halo: shape not eligible");
   if (((uintptr_t)x & 15) || ((uintptr_t)y & 15)) fail(DUET_EUNSUPPORTED, "conv_halo: 16-B aligned tensors");
   CUtensorMap tx;
@@ -335,7 +362,7 @@ void conv_halo(const CUtensorMap& tw, const void* x, const float* bias, const vo
                                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) fail(DUET_ECUDA, "conv_halo: cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
   HaloArgs a{nullptr, bias, (const __nv_bfloat16*)residual, (__nv_bfloat16*)y, s, act, s.W + 2, p.Hs, p.hb, p.ni,
-             p.bands, p.a_bytes, p.box_bytes, p.a_stages, p.b_stages, p.bres};
+             p.bands, p.a_bytes, p.box_bytes, p.a_stages, p.b_stages, p.bres, ctr};
   int dev = 0;
   cudaGetDevice(&dev);
   const int grid = (int)std::min<int64_t>(p.units, num_sms(dev));

@@ -61,6 +61,7 @@ struct StemGeom {
   int act;
   int dbg;     // micro-benchmark switches (DUET_STEM_DBG): 1 skip build, 2 skip MMA, 4 skip stores,
                // 8 skip patch TMA (builders use stale patches)
+  unsigned* ctr;  // [2] dynamic tile counter + exit count (null: static tiles block + i grid)
 };
 
 __global__ void stem_pack_kernel(const __nv_bfloat16* __restrict__ wf, int64_t ldw, __nv_bfloat16* __restrict__ wk,
@@ -94,11 +95,15 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint64_t* w_full = a_full + 8;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(w_full + 1);
   float* s_bias = reinterpret_cast<float*>(w_full + 2);
+  // tile of local work item i: s_tile[i % 16] (-1 = no more work), written by the patch issuer,
+  // published through ring_full[i % 16]; the MMA warp and the epilogue each read it and arrive on
+  // ring_empty[i % 16] before the slot is reused
+  __shared__ int s_tile[16];
+  __shared__ uint64_t ring_full[16], ring_empty[16];
 
   const int warp = ptx::warp_id();
   const int lane = threadIdx.x & 31;
   const int tiles = g.N * g.tpi;
-  const int my_tiles = blockIdx.x < tiles ? (tiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
   const uint32_t patch_tx = (uint32_t)pbytes;
 
   if (threadIdx.x == 0) {
@@ -112,6 +117,10 @@ __global__ void __launch_bounds__(THREADS, 1)
       ptx::mbar_init(&t_empty[i], NE);
     }
     ptx::mbar_init(w_full, 1);
+    for (int i = 0; i < 16; ++i) {
+      ptx::mbar_init(&ring_full[i], 1);
+      ptx::mbar_init(&ring_empty[i], 2);
+    }
     ptx::fence_mbar_init();
   }
   // zero both A tiles (rows >= Wo and K >= kh*SEG stay zero for good)
@@ -134,15 +143,28 @@ __global__ void __launch_bounds__(THREADS, 1)
   const uint32_t tmem = *tmem_slot;
   ptx::pdl_trigger();
 
-  auto issue_patch = [&](int i) {  // TMA of local tile i's input rows into patch buffer i % np
-    const int tile = blockIdx.x + i * gridDim.x;
-    const int n = tile / g.tpi, ho = (tile % g.tpi) * g.rp;
+  // Dynamic tile scheduling when g.ctr is set (a CTA whose SM frees up early keeps taking tiles;
+  // see conv_tc.cu): item i's tile is fetched when its patch is issued.  A -1 item still arrives on
+  // patch_full (no TMA) so the builders, then the MMA warp, then the epilogue see the end.
+  auto issue_patch = [&](int i) {  // TMA of local item i's input rows into patch buffer i % np
+    int tile = g.ctr ? (int)atomicAdd(g.ctr, 1u) : (int)(blockIdx.x + i * gridDim.x);
+    if (tile >= tiles) {
+      tile = -1;
+      if (g.ctr && atomicAdd(g.ctr + 1, 1u) == gridDim.x - 1) {  // last CTA done fetching: reset
+        g.ctr[0] = 0;
+        g.ctr[1] = 0;
+      }
+    }
+    if (i >= 16) ptx::mbar_wait(&ring_empty[i & 15], (uint32_t)(((i >> 4) - 1) & 1));
+    s_tile[i & 15] = tile;
+    ptx::mbar_arrive(&ring_full[i & 15]);
     const int pb = i % g.np;
-    uint8_t* dst = sP + pb * pbytes;
-    if (g.dbg & 8) {
+    if (tile < 0 || (g.dbg & 8)) {
       ptx::mbar_arrive(&patch_full[pb]);
       return;
     }
+    const int n = tile / g.tpi, ho = (tile % g.tpi) * g.rp;
+    uint8_t* dst = sP + pb * pbytes;
     ptx::mbar_arrive_expect_tx(&patch_full[pb], patch_tx);
     for (int b = 0; b < g.nbx; ++b)
       ptx::tma_load_3d(&tmX, &patch_full[pb], dst + b * bbytes, b * STEP - g.L, ho * g.stride - g.pad, n);
@@ -154,16 +176,22 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int rr = m / g.Wo, wo = m % g.Wo;   // output row within the tile, column
     const int kh_half = (g.kh + 1) / 2;
     const int r0 = threadIdx.x < ROWS ? 0 : kh_half, r1 = threadIdx.x < ROWS ? kh_half : g.kh;
-    if (threadIdx.x == 0)
-      for (int i = 0; i < g.np && i < my_tiles; ++i) issue_patch(i);
+    if (threadIdx.x == 0) {
+      int i = 0;
+      for (; i < g.np; ++i) {
+        issue_patch(i);
+        if (s_tile[i & 15] < 0) break;
+      }
+    }
     // this pixel's window: box b, element offset o (even: 4-byte aligned words), box row rr*stride
     const int off = g.stride * g.C * wo + g.L - g.pad * g.C - g.d;
     const int src0 = (off / STEP) * bbytes + (off % STEP) * 2 + rr * g.stride * g.rowb;
     const bool live_px = m < g.rp * g.Wo;
-    for (int i = 0; i < my_tiles; ++i) {
+    for (int i = 0;; ++i) {
       const int p = i & 1, pb = i % g.np;
       ptx::mbar_wait(&patch_full[pb], (i / g.np) & 1);
       if (i >= 2) ptx::mbar_wait(&a_empty[p], ((i >> 1) - 1) & 1);
+      if (s_tile[i & 15] < 0) break;  // (visible: the issuer wrote it before arriving on patch_full)
       if (live_px && !(g.dbg & 1)) {
         const uint8_t* prow = sP + pb * pbytes + src0;
         uint8_t* arow = sA + p * A_BYTES + m * 128;
@@ -182,19 +210,27 @@ __global__ void __launch_bounds__(THREADS, 1)
       asm volatile("bar.sync 2, %0;" ::"n"(32 * NB) : "memory");  // A[p] built, patch[p] consumed
       if (threadIdx.x == 0) {
         ptx::mbar_arrive(&a_full[p]);
-        if (i + g.np < my_tiles) issue_patch(i + g.np);
+        // the next item, unless the end was already issued among the items in flight
+        bool ended = false;
+        for (int k = i + 1; k < i + g.np; ++k) ended |= s_tile[k & 15] < 0;
+        if (!ended) issue_patch(i + g.np);
       }
     }
   } else if (warp == NB) {
     // ---------------- MMA issuer ----------------
     // the whole warp walks the loop (uniform descriptors); elect.sync issues each UMMA
-    if (my_tiles > 0) {
+    {
       constexpr uint32_t idesc = ptx::idesc_bf16(ROWS, CO);
       ptx::mbar_wait(w_full, 0);
       const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
       const uint64_t dw0 = ptx::desc_sw128(ptx::smem_u32(sW));
-      for (int i = 0; i < my_tiles; ++i) {
+      for (int i = 0;; ++i) {
         const int b = i & 1;
+        ptx::mbar_wait(&ring_full[i & 15], (uint32_t)((i >> 4) & 1));
+        const int tile = s_tile[i & 15];
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&ring_empty[i & 15]);
+        if (tile < 0) break;
         ptx::mbar_wait(&a_full[b], (i >> 1) & 1);
         if (i >= 2) ptx::mbar_wait(&t_empty[b], ((i >> 1) - 1) & 1);
         ptx::tc_fence_after();
@@ -212,9 +248,13 @@ __global__ void __launch_bounds__(THREADS, 1)
     // ---------------- epilogue ----------------
     const int q = warp & 3;  // TMEM lane quarter of this warp
     const int m = q * 32 + lane;
-    for (int i = 0; i < my_tiles; ++i) {
+    for (int i = 0;; ++i) {
       const int b = i & 1;
-      const int tile = blockIdx.x + i * gridDim.x;
+      ptx::mbar_wait(&ring_full[i & 15], (uint32_t)((i >> 4) & 1));
+      const int tile = s_tile[i & 15];
+      asm volatile("bar.sync 3, %0;" ::"n"(32 * NE) : "memory");  // every epilogue thread has read it
+      if (threadIdx.x == 32 * (NB + 1)) ptx::mbar_arrive(&ring_empty[i & 15]);
+      if (tile < 0) break;
       ptx::mbar_wait(&t_full[b], (i >> 1) & 1);
       ptx::tc_fence_after();
       float v[CO];
@@ -287,7 +327,7 @@ bool conv_stem_ok(const ConvShape& s) {
   if ((s.pad * s.C) % 2 + s.kw * s.C > SEG) return false;      // window fits a segment
   if ((s.stride * s.C) % 2) return false;                        // 4-byte aligned windows
   if ((s.W * s.C) % 8) return false;                             // TMA row pitch (16 B)
-  return stem_smem(geom(s, 0)) <= 227 * 1024;
+  return stem_smem(geom(s, 0)) + 512 <= 227 * 1024;  // + the static tile ring
 }
 
 void conv_stem_pack(const void* wf, int64_t ldw, void* wk, const ConvShape& s, cudaStream_t st) {
@@ -301,8 +341,9 @@ CUtensorMap conv_stem_wmap(const void* wk, int Co) {
 }
 
 void conv_stem(const CUtensorMap& tw, const void* x, const float* bias, void* y, const ConvShape& s, int act,
-               cudaStream_t st) {
-  const StemGeom g = geom(s, act);
+               unsigned* ctr, cudaStream_t st) {
+  StemGeom g = geom(s, act);
+  g.ctr = ctr;
   CUtensorMap tx;
   cuuint64_t dims[3] = {(cuuint64_t)s.W * s.C, (cuuint64_t)s.H, (cuuint64_t)s.N};
   cuuint64_t strides[2] = {(cuuint64_t)s.W * s.C * 2, (cuuint64_t)s.H * s.W * s.C * 2};
@@ -320,7 +361,11 @@ void conv_stem(const CUtensorMap& tw, const void* x, const float* bias, void* y,
 #define DUET_STEM(COV)                                                                           \
   case COV: {                                                                                    \
     auto kern = conv_stem_kernel<COV>;                                                           \
-    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));      \
+    static size_t attr = 0;                                                                      \
+    if (smem > attr) {                                                                           \
+      CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));    \
+      attr = smem;                                                                               \
+    }                                                                                            \
     launch_pdl_if(pdl_on(true), kern, dim3(grid), dim3(THREADS), smem, st, tx, tw, bias,         \
                   (__nv_bfloat16*)y, g);                                                         \
     return;                                                                                      \

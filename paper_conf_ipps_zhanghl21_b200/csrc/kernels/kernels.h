@@ -222,7 +222,7 @@ struct HaloPlan {
 };
 HaloPlan conv_halo_plan(const ConvShape& s, int num_sms, bool force = false);
 void conv_halo(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y, const ConvShape& s,
-               int act, const HaloPlan& p, cudaStream_t st);
+               int act, const HaloPlan& p, unsigned* ctr, cudaStream_t st);  // ctr: as conv_tc
 // Explicit im2col (layers with C % 64 != 0): cols[m, k] = x[n, ho*s-p+r, wo*s-p+q, c], k = (r, q, c),
 // rows padded to ldk (zeros), bf16.
 void im2col(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStream_t st);
@@ -232,7 +232,7 @@ bool conv_stem_ok(const ConvShape& s);
 void conv_stem_pack(const void* wf, int64_t ldw, void* wk, const ConvShape& s, cudaStream_t st);  // wk [Co, 192]
 CUtensorMap conv_stem_wmap(const void* wk, int Co);
 void conv_stem(const CUtensorMap& tw, const void* x, const float* bias, void* y, const ConvShape& s, int act,
-               cudaStream_t st);
+               unsigned* ctr, cudaStream_t st);  // ctr: [2] zeroed counters (dynamic tiles) or null
 
 int num_sms(int device);
 

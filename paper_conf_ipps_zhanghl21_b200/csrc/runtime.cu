@@ -548,10 +548,16 @@ void build_op(Program& P, const Node& n, Op& op) {
     // DUET_CONV_HALO: 0 = never, 2 = wherever eligible (tests), default = where measured faster
     static const int halo_mode = getenv("DUET_CONV_HALO") ? atoi(getenv("DUET_CONV_HALO")) : 1;
     const HaloPlan halo = (tma && halo_mode) ? conv_halo_plan(s, sms, halo_mode == 2) : HaloPlan{};
+    static const bool conv_dyn = !(getenv("DUET_CONV_DYN") && atoi(getenv("DUET_CONV_DYN")) == 0);
     if (halo.ok) {
       CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, halo.bn);
+      unsigned* ctr = nullptr;
+      if (conv_dyn) {
+        ctr = (unsigned*)P.alloc(2 * sizeof(unsigned));
+        CK(cudaMemset(ctr, 0, 2 * sizeof(unsigned)));
+      }
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
-        conv_halo(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, act, halo, st);
+        conv_halo(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, act, halo, ctr, st);
       };
       op.n_kernels = 1;
     } else if (tma) {
@@ -563,9 +569,8 @@ void build_op(Program& P, const Node& n, Op& op) {
       CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, plan.bn);
       const int K = (int)per_co;
       // dynamic tile scheduling (DUET_CONV_DYN=0: static persistent tiles)
-      static const bool dyn = !(getenv("DUET_CONV_DYN") && atoi(getenv("DUET_CONV_DYN")) == 0);
       unsigned* ctr = nullptr;
-      if (dyn) {
+      if (conv_dyn) {
         ctr = (unsigned*)P.alloc(2 * sizeof(unsigned));
         CK(cudaMemset(ctr, 0, 2 * sizeof(unsigned)));
       }
@@ -577,7 +582,12 @@ void build_op(Program& P, const Node& n, Op& op) {
       void* Wk = P.alloc((int64_t)s.Co * 192 * 2);
       conv_stem_pack(Wf, ldw, Wk, s, 0);
       CUtensorMap tw = conv_stem_wmap(Wk, s.Co);
-      op.launch = [=](const Ptrs& T, cudaStream_t st) { conv_stem(tw, T[in], bias, T[dst], s, act, st); };
+      unsigned* ctr = nullptr;
+      if (conv_dyn) {
+        ctr = (unsigned*)P.alloc(2 * sizeof(unsigned));
+        CK(cudaMemset(ctr, 0, 2 * sizeof(unsigned)));
+      }
+      op.launch = [=](const Ptrs& T, cudaStream_t st) { conv_stem(tw, T[in], bias, T[dst], s, act, ctr, st); };
       op.n_kernels = 1;
     } else if (cols) {
       const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
