@@ -91,7 +91,13 @@ struct RnnPersistArgs {
   int tiles_n = 0, tiles_m = 0;       // tile grid: n (gate-block tiles of bn columns) fastest
   int dbg = 0;                        // 1 = per-step timestamps (g_rp_trace)
   int stages = 0;                     // A-ring depth (set by the launcher)
+  int pair = 0;                       // 1: CTA-pair kernel (rnn_pair_kernel; 256 x 256 pair tiles)
+  const void* wcat = nullptr;         // pair: packed weights [w_rows, w_cols] (for its 128-row box)
+  int64_t w_rows = 0, w_cols = 0;
 };
+// CTA-pair recurrence eligibility and grid (2 x pairs) for the several-tiles-per-CTA case.
+bool rnn_pair_ok(int kind, int bn, int B, int tiles_n, int tiles_m, int num_sms);
+int rnn_pair_grid(int tiles_n, int tiles_m, int num_sms);
 // tx: [S*B, E] (box 128 rows), th0/th1: hbuf[0/1] [B, H] (box 128 rows), tw: packed weights
 // [tiles_n*bn, kx*64 + H] (box bn rows).
 void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1,

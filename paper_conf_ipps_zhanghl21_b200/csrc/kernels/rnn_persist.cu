@@ -626,11 +626,346 @@ void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensor
 #undef DUET_RP_CN
 }
 
+
+// ------------------------------------------------------------------------------------------------
+// CTA-pair variant of the several-tiles-per-CTA recurrence (round 2).  The several-tile steps were
+// bound by the bytes each SM can keep in flight: every 64-wide k-block of a 128 x 256 tile moved
+// 16 KB of x/h plus 32 KB of packed weights into one SM, 4 stages of 48 KB filled the shared memory,
+// and at the measured ~1.6 us L2 round trip under load that capped a k-block at ~0.41 us (tensor
+// pipe ~63% of active cycles, tools/rnn_trace_multi.py + ncu, profiles/r2_rnn.md).  Here two CTAs
+// of a cluster form one 256 x 256 pair tile (cta_group::2, UMMA M = 256): each CTA loads its own 128
+// rows of x/h and HALF of the weight rows, so a k-block costs each SM 16 + 16 KB and the ring holds
+// 7 stages.  The leader's MMA warp issues for both; its commits reach both CTAs' barriers (stage
+// free, accumulator ready); both epilogues read their own TMEM (128 rows x all 256 gate columns) and
+// release the accumulator on the leader's barrier.  Tiles, grid barrier and cell math are the
+// several-tile path's.
+constexpr int kPBN = 256;
+constexpr int kPWBytes = (kPBN / 2) * RBK * 2;  // this CTA's half of a weight k-block: 16 KB
+
+template <int KIND>
+__global__ void __launch_bounds__(kRThreads, 1)
+    rnn_pair_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmH0,
+                    const __grid_constant__ CUtensorMap tmH1, const __grid_constant__ CUtensorMap tmW,
+                    const RnnPersistArgs a) {
+  using C = RCfg<kPBN>;
+  constexpr int BN = kPBN;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int STAGES = a.stages;
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + STAGES * R_A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + STAGES * kPWBytes);
+  uint64_t* empty = full + 10;
+  uint64_t* tfull = empty + 10;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = ptx::warp_id();
+  const int lane = threadIdx.x & 31;
+  const int S = a.S, kx = a.kx, kh = a.kh;
+  const uint32_t crank = ptx::cluster_ctarank();
+  const uint32_t rank = crank & 1;
+  const uint32_t leader = crank & ~1u;
+  const int pair = (int)blockIdx.x >> 1, n_pairs = (int)gridDim.x >> 1;
+  const int n_ptiles = a.tiles_n * (a.tiles_m >> 1);
+  const int n_tiles = a.tiles_n * a.tiles_m;  // 128-row CTA tiles (grid-barrier releases per step)
+  const int my_tiles = (n_ptiles - 1 - pair) / n_pairs + 1;
+  auto tile_n0 = [&](int i) { return ((pair + i * n_pairs) % a.tiles_n) * BN; };
+  auto tile_m0 = [&](int i) { return (((pair + i * n_pairs) / a.tiles_n) * 2 + (int)rank) * RBM; };
+  // tools/rnn_trace_multi.py stamps (DUET_RNN_DBG=1), as the one-CTA kernel's
+  unsigned long long* mtr = (a.dbg & 1) && blockIdx.x < 128 ? g_rp_trace + (size_t)blockIdx.x * 64 * 16 : nullptr;
+
+  if (threadIdx.x == 0) {
+    ptx::tma_prefetch(&tmX);
+    ptx::tma_prefetch(&tmH0);
+    ptx::tma_prefetch(&tmH1);
+    ptx::tma_prefetch(&tmW);
+    for (int s = 0; s < STAGES; ++s) {
+      ptx::mbar_init(&full[s], 2);  // leader: A producer + W producer expect the pair's bytes
+      ptx::mbar_init(&empty[s], 1);  // the leader's commit, multicast to both CTAs
+    }
+    for (int b = 0; b < 2; ++b) {
+      ptx::mbar_init(&tfull[b], 1);
+      ptx::mbar_init(&tempty[b], 2 * kREpiWarps);  // leader: both CTAs' epilogue warps
+    }
+    ptx::fence_mbar_init();
+  }
+  ptx::cluster_sync();  // barrier init visible to the peer before any TMA completes on the leader's
+  if (warp == 1) {
+    ptx::tmem_alloc_2sm(tmem_slot, C::TMEM_COLS);
+    ptx::tmem_relinquish_2sm();
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t full_l0 = ptx::mapa(ptx::smem_u32(&full[0]), leader);
+
+  if (warp == 0) {
+    // ---------------- A producer: own 128 rows of x_t, [grid barrier], h_{t-1} ----------------
+    int g = 0;
+    for (int t = 0; t < S; ++t) {
+      const int nkb = kx + (t > 0 ? kh : 0);
+      for (int i = 0; i < my_tiles; ++i) {
+        const int m0 = tile_m0(i);
+        for (int j = 0; j < nkb; ++j, ++g) {
+          const int s = g % STAGES;
+          if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
+          if (j == kx && i == 0) {
+            if (lane == 0) {
+              const unsigned target = (unsigned)t * (unsigned)n_tiles;
+              while (ld_acquire_gpu(a.counter) < target) {
+              }
+              fence_proxy_async_global();
+              if (mtr && t * my_tiles < 64) mtr[(t * my_tiles) * 16 + 0] = rp_gtimer();
+            }
+            __syncwarp();
+          }
+          if (mtr && lane == 0 && j == 0 && t * my_tiles + i < 64) mtr[(t * my_tiles + i) * 16 + 7] = rp_gtimer();
+          if (lane == 0) {
+            const uint32_t fb = full_l0 + s * 8;
+            if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * R_A_BYTES);
+            if (j < kx) {
+              ptx::tma_load_2d_2sm(&tmX, fb, sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
+            } else {  // pre-swizzled 16 KB h block through a SWIZZLE_NONE map (bytes land as stored)
+              ptx::tma_load_2d_2sm(((t - 1) & 1) ? &tmH1 : &tmH0, fb, sA + s * R_A_BYTES, 0, (j - kx) * a.Bp + m0);
+            }
+          }
+          __syncwarp();
+        }
+      }
+    }
+  } else if (warp == kWWarp) {
+    // ---------------- W producer: this CTA's half of each weight k-block ----------------
+    int g = 0;
+    for (int t = 0; t < S; ++t) {
+      const int nkb = kx + (t > 0 ? kh : 0);
+      for (int i = 0; i < my_tiles; ++i) {
+        const int n0 = tile_n0(i);
+        for (int j = 0; j < nkb; ++j, ++g) {
+          const int s = g % STAGES;
+          if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
+          if (mtr && lane == 0 && j == 0 && t * my_tiles + i < 64) mtr[(t * my_tiles + i) * 16 + 11] = rp_gtimer();
+          if (lane == 0) {
+            const uint32_t fb = full_l0 + s * 8;
+            if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * kPWBytes);
+            ptx::tma_load_2d_2sm(&tmW, fb, sB + s * kPWBytes, j * RBK, n0 + (int)rank * (BN / 2));
+          }
+          __syncwarp();
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ---------------- MMA issuer: the leader, for the pair ----------------
+    if (rank == 0) {
+      constexpr uint32_t idesc = ptx::idesc_bf16(2 * RBM, BN);
+      const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
+      const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
+      int g = 0, u = 0;
+      for (int t = 0; t < S; ++t) {
+        const int nkb = kx + (t > 0 ? kh : 0);
+        for (int i = 0; i < my_tiles; ++i, ++u) {
+          const int buf = u & 1;
+          if (u >= 2) wait_sleep(&tempty[buf], ((u >> 1) - 1) & 1);
+          ptx::tc_fence_after();
+          const uint32_t d = tmem + (uint32_t)(buf * BN);
+          for (int j = 0; j < nkb; ++j, ++g) {
+            const int s = g % STAGES;
+            wait_sleep(&full[s], (g / STAGES) & 1);
+            ptx::tc_fence_after();
+            if (mtr && u < 64 && lane == 0) {
+              if (j == 0) mtr[u * 16 + 1] = rp_gtimer();
+              if (j == kx) mtr[u * 16 + 4] = rp_gtimer();
+            }
+            const uint64_t da = da0 + (uint64_t)((s * R_A_BYTES) >> 4);
+            const uint64_t db = db0 + (uint64_t)((s * kPWBytes) >> 4);
+#pragma unroll
+            for (int k = 0; k < RBK / 16; ++k) ptx::umma_bf16_2sm_elect(d, da + 2 * k, db + 2 * k, idesc, (j | k) != 0);
+            ptx::umma_commit_2sm_elect(&empty[s], (uint16_t)(3u << leader));
+          }
+          ptx::umma_commit_2sm_elect(&tfull[buf], (uint16_t)(3u << leader));
+          if (mtr && u < 64 && lane == 0) mtr[u * 16 + 5] = rp_gtimer();
+        }
+      }
+    }
+  } else {
+    // ---------------- epilogue (the several-tile path's, own 128 rows) ----------------
+    constexpr int U = C::U, UH = C::UH;
+    const int q = warp & 3;
+    const int half = (warp - 2) >> 2;
+    const int H = a.H;
+    const uint32_t tempty_l = ptx::mapa(ptx::smem_u32(&tempty[0]), leader);
+    constexpr bool kRegs = KIND == EPI_LSTM;
+    constexpr int RS = kRegs ? UH : 1;
+    const bool regs = kRegs && my_tiles <= 2;
+    float rs0[RS], rs1[RS];
+#pragma unroll
+    for (int k2 = 0; k2 < RS; ++k2) rs0[k2] = rs1[k2] = 0.0f;
+    int u = 0;
+    for (int t = 0; t < S; ++t) {
+      for (int i = 0; i < my_tiles; ++i, ++u) {
+        const int buf = u & 1;
+        const int row = tile_m0(i) + q * 32 + lane;
+        const int n0 = tile_n0(i);
+        float stp[UH / 8][8];
+        {
+          const __nv_bfloat16* hprev = a.hbuf[(t - 1) & 1];
+#pragma unroll
+          for (int c = 0; c < UH / 8; ++c) {
+            const int unit = (n0 / BN) * U + half * UH + 8 * c;
+            if (regs || t == 0 || row >= a.B || unit >= H) {
+#pragma unroll
+              for (int e = 0; e < 8; ++e) stp[c][e] = 0.0f;
+            } else if constexpr (KIND == EPI_LSTM) {
+              const size_t off = (size_t)row * H + unit;
+              const float4 c0 = *reinterpret_cast<const float4*>(a.c_state + off);
+              const float4 c1 = *reinterpret_cast<const float4*>(a.c_state + off + 4);
+              stp[c][0] = c0.x, stp[c][1] = c0.y, stp[c][2] = c0.z, stp[c][3] = c0.w;
+              stp[c][4] = c1.x, stp[c][5] = c1.y, stp[c][6] = c1.z, stp[c][7] = c1.w;
+            } else {
+              const uint4 raw = *reinterpret_cast<const uint4*>(hprev + hs_index(row, unit, a.Bp));
+              const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&raw);
+#pragma unroll
+              for (int e = 0; e < 8; ++e) stp[c][e] = __bfloat162float(hv[e]);
+            }
+          }
+        }
+        wait_sleep(&tfull[buf], (u >> 1) & 1);
+        ptx::tc_fence_after();
+        if (mtr && u < 64 && threadIdx.x == 64) mtr[u * 16 + 2] = rp_gtimer();
+        const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN);
+        float acc[UH / 8][4][8];
+#pragma unroll
+        for (int c = 0; c < UH / 8; ++c) {
+          const uint32_t a0 = tq + half * UH + 8 * c;
+          ptx::tmem_ld8x4(a0, a0 + U, a0 + 2 * U, a0 + 3 * U, acc[c]);
+          if (c == UH / 8 - 1) {  // accumulator buffer read: release it on the leader
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive_cl_relaxed(tempty_l + buf * 8);
+            if (mtr && u < 64 && threadIdx.x == 64) mtr[u * 16 + 6] = rp_gtimer();
+          }
+          const int unit = (n0 / BN) * U + half * UH + 8 * c;
+          if (row >= a.B || unit >= H) continue;
+          const size_t off = (size_t)row * H + unit;
+          float st[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) {
+            if constexpr (kRegs) st[e] = regs ? (i == 0 ? rs0[8 * c + e] : rs1[8 * c + e]) : stp[c][e];
+            else st[e] = stp[c][e];
+          }
+          const int cb = n0 + half * UH + 8 * c;  // packed bias column of gate block 0
+          float h[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e)
+            h[e] = cell<KIND>(acc[c][0][e] + __ldg(a.bias + cb + e), acc[c][1][e] + __ldg(a.bias + cb + U + e),
+                              acc[c][2][e] + __ldg(a.bias + cb + 2 * U + e),
+                              acc[c][3][e] + __ldg(a.bias + cb + 3 * U + e), st[e]);
+          if (regs) {
+            if constexpr (kRegs) {
+#pragma unroll
+              for (int e = 0; e < 8; ++e) {
+                if (i == 0) rs0[8 * c + e] = st[e];
+                else rs1[8 * c + e] = st[e];
+              }
+            }
+          } else if constexpr (KIND == EPI_LSTM) {
+            *reinterpret_cast<float4*>(a.c_state + off) = make_float4(st[0], st[1], st[2], st[3]);
+            *reinterpret_cast<float4*>(a.c_state + off + 4) = make_float4(st[4], st[5], st[6], st[7]);
+          }
+          if (a.seq) store_bf16x8(a.seq + (size_t)t * a.B * H + off, h);
+          if (t == S - 1) store_bf16x8(a.out + off, h);
+          else store_bf16x8(a.hbuf[t & 1] + hs_index(row, unit, a.Bp), h);
+        }
+        if (t < S - 1) {
+          fence_proxy_async_global();
+          asm volatile("bar.sync 1, %0;" ::"n"(32 * kREpiWarps) : "memory");
+          if (threadIdx.x == 64) {
+            red_release_gpu_add(a.counter, 1u);
+            if (mtr && u < 64) mtr[u * 16 + 3] = rp_gtimer();
+          }
+        }
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  ptx::cluster_sync();  // no CTA exits while its peer can still signal its barriers / TMEM
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc_2sm(tmem, C::TMEM_COLS);
+  }
+}
+
+CUtensorMap rp_map_plain(const void* base, int64_t rows) {
+  // [rows, 64] bf16 rows of 128 B, box 128 rows, no swizzle (the h blocks are stored pre-swizzled)
+  CUtensorMap m;
+  cuuint64_t dims[2] = {64, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {128};
+  cuuint32_t box[2] = {64, 128};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = tmap_encode_tiled()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box,
+                                   estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) fail(DUET_ECUDA, "rnn_pair: h tensor map (" + std::to_string((int)r) + ")");
+  return m;
+}
+
+template <int KIND>
+void launch_rp_pair(const CUtensorMap& tx, RnnPersistArgs a, int grid, cudaStream_t st) {
+  auto kern = rnn_pair_kernel<KIND>;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kRSmemBudget));
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+    attr = true;
+  }
+  a.stages = std::min(10, (kRSmemBudget - RCfg<kPBN>::EXTRA) / (R_A_BYTES + kPWBytes));
+  const int smem = a.stages * (R_A_BYTES + kPWBytes) + RCfg<kPBN>::EXTRA;
+  const int64_t hrows = (int64_t)a.kh * a.Bp;
+  const CUtensorMap th0 = rp_map_plain(a.hbuf[0], hrows), th1 = rp_map_plain(a.hbuf[1], hrows);
+  const CUtensorMap tw = make_tmap_bf16_2d(a.wcat, a.w_rows, a.w_cols, kPBN / 2);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kRThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  at[1].id = cudaLaunchAttributeClusterDimension;
+  at[1].val.clusterDim.x = 2;
+  at[1].val.clusterDim.y = 1;
+  at[1].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 2;
+  CK(cudaLaunchKernelEx(&cfg, kern, tx, th0, th1, tw, a));
+}
+
 }  // namespace
+
+bool rnn_pair_ok(int kind, int bn, int B, int tiles_n, int tiles_m, int sms) {
+  // DUET_RNN_PAIR: 0 = never, 2 = LSTM too (tests), default = GRU only -- measured against the
+  // one-CTA kernel on one box: GRU1024 at B = 4096 571 -> 542 us, GRU512 447 -> 447, LSTM512
+  // 503 -> 537
+  static const int mode = getenv("DUET_RNN_PAIR") ? atoi(getenv("DUET_RNN_PAIR")) : 1;
+  if (mode == 0 || (kind == EPI_LSTM && mode != 2)) return false;
+  return bn == kPBN && tiles_m % 2 == 0 && B % 8 == 0 && tiles_n * tiles_m > sms;
+}
+
+int rnn_pair_grid(int tiles_n, int tiles_m, int sms) {
+  // the fewest pairs with the same most-pair-tiles-per-pair as all SMs (cf. the CTA grid)
+  const int pt = tiles_n * (tiles_m / 2), pairs = sms / 2;
+  const int per = (pt + pairs - 1) / pairs;
+  return 2 * ((pt + per - 1) / per);
+}
 
 void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1,
                  const CUtensorMap& tw, const RnnPersistArgs& a_in, int grid, cudaStream_t st) {
   RnnPersistArgs a = a_in;
+  if (a.pair) {
+    if (kind == EPI_LSTM) return launch_rp_pair<EPI_LSTM>(tx, a, grid, st);
+    return launch_rp_pair<EPI_GRU>(tx, a, grid, st);
+  }
   if (kind == EPI_LSTM && bn == 64) return launch_rp_any<64, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_LSTM && bn == 128) return launch_rp_any<128, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_GRU && bn == 64) return launch_rp_any<64, EPI_GRU>(tx, th0, th1, tw, a, grid, st);

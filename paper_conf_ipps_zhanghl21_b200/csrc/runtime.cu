@@ -407,7 +407,11 @@ void build_op(Program& P, const Node& n, Op& op) {
       const int Np = tiles * bn;
       const int Ep = (E + 63) / 64 * 64;
       const int Kc = Ep + H;
-      const int grid = std::min(rp_grid, tiles * mt);
+      // several tiles per CTA with 128 x 256 tiles: the CTA-pair kernel (256 x 256 pair tiles, each
+      // SM loads half the weights; DUET_RNN_PAIR=0 keeps the one-CTA kernel)
+      static const int grid_env2 = getenv("DUET_RNN_GRID") ? atoi(getenv("DUET_RNN_GRID")) : 0;
+      const bool pair = !grid_env2 && rnn_pair_ok(kind, bn, B, tiles, mt, sms);
+      const int grid = pair ? rnn_pair_grid(tiles, mt, sms) : std::min(rp_grid, tiles * mt);
       void* Wcat = P.alloc((int64_t)Np * Kc * 2);
       float* bias = (float*)P.alloc((int64_t)Np * 4);
       unsigned* counter = (unsigned*)P.alloc(256);
@@ -435,6 +439,10 @@ void build_op(Program& P, const Node& n, Op& op) {
       ra.tiles_n = tiles;
       ra.tiles_m = mt;
       ra.dbg = getenv("DUET_RNN_DBG") ? atoi(getenv("DUET_RNN_DBG")) : 0;
+      ra.pair = pair ? 1 : 0;
+      ra.wcat = Wcat;
+      ra.w_rows = Np;
+      ra.w_cols = Kc;
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
         CK(cudaMemsetAsync(counter, 0, sizeof(unsigned), st));
         CUtensorMap tx = make_tmap_bf16_2d(T[in], (int64_t)S * B, E, 128);

@@ -443,6 +443,33 @@ def test_rnn_node(kind, S, B, E, H, dt):
     ("gru", 4, 33, 24, 40, "f32"),        # CUDA-core parity path
 ])
 def test_rnn_node_seq_output(kind, S, B, E, H, dt):
+    rnn_seq_case(kind, S, B, E, H, dt)
+
+
+_PAIR_SCRIPT = r'''
+import os, sys
+sys.path.insert(0, os.environ["REPO"])
+from tests.test_gpu_parity import rnn_seq_case
+for case in [("lstm", 3, 4096, 256, 512, "bf16"), ("gru", 3, 4000, 136, 520, "bf16"), ("lstm", 4, 3840, 128, 264, "bf16")]:
+    rnn_seq_case(*case)
+    print("ok", case)
+'''
+
+
+def test_rnn_pair_lstm_forced():
+    """The CTA-pair recurrence on LSTM (DUET_RNN_PAIR=2; by default only GRU uses it), ragged H,
+    every h_t against the oracle; a subprocess because the switch is read once."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, DUET_RNN_PAIR="2", REPO=root)
+    r = subprocess.run([sys.executable, "-c", _PAIR_SCRIPT], env=env, capture_output=True, text=True, timeout=300,
+                       cwd=root)
+    assert r.returncode == 0 and r.stdout.count("ok") == 3, r.stdout[-3000:] + r.stderr[-3000:]
+
+
+def rnn_seq_case(kind, S, B, E, H, dt):
     """Stacked-RNN lower layer (seq=1, PAPER.md:89 Fig. 14): every h_t, [S, B, H] time-major."""
     G = 4 if kind == "lstm" else 3
     ir = _single_node_graph(
