@@ -150,9 +150,10 @@ def test_state_errors():
     with pytest.raises(duet.DuetError) as e:
         part.profile_from_table([0], [[-1]])
     assert e.value.name == "EINVAL"
-    with pytest.raises(duet.DuetError) as e:
-        duet.Graph("%x = input() : f32[2]\n").partition(batch_shards=2)
-    assert e.value.name == "EUNSUPPORTED"
+    for k in (0, 65):  # batch_shards in [1, 64]
+        with pytest.raises(duet.DuetError) as e:
+            duet.Graph("%x = input() : f32[2]\n").partition(batch_shards=k)
+        assert e.value.name == "EINVAL"
     s = part.profile_from_table([0], [[5]]).schedule()
     with pytest.raises(duet.DuetError) as e:
         s.launch_count()
