@@ -103,26 +103,6 @@ int rnn_pair_grid(int tiles_n, int tiles_m, int num_sms);
 void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1,
                  const CUtensorMap& tw, const RnnPersistArgs& a, int grid, cudaStream_t st);
 
-// Persistent chain of linear layers (mlp_chain.cu): Y_l = act_l(Y_{l-1} W_l^T + b_l), bf16, every
-// N_l % 128 == 0, 256 x 128 tiles on CTA pairs, one cooperative launch for all layers.
-constexpr int kMlpChainMax = 4;
-struct MlpChainMaps {
-  CUtensorMap a[kMlpChainMax];  // layer input [M, K_l] (box 128 rows)
-  CUtensorMap w[kMlpChainMax];  // weights [N_l, K_l] (box 64 rows)
-  CUtensorMap o[kMlpChainMax];  // layer output [M, N_l] (TMA store, box 32 rows x 64 columns)
-};
-struct MlpChainArgs {
-  int L = 0, M = 0, m_blocks = 0;
-  int K[kMlpChainMax] = {}, tiles_n[kMlpChainMax] = {}, act[kMlpChainMax] = {};
-  const float* bias[kMlpChainMax] = {};
-  int item0[kMlpChainMax + 1] = {};  // first work item of each layer (set by mlp_chain)
-  unsigned* done = nullptr;          // [L][m_blocks] tile-completion counters (zeroed per launch)
-  int dbg = 0;                       // 1 = per-item timestamps (g_chain_trace)
-};
-bool mlp_chain_ok(int M, const int* N, const int* K, int L);
-void mlp_chain(const MlpChainMaps& maps, MlpChainArgs a, int sms, cudaStream_t st);
-CUtensorMap mlp_chain_out_map(void* out, int M, int N);
-
 // CTA-pair GEMM with the deep tower's gather-concat fused into the A producer (gemm_tc2.cu):
 // tE = make_tmap_gather4(E, F * R) ([F*R, 64] rows, box 64 x 1, tile::gather4 loads 4 rows each);
 // ep.g_ids / g_F / g_R set; K = 64 F, F <= kGatherMaxF.  bf16 output.

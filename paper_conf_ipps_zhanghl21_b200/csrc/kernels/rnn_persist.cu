@@ -910,8 +910,10 @@ CUtensorMap rp_map_plain(const void* base, int64_t rows) {
   return m;
 }
 
+// false (nothing launched) when the device cannot hold grid / 2 co-resident CTA pairs right now
+// (e.g. under a profiler that reserves SM resources); the caller then runs the one-CTA kernel
 template <int KIND>
-void launch_rp_pair(const CUtensorMap& tx, RnnPersistArgs a, int grid, cudaStream_t st) {
+bool launch_rp_pair(const CUtensorMap& tx, RnnPersistArgs a, int grid, cudaStream_t st) {
   auto kern = rnn_pair_kernel<KIND>;
   static bool attr = false;
   if (!attr) {
@@ -921,6 +923,30 @@ void launch_rp_pair(const CUtensorMap& tx, RnnPersistArgs a, int grid, cudaStrea
   }
   a.stages = std::min(10, (kRSmemBudget - RCfg<kPBN>::EXTRA) / (R_A_BYTES + kPWBytes));
   const int smem = a.stages * (R_A_BYTES + kPWBytes) + RCfg<kPBN>::EXTRA;
+  {
+    static int max_clusters = -1;
+    if (max_clusters < 0) {
+      cudaLaunchConfig_t q{};
+      q.gridDim = dim3(grid);
+      q.blockDim = dim3(kRThreads);
+      q.dynamicSmemBytes = smem;
+      cudaLaunchAttribute ca[1];
+      ca[0].id = cudaLaunchAttributeClusterDimension;
+      ca[0].val.clusterDim.x = 2;
+      ca[0].val.clusterDim.y = 1;
+      ca[0].val.clusterDim.z = 1;
+      q.attrs = ca;
+      q.numAttrs = 1;
+      int n = 0;
+      if (cudaOccupancyMaxActiveClusters(&n, kern, &q) != cudaSuccess) {
+        cudaGetLastError();
+        n = 0;
+      }
+      max_clusters = n;
+      if (getenv("DUET_RNN_DBG")) fprintf(stderr, "[rnn_pair] max active 2-CTA clusters %d (need %d)\n", n, grid / 2);
+    }
+    if (max_clusters < grid / 2) return false;
+  }
   const int64_t hrows = (int64_t)a.kh * a.Bp;
   const CUtensorMap th0 = rp_map_plain(a.hbuf[0], hrows), th1 = rp_map_plain(a.hbuf[1], hrows);
   const CUtensorMap tw = make_tmap_bf16_2d(a.wcat, a.w_rows, a.w_cols, kPBN / 2);
@@ -939,6 +965,7 @@ void launch_rp_pair(const CUtensorMap& tx, RnnPersistArgs a, int grid, cudaStrea
   cfg.attrs = at;
   cfg.numAttrs = 2;
   CK(cudaLaunchKernelEx(&cfg, kern, tx, th0, th1, tw, a));
+  return true;
 }
 
 }  // namespace
@@ -963,8 +990,9 @@ void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0
                  const CUtensorMap& tw, const RnnPersistArgs& a_in, int grid, cudaStream_t st) {
   RnnPersistArgs a = a_in;
   if (a.pair) {
-    if (kind == EPI_LSTM) return launch_rp_pair<EPI_LSTM>(tx, a, grid, st);
-    return launch_rp_pair<EPI_GRU>(tx, a, grid, st);
+    if (kind == EPI_LSTM && launch_rp_pair<EPI_LSTM>(tx, a, grid, st)) return;
+    if (kind == EPI_GRU && launch_rp_pair<EPI_GRU>(tx, a, grid, st)) return;
+    a.pair = 0;  // not co-resident: the one-CTA several-tile kernel, same grid and tiles per CTA
   }
   if (kind == EPI_LSTM && bn == 64) return launch_rp_any<64, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);
   if (kind == EPI_LSTM && bn == 128) return launch_rp_any<128, EPI_LSTM>(tx, th0, th1, tw, a, grid, st);

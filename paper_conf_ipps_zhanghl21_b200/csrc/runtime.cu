@@ -37,8 +37,6 @@ struct Program {
   std::vector<void*> allocs;               // device memory to free
   std::map<int, std::pair<int, int>> fuse_res;  // conv node -> (residual node, add node it writes)
   std::set<int> fused_adds;
-  std::map<int, std::vector<int>> chains;  // head linear node -> chain of linear nodes (mlp_chain.cu)
-  std::map<int, Op> chain_ops;             // head -> one launch for the whole chain
   std::map<int, int> gather_fused;         // linear node -> the gather_concat it absorbs (gemm2 GA)
   std::map<int, int> fused_gathers;        // gather_concat node -> the linear that gathers its rows
   std::map<int, Op> gather_ops;            // linear node -> fused gather + GEMM launch
@@ -841,79 +839,6 @@ void plan_residual_fusion(Program& P) {
   }
 }
 
-// Chains of bf16 linear layers where each layer's only consumer is the next (the deep towers'
-// MLPs): one persistent launch runs the whole chain (kernels/mlp_chain.cu) when every member is in
-// the same subgraph at run time (launch_subgraph).  Intermediate outputs still land in their nodes'
-// buffers.  Opt-in: DUET_MLP_CHAIN=1.
-void plan_linear_chains(Program& P, int sms) {
-  // opt-in: measured slower than per-layer launches on c2 (the cross-CTA dependency hand-off costs
-  // ~3 us per layer boundary: TMA-store completion + release + polling + TMA load latency), see
-  // DESIGN.md "MLP chain"
-  static const int env = getenv("DUET_MLP_CHAIN") ? atoi(getenv("DUET_MLP_CHAIN")) : 0;
-  if (!env) return;
-  const Graph& g = *P.g;
-  std::vector<int> n_cons(g.nodes.size(), 0), consumer(g.nodes.size(), -1);
-  for (auto& n : g.nodes)
-    for (int u : n.inputs) n_cons[u]++, consumer[u] = n.id;
-  std::set<int> outs(g.outputs.begin(), g.outputs.end());
-  auto eligible = [&](const Node& n) {
-    if (n.op != "linear" || n.arg_nodes.size() != 1 || n.params.size() != 2) return false;
-    const Node& x = g.nodes[n.arg_nodes[0]];
-    const auto& w = g.params.at(n.params[0]);
-    return x.dtype == kBF16 && w.dtype == kBF16 && n.dtype == kBF16 && x.shape.size() == 2 && x.shape[0] > 128 &&
-           n.shape[1] % 128 == 0 && x.shape[1] % 8 == 0;
-  };
-  auto next_of = [&](int v) -> int {
-    if (n_cons[v] != 1 || outs.count(v)) return -1;
-    const Node& c = g.nodes[consumer[v]];
-    if (!eligible(c) || c.arg_nodes[0] != v || c.shape[0] != g.nodes[v].shape[0]) return -1;
-    return c.id;
-  };
-  std::set<int> taken;
-  for (int v : g.topo) {
-    if (taken.count(v) || !eligible(g.nodes[v])) continue;
-    std::vector<int> ch{v};
-    for (int c = next_of(v); c >= 0 && (int)ch.size() < kMlpChainMax; c = next_of(c)) ch.push_back(c);
-    if (ch.size() < 2) continue;
-    for (int c : ch) taken.insert(c);
-    P.chains[v] = ch;
-    const int M = (int)g.nodes[v].shape[0];
-    MlpChainArgs a;
-    a.L = (int)ch.size();
-    a.M = M;
-    a.m_blocks = (M + 255) / 256;
-    std::vector<int> ins, Ns, Ks;
-    std::vector<CUtensorMap> wmaps;
-    for (int l = 0; l < a.L; ++l) {
-      const Node& n = g.nodes[ch[l]];
-      const auto& w = g.params.at(n.params[0]);
-      Ns.push_back((int)w.shape[0]);
-      Ks.push_back((int)w.shape[1]);
-      a.K[l] = (int)w.shape[1];
-      a.tiles_n[l] = (int)w.shape[0] / 128;
-      a.act[l] = act_code(n.attr_str("act", "none"));
-      a.bias[l] = (const float*)P.param(n.params[1]);
-      wmaps.push_back(make_tmap_bf16_2d(P.param(n.params[0]), w.shape[0], w.shape[1], 64));
-    }
-    a.done = (unsigned*)P.alloc((int64_t)a.L * a.m_blocks * 4);
-    a.dbg = getenv("DUET_CHAIN_DBG") ? atoi(getenv("DUET_CHAIN_DBG")) : 0;
-    const int in = g.nodes[v].arg_nodes[0];
-    Op op;
-    op.launch = [=](const Ptrs& T, cudaStream_t st) {
-      MlpChainMaps maps;
-      for (int l = 0; l < a.L; ++l) {
-        const void* src = T[l == 0 ? in : ch[l - 1]];
-        maps.a[l] = make_tmap_bf16_2d(src, M, Ks[l], 128);
-        maps.w[l] = wmaps[l];
-        maps.o[l] = mlp_chain_out_map(T[ch[l]], M, Ns[l]);
-      }
-      mlp_chain(maps, a, sms, st);
-    };
-    op.n_kernels = 1;
-    P.chain_ops[v] = op;
-  }
-}
-
 // gather_concat -> linear (the deep tower's first layer, SURVEY.md §8(a) A4 + A5): when the gather's
 // only consumer is a bf16 pair-GEMM linear with D = 64 rows and both sit in the same subgraph at
 // run time, the GEMM's producer warp gathers the embedding rows straight into the swizzled A stages
@@ -925,11 +850,9 @@ void plan_gather_fusion(Program& P, int sms) {
   std::vector<int> n_cons(g.nodes.size(), 0);
   for (auto& n : g.nodes)
     for (int u : n.inputs) n_cons[u]++;
-  std::set<int> outs(g.outputs.begin(), g.outputs.end()), in_chain;
-  for (auto& kv : P.chains)
-    for (int c : kv.second) in_chain.insert(c);
+  std::set<int> outs(g.outputs.begin(), g.outputs.end());
   for (auto& c : g.nodes) {
-    if (c.op != "linear" || c.arg_nodes.size() != 1 || c.params.size() != 2 || in_chain.count(c.id)) continue;
+    if (c.op != "linear" || c.arg_nodes.size() != 1 || c.params.size() != 2) continue;
     const Node& x = g.nodes[c.arg_nodes[0]];
     if (x.op != "gather_concat" || n_cons[x.id] != 1 || outs.count(x.id) || x.params.size() != 1 ||
         P.hash_src.count(x.id))
@@ -985,19 +908,10 @@ std::shared_ptr<Program> ensure_program(Graph* g) {
   plan_residual_fusion(*P);
   plan_hash_fusion(*P);
   for (auto& n : g->nodes) build_op(*P, n, P->ops[n.id]);
-  plan_linear_chains(*P, num_sms(dev));
   plan_gather_fusion(*P, num_sms(dev));
   CK(cudaDeviceSynchronize());
   g->prog = P;
   return P;
-}
-
-bool chain_in_subgraph(const Program& P, const Partition& part, int s, int head) {
-  auto it = P.chains.find(head);
-  if (it == P.chains.end()) return false;
-  for (int c : it->second)
-    if (part.node_to_sg[c] != s) return false;
-  return true;
 }
 
 // the gather is done by its consumer GEMM (plan_gather_fusion) when both run in subgraph s
@@ -1023,11 +937,6 @@ void launch_subgraph(const Program& P, const Partition& part, int s, const Ptrs&
       go->launch(T, st);
       continue;
     }
-    if (chain_in_subgraph(P, part, s, v)) {
-      P.chain_ops.at(v).launch(T, st);
-      for (int c : P.chains.at(v)) skip.insert(c);
-      continue;
-    }
     if (P.ops[v].launch) P.ops[v].launch(T, st);
   }
 }
@@ -1043,11 +952,6 @@ int subgraph_kernels(const Program& P, const Partition& part, int s) {
     }
     if (gathering_linear(P, part, s, v)) {
       nk += 1;
-      continue;
-    }
-    if (chain_in_subgraph(P, part, s, v)) {
-      nk += 1;
-      for (int c : P.chains.at(v)) skip.insert(c);
       continue;
     }
     nk += P.ops[v].n_kernels;

@@ -676,51 +676,6 @@ def test_concurrent_slots_no_deadlock():
     assert r.returncode == 0 and "done" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
 
 
-_CHAIN_SCRIPT = r'''
-import os, sys, numpy as np, torch
-sys.path.insert(0, os.environ["REPO"])
-from oracle import forward as OF
-from paper_conf_ipps_zhanghl21_b200 import duet
-from tests.helpers import rel_err, to_np
-M, K, Ns = 640, 200, [256, 384, 128]
-lines, prev, binds = [f"%x = input() : bf16[{M},{K}]"], ("x", K), {}
-g = torch.Generator().manual_seed(5)
-for i, n in enumerate(Ns):
-    lines = [f"param @W{i} : bf16[{n},{prev[1]}]", f"param @b{i} : f32[{n}]"] + lines
-    lines.append(f"%y{i} = linear(%{prev[0]}, @W{i}, @b{i}) {{act={'relu' if i < 2 else 'none'}}} : bf16[{M},{n}]")
-    binds[f"W{i}"] = ((torch.rand(n, prev[1], generator=g) * 2 - 1) / prev[1] ** 0.5).to(torch.bfloat16)
-    binds[f"b{i}"] = (torch.rand(n, generator=g) * 0.2 - 0.1)
-    prev = (f"y{i}", n)
-ir = "\n".join(lines + [f"output %{prev[0]}"]) + "\n"
-gr = duet.Graph(ir)
-gr.bind_all({k: v.cuda() for k, v in binds.items()})
-s = gr.partition().profile_from_table([0], [[1000]]).schedule()
-x = (torch.rand(M, K, generator=g) * 2 - 1).to(torch.bfloat16)
-y = torch.empty(M, Ns[-1], device="cuda", dtype=torch.bfloat16)
-st = torch.cuda.Stream()
-s.run([(0, st)], [x.cuda()], [y])
-torch.cuda.synchronize()
-assert s.launch_count() == 1, s.launch_count()
-want = OF.run(ir, {k: to_np(v) for k, v in binds.items()}, {"x": to_np(x)})["y2"]
-err = rel_err(y.float().cpu().numpy(), want)
-print("chain rel err", err)
-assert err <= 2e-2, err
-'''
-
-
-def test_mlp_chain_opt_in():
-    """The opt-in persistent MLP chain (DUET_MLP_CHAIN=1, one launch for three linear layers of
-    one subgraph) against the float64 oracle; run in a subprocess because the switch is read once."""
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    env = dict(os.environ, DUET_MLP_CHAIN="1", REPO=root)
-    r = subprocess.run([sys.executable, "-c", _CHAIN_SCRIPT], env=env, capture_output=True, text=True, timeout=300,
-                       cwd=root)
-    assert r.returncode == 0, r.stdout + r.stderr
-
-
 def test_branch_placement_pieces_on_device():
     """SURVEY.md §8(e) item 2: c5's branches placed on 2 GPUs by greedy-correction over one slot per
     GPU, cut into (GPU, phase) pieces, each piece compiled and run by libduet.  On this one-GPU box
