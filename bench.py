@@ -392,7 +392,7 @@ def make_session(args, cfg, local, batch=None):
     torch.cuda.synchronize()
     model_s = sess.schedule(duet.GREEDY_CORRECTION)
     if duet_s is None:
-        duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=30) if args.sched == "measured" else model_s
+        duet_s = sess.schedule(duet.GREEDY_CORRECTION, measured=True, samples=60) if args.sched == "measured" else model_s
     serial_s = base.schedule(duet.SERIAL)
     return dict(wl=wl, sess=sess, base=base, duet_s=duet_s, model_s=model_s, serial_s=serial_s, tile_ns=tile_ns)
 

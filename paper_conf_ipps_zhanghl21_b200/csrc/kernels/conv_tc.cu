@@ -32,12 +32,14 @@ constexpr int CBK = 64;                 // one SWIZZLE_128B atom of K
 constexpr int KB = 2;                   // k-blocks per pipeline stage (halves barrier round trips)
 constexpr int CA_BYTES = KB * CBM * CBK * 2;
 
-template <int BN>
+// OCC CTAs per SM: the stage ring is split between them (two CTAs hide each other's TMA round
+// trips on the 64-channel layers, whose 4-stage ring holds less than one tile)
+template <int BN, int OCC = 1>
 struct ConvCfg {
   static constexpr int B_ATOM = BN * CBK * 2;
   static constexpr int B_BYTES = KB * B_ATOM;
   static constexpr int STAGE = CA_BYTES + B_BYTES;
-  static constexpr int STAGES = (192 * 1024) / STAGE > 8 ? 8 : (192 * 1024) / STAGE;
+  static constexpr int STAGES = (192 * 1024 / OCC) / STAGE > 8 ? 8 : (192 * 1024 / OCC) / STAGE;
   static constexpr int LAG = STAGES - 1;  // cp.async groups kept in flight per producer thread
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;  // x2 (double buffer)
   static constexpr int SMEM = STAGES * STAGE + 1024 + 512 + BN * 4;
@@ -59,10 +61,10 @@ struct ConvArgs {
 
 // TMA-im2col variant (C % 64 == 0): one thread streams both operands; A tile = 128 consecutive
 // output pixels x 64 channels of filter tap (r, s) loaded by one im2col TMA.
-template <int BN>
-__global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant__ CUtensorMap tmX,
-                                                          const __grid_constant__ CUtensorMap tmW, const ConvArgs a) {
-  using C = ConvCfg<BN>;
+template <int BN, int OCC>
+__global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constant__ CUtensorMap tmX,
+                                                            const __grid_constant__ CUtensorMap tmW, const ConvArgs a) {
+  using C = ConvCfg<BN, OCC>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
@@ -262,10 +264,10 @@ __global__ void __launch_bounds__(192, 1) conv_tma_kernel(const __grid_constant_
   }
 }
 
-template <int BN>
+template <int BN, int OCC = 1>
 void launch_conv_tma(const CUtensorMap& tx, const CUtensorMap& tw, const ConvArgs& a, cudaStream_t st) {
-  using C = ConvCfg<BN>;
-  auto kern = conv_tma_kernel<BN>;
+  using C = ConvCfg<BN, OCC>;
+  auto kern = conv_tma_kernel<BN, OCC>;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
@@ -275,7 +277,7 @@ void launch_conv_tma(const CUtensorMap& tx, const CUtensorMap& tw, const ConvArg
   const int64_t units = ((M + CBM - 1) / CBM) * ((a.s.Co + BN - 1) / BN);
   int dev = 0;
   cudaGetDevice(&dev);
-  const int grid = (int)std::min<int64_t>(units, num_sms(dev));
+  const int grid = (int)std::min<int64_t>(units, (int64_t)OCC * num_sms(dev));
   launch_pdl_if(pdl_on(true), kern, dim3(grid), dim3(192), C::SMEM, st, tx, tw, a);
 }
 
@@ -348,7 +350,13 @@ void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void
   if (conv_tma_ok(s) && ((uintptr_t)x % 16) == 0) {
     CUtensorMap tx = make_tmap_im2col(x, s);
     switch (bn) {
-      case 64: return launch_conv_tma<64>(tx, tw, a, st);
+      case 64: {
+        // two CTAs per SM for the 64-channel layers (2 stages each): measured c5 layer 1 (8x8x64,
+        // B = 4096) 70.6 -> 56.9 us, c5 p50 -2.5% (two runs each); DUET_CONV_OCC=1: one CTA, 4 stages
+        static const int occ = getenv("DUET_CONV_OCC") ? atoi(getenv("DUET_CONV_OCC")) : 2;
+        if (occ == 2) return launch_conv_tma<64, 2>(tx, tw, a, st);
+        return launch_conv_tma<64>(tx, tw, a, st);
+      }
       case 128: return launch_conv_tma<128>(tx, tw, a, st);
       case 256: return launch_conv_tma<256>(tx, tw, a, st);
     }

@@ -67,7 +67,7 @@ class Session:
 
 
 def tuned_session(wl: Workload, n_slots: int = 2, device: int = 0, profile: dict | None = None,
-                  tile_candidates=(0, 128), samples: int = 30, mode=duet.GREEDY_CORRECTION):
+                  tile_candidates=(0, 128), samples: int = 60, mode=duet.GREEDY_CORRECTION):
     """Kernel-variant choice by measurement (the compiler-aware profiler's idea, §IV-B:
     each compiled variant is profiled, and the correction's, :81 §IV-C: candidate schedules are
     compared by measured latency).  The variant here is the persistent recurrence's gate-tile width,
