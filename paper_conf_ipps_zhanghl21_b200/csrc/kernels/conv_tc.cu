@@ -29,13 +29,13 @@ namespace {
 
 constexpr int CBM = 128;
 constexpr int CBK = 64;                 // one SWIZZLE_128B atom of K
-constexpr int KB = 2;                   // k-blocks per pipeline stage (halves barrier round trips)
-constexpr int CA_BYTES = KB * CBM * CBK * 2;
 
 // OCC CTAs per SM: the stage ring is split between them (two CTAs hide each other's TMA round
 // trips on the 64-channel layers, whose 4-stage ring holds less than one tile)
-template <int BN, int OCC = 1>
+template <int BN, int OCC = 1, int KB_ = 2>
 struct ConvCfg {
+  static constexpr int KB = KB_;  // k-blocks per pipeline stage (2 halves the barrier round trips)
+  static constexpr int CA_BYTES = KB * CBM * CBK * 2;
   static constexpr int B_ATOM = BN * CBK * 2;
   static constexpr int B_BYTES = KB * B_ATOM;
   static constexpr int STAGE = CA_BYTES + B_BYTES;
@@ -61,10 +61,11 @@ struct ConvArgs {
 
 // TMA-im2col variant (C % 64 == 0): one thread streams both operands; A tile = 128 consecutive
 // output pixels x 64 channels of filter tap (r, s) loaded by one im2col TMA.
-template <int BN, int OCC>
+template <int BN, int OCC, int KB>
 __global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constant__ CUtensorMap tmX,
                                                             const __grid_constant__ CUtensorMap tmW, const ConvArgs a) {
-  using C = ConvCfg<BN, OCC>;
+  using C = ConvCfg<BN, OCC, KB>;
+  constexpr int CA_BYTES = C::CA_BYTES;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
@@ -264,10 +265,10 @@ __global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constan
   }
 }
 
-template <int BN, int OCC = 1>
+template <int BN, int OCC = 1, int KB = 2>
 void launch_conv_tma(const CUtensorMap& tx, const CUtensorMap& tw, const ConvArgs& a, cudaStream_t st) {
-  using C = ConvCfg<BN, OCC>;
-  auto kern = conv_tma_kernel<BN, OCC>;
+  using C = ConvCfg<BN, OCC, KB>;
+  auto kern = conv_tma_kernel<BN, OCC, KB>;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
@@ -357,6 +358,8 @@ void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void
         if (occ == 2) return launch_conv_tma<64, 2>(tx, tw, a, st);
         return launch_conv_tma<64>(tx, tw, a, st);
       }
+      // (two CTAs per SM with one-k-block stages for 128-wide tiles measured -9% .. +18% across
+      // the c4 / c5 shapes and c4 p50 unchanged: not used, profiles/r2_conv.md)
       case 128: return launch_conv_tma<128>(tx, tw, a, st);
       case 256: return launch_conv_tma<256>(tx, tw, a, st);
     }
