@@ -43,15 +43,10 @@ __device__ __forceinline__ int32_t hash_id(int64_t x, int64_t V) {
   return (int32_t)r;
 }
 
-// Where a gather's ids come from: the hash node's int32 output, or (hash absorbed into its gathers,
-// runtime.cu plan_hash_fusion) the raw int64 features hashed on the fly.
+// A gather's ids (the hash node's int32 output), read through the read-only path.
 struct IdSrc {
   const int32_t* ids;
-  const int64_t* raw;
-  int64_t V;
-  __device__ __forceinline__ int32_t operator()(int64_t i) const {
-    return raw ? hash_id(__ldg(raw + i), V) : __ldg(ids + i);
-  }
+  __device__ __forceinline__ int32_t operator()(int64_t i) const { return __ldg(ids + i); }
 };
 
 __global__ void hash_mod_kernel(const int64_t* __restrict__ raw, int32_t* __restrict__ ids, int64_t n, int64_t V) {
@@ -229,9 +224,9 @@ void hash_mod(const int64_t* raw, int32_t* ids, int64_t n, int64_t V, cudaStream
 }
 
 void gather_sum(const int32_t* ids_, const void* T, int t_bf16, const float* b, float* y, int B, int F, int64_t R,
-                cudaStream_t st, const int64_t* raw, int64_t V) {
+                cudaStream_t st) {
   if (B == 0) return;
-  const IdSrc ids{ids_, raw, V};
+  const IdSrc ids{ids_};
   int blocks = (B + 7) / 8;
   if (t_bf16)
     launch_pdl(gather_sum_kernel<__nv_bfloat16>, dim3(blocks), dim3(256), 0, st, ids, (const __nv_bfloat16*)T, b, y, B, F, R);
@@ -273,13 +268,13 @@ static void gather_rows(int mode, const IdSrc idx, const void* tab, int esize, v
 }
 
 void gather_concat(const int32_t* ids, const void* E, int esize, void* X, int B, int F, int64_t R, int D,
-                   cudaStream_t st, const int64_t* raw, int64_t V) {
-  gather_rows(0, IdSrc{ids, raw, V}, E, esize, X, (int64_t)B * F, D, F, R, B, 0, st);
+                   cudaStream_t st) {
+  gather_rows(0, IdSrc{ids}, E, esize, X, (int64_t)B * F, D, F, R, B, 0, st);
 }
 
 void embed_seq(const int32_t* tok, const void* E, int esize, void* X, int B, int S, int64_t V, int D,
                cudaStream_t st) {
-  gather_rows(1, IdSrc{tok, nullptr, 0}, E, esize, X, (int64_t)B * S, D, 1, V, B, S, st);
+  gather_rows(1, IdSrc{tok}, E, esize, X, (int64_t)B * S, D, 1, V, B, S, st);
 }
 
 void fill_random(void* p, int dtype, int64_t n, int64_t high, uint64_t seed, cudaStream_t st) {

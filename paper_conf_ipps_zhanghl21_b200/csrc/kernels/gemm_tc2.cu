@@ -38,7 +38,7 @@ constexpr int KB2 = 2;    // k-blocks per pipeline stage: halves barrier round t
 constexpr int A2_ATOM = BM2 * BK2 * 2;
 constexpr int A2_BYTES = KB2 * A2_ATOM;
 
-template <int BN, bool GA = false>
+template <int BN>
 struct Cfg2 {
   static constexpr int BH = BN / 2;  // W rows per CTA
   static constexpr int B_ATOM = BH * BK2 * 2;
@@ -46,24 +46,17 @@ struct Cfg2 {
   static constexpr int STAGE = A2_BYTES + B_BYTES;
   static constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
-  // GA: + the CTA's gather row coordinates [128][F] (int32)
-  static constexpr int SMEM = STAGES * STAGE + 1024 + 256 + BN * 4 + (GA ? 128 * kGatherMaxF * 4 : 0);
+  static constexpr int SMEM = STAGES * STAGE + 1024 + 256 + BN * 4;
 };
 
-// NP > 1: cluster of 2*NP CTAs = NP pairs along N sharing the A rows.  Each A k-block is split
-// into NP row slices of 128/NP rows; pair p's CTA r loads slice p of its rows and multicasts it
-// to CTA r of every pair, so the cluster reads A from L2 once instead of NP times.  MMA commits go
-// to all 2*NP CTAs so a stage is refilled only after every pair consumed it (empty count NP).
-//
-// GA: A is gathered (the deep tower's gather-concat fused into this GEMM, SURVEY.md §8(a) A4+A5):
-// k-block f of row b is the 128-byte embedding row E[f, ids[b, f]] (D = 64 = one SWIZZLE_128B
-// atom), fetched by tile::gather4 TMA loads of 4 rows each, issued by all 32 lanes of the producer
-// warp from row coordinates f*R + ids[b, f] that the epilogue warps stage in shared memory.
-template <int BN, typename OutT, int NP, bool GA = false>
+// (Round 1 also carried A multicast across pairs, a gathered-A variant fusing the deep tower's
+// gather-concat, and early A loads before the TMEM allocation -- all correct, all measured slower
+// or no faster; removed in round 2.)
+template <int BN, typename OutT>
 __global__ void __launch_bounds__(kThreads2, 1)
     gemm2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                  const __grid_constant__ CUtensorMap tmO, const TcEpilogue ep, int M, int N, int K) {
-  using C = Cfg2<BN, GA>;
+  using C = Cfg2<BN>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
@@ -73,19 +66,15 @@ __global__ void __launch_bounds__(kThreads2, 1)
   uint64_t* tmem_full = empty + C::STAGES;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
   float* s_bias = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(full) + 256);
-  int* s_rows = reinterpret_cast<int*>(s_bias + BN);  // GA: [128][F] gather row coordinates
 
   const int warp = ptx::warp_id();
   const int lane = threadIdx.x & 31;
   const bool tr = (ep.dbg & 32) != 0;
   unsigned long long* trace = g_tc2_trace + 16 * ((blockIdx.y * gridDim.x + blockIdx.x) & 4095);
   if (tr && threadIdx.x == 0) trace[0] = gtimer();
-  constexpr bool MC = NP > 1;
-  constexpr int SLICE = BM2 / NP;  // A rows per multicast slice
   const uint32_t crank = ptx::cluster_ctarank();
   const uint32_t rank = crank & 1;          // rank within the CTA pair
-  const int pair = MC ? (int)(crank >> 1) : 0;
-  const int tile_n = (int)(blockIdx.x / (2 * NP)) * NP + pair;
+  const int tile_n = (int)(blockIdx.x / 2);
   const int n0 = tile_n * BN;
   const int m0 = blockIdx.y * (2 * BM2) + (int)rank * BM2;  // this CTA's rows
   const int nk = (K + KB2 * BK2 - 1) / (KB2 * BK2);  // stages of KB2 k-blocks
@@ -96,7 +85,7 @@ __global__ void __launch_bounds__(kThreads2, 1)
     ptx::tma_prefetch(&tmW);
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
-      ptx::mbar_init(&empty[s], NP);
+      ptx::mbar_init(&empty[s], 1);
     }
     ptx::mbar_init(tmem_full, 1);
     ptx::fence_mbar_init();
@@ -123,16 +112,6 @@ __global__ void __launch_bounds__(kThreads2, 1)
   // two slots)
   ptx::pdl_wait();
   if (tr && threadIdx.x == 0) trace[13] = gtimer();
-  // A tiles of the first stages go out right after the wait, overlapping the TMEM allocation; the
-  // pair-wide barrier below (instead of __syncthreads) then guarantees that both CTAs hold their
-  // TMEM before the leader's MMA warp can pass it (ep.early_a)
-  const int na_early = (ep.early_a && !MC && !(ep.dbg & 2)) ? npre : 0;
-  if (warp == 0 && lane == 0) {
-    for (int kb = 0; kb < na_early; ++kb)
-#pragma unroll
-      for (int h = 0; h < KB2; ++h)
-        ptx::tma_load_2d_2sm(&tmA, full_leader0 + kb * 8, sA + kb * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
-  }
   if (warp == 1) {
     ptx::tmem_alloc_2sm(tmem_slot, C::TMEM_COLS);
     ptx::tmem_relinquish_2sm();
@@ -140,54 +119,15 @@ __global__ void __launch_bounds__(kThreads2, 1)
   }
   ptx::tc_fence_before();
   // A loads (below) follow this CTA's alloc, so the leader's first full barrier implies both CTAs'
-  // TMEM is allocated before the first MMA.  With multicast, a pair receives A slices from the
-  // other pairs, so the whole cluster synchronises instead.
-  if constexpr (MC) {
-    ptx::cluster_sync();
-  } else if (na_early) {
-    // CTA barrier (orders the TMEM address in smem) + relaxed pair barrier (the peer's allocation
-    // happened; tcgen05 fences order it): the .release cluster arrive would wait for the A loads
-    __syncthreads();
-    ptx::cluster_sync_relaxed();
-  } else {
-    __syncthreads();
-  }
+  // TMEM is allocated before the first MMA
+  __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   if (tr && threadIdx.x == 0) trace[1] = gtimer();
   ptx::pdl_trigger();
 
-  if (GA && warp == 0) {
-    // gathered A: wait for the row coordinates, then per stage every lane issues the gather4 loads
-    // of its 4 rows (both k-blocks); lane 0 handles the barrier waits, expect-tx and W tiles
-    const int F = ep.g_F;
-    asm volatile("bar.sync 2, %0;" ::"n"(kEpiThreads2 + 32) : "memory");
-    for (int kb = 0; kb < nk; ++kb) {
-      const int s = kb % C::STAGES;
-      const bool pre = kb < npre && !(ep.dbg & 2);
-      const uint32_t fb = full_leader0 + s * 8;
-      if (lane == 0) {
-        if (kb >= C::STAGES) ptx::mbar_wait(&empty[s], ((kb / C::STAGES) - 1) & 1);
-        if (!pre && rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
-      }
-      __syncwarp();
-#pragma unroll
-      for (int h = 0; h < KB2; ++h) {
-        const int f = kb * KB2 + h;
-        // a k-block past the last field (odd F) re-reads field F-1: the matching W k-block is out of
-        // bounds (K = 64 F), zero-filled by TMA, so it adds nothing
-        const int fc = f < F ? f : F - 1;
-        const int* rr = s_rows + (4 * lane) * F + fc;
-        ptx::tma_gather4_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM + lane * 512, 0, rr[0], rr[F], rr[2 * F],
-                             rr[3 * F]);
-        if (lane == 0 && !pre)
-          ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
-                               n0 + (int)rank * C::BH);
-      }
-    }
-  } else if (warp == 0) {
+  if (warp == 0) {
     if (lane == 0) {
-      const uint16_t a_mask = (uint16_t)((NP == 4 ? 0x55u : NP == 2 ? 0x5u : 0x1u) << rank);  // CTA r of every pair
       for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % C::STAGES;
         const bool pre = kb < npre && !(ep.dbg & 2);
@@ -198,14 +138,9 @@ __global__ void __launch_bounds__(kThreads2, 1)
           continue;
         }
         if (!pre && rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
-        if (kb < na_early) continue;
 #pragma unroll
         for (int h = 0; h < KB2; ++h) {
-          if (!MC)
-            ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
-          else
-            ptx::tma_load_2d_2sm_mc(&tmA, &full[s], sA + s * A2_BYTES + h * A2_ATOM + pair * SLICE * 128,
-                                    (kb * KB2 + h) * BK2, m0 + pair * SLICE, a_mask);
+          ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
           if (!pre)
             ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
                                  n0 + (int)rank * C::BH);
@@ -216,8 +151,8 @@ __global__ void __launch_bounds__(kThreads2, 1)
     if (rank == 0) {
       // the whole warp walks the k loop (uniform descriptors); elect.sync issues each UMMA
       constexpr uint32_t idesc = ptx::idesc_bf16(2 * BM2, BN);
-      const uint16_t empty_mask = (uint16_t)((1u << (2 * NP)) - 1);
-      const uint16_t pair_mask = (uint16_t)(0x3u << (2 * pair));
+      const uint16_t empty_mask = 0x3u;
+      const uint16_t pair_mask = 0x3u;
       const uint64_t da0 = ptx::desc_sw128(ptx::smem_u32(sA));
       const uint64_t db0 = ptx::desc_sw128(ptx::smem_u32(sB));
       for (int kb = 0; kb < nk; ++kb) {
@@ -245,17 +180,6 @@ __global__ void __launch_bounds__(kThreads2, 1)
     // rule); the two warps of a quarter split the columns.  Bias of this tile -> smem first
     // (overlaps the mainloop).
     for (int c = threadIdx.x - 64; c < BN; c += kEpiThreads2) s_bias[c] = (ep.bias && n0 + c < N) ? ep.bias[n0 + c] : 0.0f;
-    if constexpr (GA) {
-      // row coordinates f*R + ids[b, f] of this CTA's 128 rows (rows >= M read row 0 of table f;
-      // their outputs are clipped by the TMA store)
-      const int F = ep.g_F;
-      for (int i = threadIdx.x - 64; i < 128 * F; i += kEpiThreads2) {
-        const int r = i / F, f = i - r * F;
-        const int b = m0 + r;
-        s_rows[i] = f * ep.g_R + (b < M ? __ldg(ep.g_ids + (size_t)b * F + f) : 0);
-      }
-      asm volatile("bar.sync 2, %0;" ::"n"(kEpiThreads2 + 32) : "memory");
-    }
     asm volatile("bar.sync 1, %0;" ::"n"(kEpiThreads2) : "memory");
     if (tr && warp == 2 && lane == 0) trace[15] = gtimer();
     const int q = warp & 3;
@@ -359,27 +283,25 @@ __global__ void __launch_bounds__(kThreads2, 1)
   }
 }
 
-template <int BN, typename OutT, int NP>
+template <int BN, typename OutT>
 void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep_in, int M, int N, int K, cudaStream_t st) {
   using C = Cfg2<BN>;
   static const bool no_tma_store = getenv("DUET_TMA_STORE") && atoi(getenv("DUET_TMA_STORE")) == 0;
   TcEpilogue ep = ep_in;
-  static const int early_a = getenv("DUET_GEMM_EARLY_A") ? atoi(getenv("DUET_GEMM_EARLY_A")) : 0;
-  ep.early_a = early_a;  // opt-in: shorter single launch, but measured slower back to back
   CUtensorMap to{};
   constexpr int EB = (int)sizeof(OutT);
   constexpr int SPAN = (BN / 2) * EB < 128 ? (BN / 2) * EB : 128;
   static_assert(2 * 32 * SPAN * 8 <= C::STAGES * A2_BYTES, "TMA-store staging must fit in the A stages");
   ep.tma_store = !no_tma_store && !(ep.dbg & 8) && SPAN >= 32 &&
                  make_tmap_store_2d(&to, ep.out, EB, M, N, ep.ldo, SPAN);
-  auto kern = gemm2_kernel<BN, OutT, NP>;
+  auto kern = gemm2_kernel<BN, OutT>;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
     attr = true;
   }
   const int tn = (N + BN - 1) / BN;
-  dim3 grid(2 * NP * ((tn + NP - 1) / NP), (M + 2 * BM2 - 1) / (2 * BM2));
+  dim3 grid(2 * tn, (M + 2 * BM2 - 1) / (2 * BM2));
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = grid;
   cfg.blockDim = dim3(kThreads2);
@@ -390,7 +312,7 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep_in
   attr2[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr2[0].val.programmaticStreamSerializationAllowed = no_pdl ? 0 : 1;
   attr2[1].id = cudaLaunchAttributeClusterDimension;
-  attr2[1].val.clusterDim.x = 2 * NP;
+  attr2[1].val.clusterDim.x = 2;
   attr2[1].val.clusterDim.y = 1;
   attr2[1].val.clusterDim.z = 1;
   cfg.attrs = attr2;
@@ -398,71 +320,7 @@ void launch2(const CUtensorMap& a, const CUtensorMap& w, const TcEpilogue& ep_in
   CK(cudaLaunchKernelEx(&cfg, kern, a, w, to, ep, M, N, K));
 }
 
-template <int BN>
-void launch2_gather(const CUtensorMap& tE, const CUtensorMap& w, const TcEpilogue& ep_in, int M, int N, int K,
-                    cudaStream_t st) {
-  using C = Cfg2<BN, true>;
-  TcEpilogue ep = ep_in;
-  ep.early_a = 0;
-  CUtensorMap to{};
-  static_assert(2 * 32 * 128 * 8 <= C::STAGES * A2_BYTES, "TMA-store staging must fit in the A stages");
-  ep.tma_store = make_tmap_store_2d(&to, ep.out, 2, M, N, ep.ldo, (BN / 2) * 2 < 128 ? (BN / 2) * 2 : 128);
-  auto kern = gemm2_kernel<BN, __nv_bfloat16, 1, true>;
-  static bool attr = false;
-  if (!attr) {
-    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
-    attr = true;
-  }
-  cudaLaunchConfig_t cfg{};
-  cfg.gridDim = dim3(2 * ((N + BN - 1) / BN), (M + 2 * BM2 - 1) / (2 * BM2));
-  cfg.blockDim = dim3(kThreads2);
-  cfg.dynamicSmemBytes = C::SMEM;
-  cfg.stream = st;
-  cudaLaunchAttribute at[2];
-  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = pdl_on(true) ? 1 : 0;
-  at[1].id = cudaLaunchAttributeClusterDimension;
-  at[1].val.clusterDim.x = 2;
-  at[1].val.clusterDim.y = 1;
-  at[1].val.clusterDim.z = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = 2;
-  CK(cudaLaunchKernelEx(&cfg, kern, tE, w, to, ep, M, N, K));
-}
-
 }  // namespace
-
-CUtensorMap make_tmap_gather4(const void* E, int64_t rows) {
-  if ((uintptr_t)E & 15) fail(DUET_EUNSUPPORTED, "gather4 table needs a 16-byte aligned base");
-  CUtensorMap m;
-  cuuint64_t dims[2] = {64, (cuuint64_t)rows};
-  cuuint64_t strides[1] = {128};
-  cuuint32_t box[2] = {64, 1};
-  cuuint32_t estr[2] = {1, 1};
-  CUresult r = tmap_encode_tiled()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(E), dims, strides, box,
-                                   estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) fail(DUET_ECUDA, "cuTensorMapEncodeTiled (gather4) failed (" + std::to_string((int)r) + ")");
-  return m;
-}
-
-bool gemm_tc2_gather_ok(int M, int N, int K, int F, int64_t R) {
-  // opt-in (DUET_GATHER_FUSE=1): correct, but tile::gather4 moves 512 B per TMA request and the
-  // per-SM request rate makes the fused fc1 ~3x slower than gather kernel + GEMM
-  static const bool on = getenv("DUET_GATHER_FUSE") && atoi(getenv("DUET_GATHER_FUSE")) == 1;
-  return on && M > 128 && K == 64 * F && F >= 1 && F <= kGatherMaxF && N >= 64 && N % 8 == 0 &&
-         (int64_t)F * R < (int64_t)INT32_MAX;
-}
-
-void gemm_tc2_gather(const CUtensorMap& tE, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
-                     cudaStream_t st) {
-  switch (bn) {
-    case 64: return launch2_gather<64>(tE, tw, ep, M, N, K, st);
-    case 128: return launch2_gather<128>(tE, tw, ep, M, N, K, st);
-    case 256: return launch2_gather<256>(tE, tw, ep, M, N, K, st);
-  }
-  fail(DUET_EUNSUPPORTED, "gemm_tc2_gather: bn must be 64, 128 or 256");
-}
 
 int tc2_pick_bn(int M, int N, int K, int sms) {
   // Widest tile that still occupies ~80% of the SM pairs (measured on B200):
@@ -477,35 +335,15 @@ int tc2_pick_bn(int M, int N, int K, int sms) {
   return 64;
 }
 
-int tc2_pick_np(int M, int N, int bn) {
-  // pairs per cluster sharing A by multicast (1, 2 or 4); DUET_GEMM_MC overrides
-  (void)M;
-  static const int env = getenv("DUET_GEMM_MC") ? atoi(getenv("DUET_GEMM_MC")) : -1;
-  const int tn = (N + bn - 1) / bn;
-  int np = env >= 0 ? env : 1;
-  if (np != 1 && np != 2 && np != 4) np = 1;
-  while (np > 1 && tn % np) np >>= 1;
-  return np;
-}
-
-void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, int np,
-                   const TcEpilogue& ep, int out_bf16, cudaStream_t st) {
-  // `ta` must have been encoded with box rows 128 / np (A multicast slices)
-#define DUET_L2(BNV)                                                                      \
-  if (np == 4)                                                                            \
-    return out_bf16 ? launch2<BNV, __nv_bfloat16, 4>(ta, tw, ep, M, N, K, st)            \
-                    : launch2<BNV, float, 4>(ta, tw, ep, M, N, K, st);                    \
-  if (np == 2)                                                                            \
-    return out_bf16 ? launch2<BNV, __nv_bfloat16, 2>(ta, tw, ep, M, N, K, st)            \
-                    : launch2<BNV, float, 2>(ta, tw, ep, M, N, K, st);                    \
-  return out_bf16 ? launch2<BNV, __nv_bfloat16, 1>(ta, tw, ep, M, N, K, st)              \
-                  : launch2<BNV, float, 1>(ta, tw, ep, M, N, K, st);
+void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
+                   int out_bf16, cudaStream_t st) {
   switch (bn) {
-    case 64: DUET_L2(64)
-    case 128: DUET_L2(128)
-    case 256: DUET_L2(256)
+    case 64: return out_bf16 ? launch2<64, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<64, float>(ta, tw, ep, M, N, K, st);
+    case 128:
+      return out_bf16 ? launch2<128, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<128, float>(ta, tw, ep, M, N, K, st);
+    case 256:
+      return out_bf16 ? launch2<256, __nv_bfloat16>(ta, tw, ep, M, N, K, st) : launch2<256, float>(ta, tw, ep, M, N, K, st);
   }
-#undef DUET_L2
   fail(DUET_EUNSUPPORTED, "gemm_tc2: bn must be 64, 128 or 256");
 }
 

@@ -39,15 +39,10 @@ struct TcEpilogue {
   int kx = 0;                  // k-blocks read from the X map (x_t) before switching to A (h)
   int x_row0 = 0;              // row offset of x_t in the X map ([S*B, E] time-major)
   int tma_store = 0;  // EPI_BIAS_ACT: 1 = output tile leaves through TMA stores (map passed separately)
-  int early_a = 0;  // pair GEMM: issue the first A stages right after the PDL wait (before TMEM alloc)
   // single-CTA GEMM split-K (EPI_BIAS_ACT): grid.z = splits CTAs per tile store raw fp32 partials to
   // ws [splits, M, N]; gemm_splitk_reduce then applies bias + activation
   int splits = 1;
   float* ws = nullptr;
-  // pair GEMM with a gathered A operand (gather-concat fused into the GEMM, gemm2_gather): row b of
-  // A is [E[0, ids[b,0]], ..., E[F-1, ids[b,F-1]]], E = [F, R, 64] bf16, K = 64 F
-  const int32_t* g_ids = nullptr;  // [M, F]
-  int g_F = 0, g_R = 0;
   int dbg = 0;  // micro-benchmark switches: 1 = skip UMMA, 2 = skip TMA, 4 = epilogue backoff
 };
 
@@ -103,20 +98,11 @@ int rnn_pair_grid(int tiles_n, int tiles_m, int num_sms);
 void rnn_persist(int kind, int bn, const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1,
                  const CUtensorMap& tw, const RnnPersistArgs& a, int grid, cudaStream_t st);
 
-// CTA-pair GEMM with the deep tower's gather-concat fused into the A producer (gemm_tc2.cu):
-// tE = make_tmap_gather4(E, F * R) ([F*R, 64] rows, box 64 x 1, tile::gather4 loads 4 rows each);
-// ep.g_ids / g_F / g_R set; K = 64 F, F <= kGatherMaxF.  bf16 output.
-constexpr int kGatherMaxF = 32;
-CUtensorMap make_tmap_gather4(const void* E, int64_t rows);
-bool gemm_tc2_gather_ok(int M, int N, int K, int F, int64_t R);
-void gemm_tc2_gather(const CUtensorMap& tE, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
-                     cudaStream_t st);
 // CTA-pair GEMM (gemm_tc2.cu): 256 x bn tiles, bn in {64,128,256}; W map box rows = bn / 2.
 int tc2_pick_bn(int M, int N, int K, int num_sms);
-// pairs per cluster that share the A tile by TMA multicast (A map box rows = 128 / np)
-int tc2_pick_np(int M, int N, int bn);
-void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, int np,
-                   const TcEpilogue& ep, int out_bf16, cudaStream_t st);
+// A map box rows = 128.
+void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
+                   int out_bf16, cudaStream_t st);
 
 // ---- SIMT fallbacks / small kernels (simt.cu) ----
 // Y[M,N] = act(X[M,K] W[N,K]^T + b) ; X/W dtype per flags; fp32 accumulate.
@@ -149,11 +135,10 @@ void select_rows(const void* x, void* y, int esize, int64_t rows, int64_t cols, 
 
 // ---- gathers (gather.cu) ----
 void hash_mod(const int64_t* raw, int32_t* ids, int64_t n, int64_t V, cudaStream_t st);
-// raw != nullptr: the hash is absorbed (runtime.cu plan_hash_fusion) -- ids = raw mod V on the fly
 void gather_sum(const int32_t* ids, const void* T, int t_bf16, const float* b, float* y, int B, int F, int64_t R,
-                cudaStream_t st, const int64_t* raw = nullptr, int64_t V = 0);
+                cudaStream_t st);
 void gather_concat(const int32_t* ids, const void* E, int esize, void* X, int B, int F, int64_t R, int D,
-                   cudaStream_t st, const int64_t* raw = nullptr, int64_t V = 0);
+                   cudaStream_t st);
 void embed_seq(const int32_t* tok, const void* E, int esize, void* X, int B, int S, int64_t V, int D,
                cudaStream_t st);
 void fill_random(void* p, int dtype, int64_t n, int64_t high, uint64_t seed, cudaStream_t st);

@@ -99,32 +99,6 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 
-// same, multicast to every CTA of `mask` (same smem offset, each CTA's own barrier at `bar`'s offset)
-__device__ __forceinline__ void bulk_g2s_mc(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint16_t mask) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], %4;" ::"r"(
-          smem_u32(dst)),
-      "l"((uint64_t)src), "r"(bytes), "r"(smem_u32(bar)), "h"(mask)
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_2d_mc(const CUtensorMap* m, uint64_t* bar, void* dst, int c0, int c1,
-                                               uint16_t mask) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1, {%4, "
-      "%5}], [%2], %3;" ::"r"(smem_u32(dst)),
-      "l"((uint64_t)m), "r"(smem_u32(bar)), "h"(mask), "r"(c0), "r"(c1)
-      : "memory");
-}
-// commit (single-CTA MMA) arriving on the barrier at the same offset in every CTA of `mask`
-__device__ __forceinline__ void umma_commit_mc_elect(uint64_t* bar, uint16_t mask) {
-  asm volatile(
-      "{\n\t.reg .pred e;\n\t"
-      "elect.sync _|e, 0xffffffff;\n\t"
-      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n\t}" ::"r"(
-          smem_u32(bar)),
-      "h"(mask)
-      : "memory");
-}
 
 __device__ __forceinline__ void tma_load_3d(const CUtensorMap* m, uint64_t* bar, void* dst, int c0, int c1, int c2) {
   asm volatile(
@@ -441,27 +415,6 @@ __device__ __forceinline__ void tma_load_2d_2sm(const CUtensorMap* m, uint32_t b
       "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], "
       "[%2];" ::"r"(smem_u32(dst)),
       "l"((uint64_t)m), "r"(bar_cl), "r"(c0), "r"(c1)
-      : "memory");
-}
-// 2-SM gather of 4 rows (tile::gather4): rows r0..r3 of a [rows, cols] map whose box is
-// {cols_box, 1}; the 4 rows land contiguously at dst (swizzled by address like a tile load).
-__device__ __forceinline__ void tma_gather4_2sm(const CUtensorMap* m, uint32_t bar_cl, void* dst, int c0, int r0,
-                                                int r1, int r2, int r3) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes "
-      "[%0], [%1, {%3, %4, %5, %6, %7}], [%2];" ::"r"(smem_u32(dst)),
-      "l"((uint64_t)m), "r"(bar_cl), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3)
-      : "memory");
-}
-// 2-SM TMA with multicast: copies land at the same smem offset in every CTA of `mask`; each
-// destination's transaction bytes complete on its pair leader's barrier (peer bit cleared).
-__device__ __forceinline__ void tma_load_2d_2sm_mc(const CUtensorMap* m, uint64_t* bar, void* dst, int c0, int c1,
-                                                   uint16_t mask) {
-  const uint32_t b = smem_u32(bar) & 0xFEFFFFFFu;
-  asm volatile(
-      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster "
-      "[%0], [%1, {%4, %5}], [%2], %3;" ::"r"(smem_u32(dst)),
-      "l"((uint64_t)m), "r"(b), "h"(mask), "r"(c0), "r"(c1)
       : "memory");
 }
 __device__ __forceinline__ void tmem_alloc_2sm(uint32_t* dst_smem, uint32_t ncols) {

@@ -164,7 +164,7 @@ __device__ __forceinline__ void tmem_ld_n(uint32_t taddr, float* v) {
   else ptx::tmem_ld8(taddr, v);
 }
 
-template <int BN, int KIND, bool WRES, bool MULTI, int CN>
+template <int BN, int KIND, bool WRES, bool MULTI>
 __global__ void __launch_bounds__(kRThreads, 1)
     rnn_persist_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmH0,
                        const __grid_constant__ CUtensorMap tmH1, const __grid_constant__ CUtensorMap tmW,
@@ -207,7 +207,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
     ptx::tma_prefetch(&tmW);
     for (int s = 0; s < STAGES; ++s) {
       ptx::mbar_init(&full[s], WRES ? 1 : 2);  // A producer (+ W producer), each with its tx bytes
-      ptx::mbar_init(&empty[s], CN);  // every CTA of the cluster consumed the (multicast) stage
+      ptx::mbar_init(&empty[s], 1);
     }
     ptx::mbar_init(w_full, 1);
     for (int b = 0; b < 2; ++b) {
@@ -222,13 +222,8 @@ __global__ void __launch_bounds__(kRThreads, 1)
   }
   if (!MULTI)
     for (int c = (int)threadIdx.x - 64; c >= 0 && c < BN; c += 32 * kREpiWarps) s_bias[c] = a.bias[tile_n0(0) + c];
-  // CN > 1: the cluster's CN CTAs are consecutive n-tiles of one row tile and read the same x_t / h
-  // blocks; k-block j is loaded once, by CTA j % CN, and multicast to all (L2 -> SM traffic / CN:
-  // with one load per CTA, 32 SMs pulling the same 128 KB of h_{t-1} saturated the L2 slices)
-  const uint32_t crank = CN > 1 ? ptx::cluster_ctarank() : 0;
-  constexpr uint16_t kMask = (uint16_t)((1u << CN) - 1);
   ptx::tc_fence_before();
-  if constexpr (CN > 1) ptx::cluster_sync(); else __syncthreads();
+  __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
@@ -262,17 +257,11 @@ __global__ void __launch_bounds__(kRThreads, 1)
           if (mtr && lane == 0 && j == 0 && t * my_tiles + i < 64) mtr[(t * my_tiles + i) * 16 + 7] = rp_gtimer();
           if (lane == 0) {
             ptx::mbar_arrive_expect_tx(&full[s], R_A_BYTES);
-            if (CN == 1 || (int)crank == j % CN) {
-              if (j < kx) {
-                if constexpr (CN > 1)
-                  ptx::tma_load_2d_mc(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0, kMask);
-                else
-                  ptx::tma_load_2d(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
-              } else {  // h_{t-1}: one contiguous, pre-swizzled 16 KB block (see hs_index)
-                const __nv_bfloat16* src = a.hbuf[(t - 1) & 1] + ((size_t)(j - kx) * a.Bp + m0) * RBK;
-                if constexpr (CN > 1) ptx::bulk_g2s_mc(sA + s * R_A_BYTES, src, R_A_BYTES, &full[s], kMask);
-                else ptx::bulk_g2s(sA + s * R_A_BYTES, src, R_A_BYTES, &full[s]);
-              }
+            if (j < kx) {
+              ptx::tma_load_2d(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
+            } else {  // h_{t-1}: one contiguous, pre-swizzled 16 KB block (see hs_index)
+              const __nv_bfloat16* src = a.hbuf[(t - 1) & 1] + ((size_t)(j - kx) * a.Bp + m0) * RBK;
+              ptx::bulk_g2s(sA + s * R_A_BYTES, src, R_A_BYTES, &full[s]);
             }
           }
           __syncwarp();
@@ -339,8 +328,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
           if (!(a.dbg & 16))
 #pragma unroll
             for (int k = 0; k < RBK / 16; ++k) ptx::umma_bf16_elect(d, da + 2 * k, db + 2 * k, idesc, (j | k) != 0);
-          if constexpr (CN > 1) ptx::umma_commit_mc_elect(&empty[s], kMask);  // frees the stage cluster-wide
-          else ptx::umma_commit_elect(&empty[s]);
+          ptx::umma_commit_elect(&empty[s]);
         }
         ptx::umma_commit_elect(&tfull[buf]);
         if (trace && t < 64 && lane == 0) trace[t * 16 + 5] = rp_gtimer();  // last UMMA issued
@@ -546,19 +534,18 @@ __global__ void __launch_bounds__(kRThreads, 1)
     }
   }
   ptx::tc_fence_before();
-  // no CTA may exit while a peer can still multicast into its shared memory / arrive on it
-  if constexpr (CN > 1) ptx::cluster_sync(); else __syncthreads();
+  __syncthreads();
   if (warp == 1) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc(tmem, C::TMEM_COLS);
   }
 }
 
-template <int BN, int KIND, bool WRES, bool MULTI, int CN>
+template <int BN, int KIND, bool WRES, bool MULTI>
 void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap& th1, const CUtensorMap& tw,
                const RnnPersistArgs& a, int grid, cudaStream_t st) {
   using C = RCfg<BN>;
-  auto kern = rnn_persist_kernel<BN, KIND, WRES, MULTI, CN>;
+  auto kern = rnn_persist_kernel<BN, KIND, WRES, MULTI>;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kRSmemBudget));
@@ -570,15 +557,11 @@ void launch_rp(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensorMap&
   cfg.blockDim = dim3(kRThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute at[2];
+  cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeCooperative;
   at[0].val.cooperative = 1;
-  at[1].id = cudaLaunchAttributeClusterDimension;
-  at[1].val.clusterDim.x = CN;
-  at[1].val.clusterDim.y = 1;
-  at[1].val.clusterDim.z = 1;
   cfg.attrs = at;
-  cfg.numAttrs = CN > 1 ? 2 : 1;
+  cfg.numAttrs = 1;
   CK(cudaLaunchKernelEx(&cfg, kern, tx, th0, th1, tw, a));
 }
 
@@ -588,7 +571,7 @@ void launch_rp_multi(const CUtensorMap& tx, const CUtensorMap& th0, const CUtens
   // several tiles per CTA: W changes per tile, so it is streamed
   a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
   if (a.stages > 10) a.stages = 10;
-  return launch_rp<BN, KIND, false, true, 1>(tx, th0, th1, tw, a, grid, st);
+  return launch_rp<BN, KIND, false, true>(tx, th0, th1, tw, a, grid, st);
 }
 
 template <int BN, int KIND>
@@ -604,26 +587,11 @@ void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensor
     a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
     if (a.stages > 10) a.stages = 10;
   }
-  // cluster multicast of x_t / h blocks (DUET_RNN_CN = 2/4/8, opt-in): measured h-phase -9% (LSTM
-  // 256x512) / -13% (GRU 64x1024) only -- the per-SM receive rate, not L2, bounds it -- while
-  // clusters of 8 keep c3's two co-scheduled towers from being co-resident (c3 0.38 -> 0.66 ms)
-  static const int cn_env = getenv("DUET_RNN_CN") ? atoi(getenv("DUET_RNN_CN")) : 1;
-  int cn = 1;
-  for (int c : {8, 4, 2})
-    if (c <= cn_env && a.tiles_n % c == 0) {
-      cn = c;
-      break;
-    }
-#define DUET_RP_CN(CNV)                                                                        \
-  if (cn == CNV) {                                                                             \
-    if (wres) return launch_rp<BN, KIND, true, false, CNV>(tx, th0, th1, tw, a, grid, st);     \
-    return launch_rp<BN, KIND, false, false, CNV>(tx, th0, th1, tw, a, grid, st);              \
-  }
-  DUET_RP_CN(8)
-  DUET_RP_CN(4)
-  DUET_RP_CN(2)
-  DUET_RP_CN(1)
-#undef DUET_RP_CN
+  // (TMA multicast of the x_t / h blocks across clusters of 2-8 CTAs was measured in round 1 and
+  // removed in round 2: h phase -9..-13% only, and clusters of 8 keep c3's two towers from being
+  // co-resident, c3 0.38 -> 0.66 ms)
+  if (wres) return launch_rp<BN, KIND, true, false>(tx, th0, th1, tw, a, grid, st);
+  return launch_rp<BN, KIND, false, false>(tx, th0, th1, tw, a, grid, st);
 }
 
 

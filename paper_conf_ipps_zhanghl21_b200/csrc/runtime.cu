@@ -37,12 +37,6 @@ struct Program {
   std::vector<void*> allocs;               // device memory to free
   std::map<int, std::pair<int, int>> fuse_res;  // conv node -> (residual node, add node it writes)
   std::set<int> fused_adds;
-  std::map<int, int> gather_fused;         // linear node -> the gather_concat it absorbs (gemm2 GA)
-  std::map<int, int> fused_gathers;        // gather_concat node -> the linear that gathers its rows
-  std::map<int, Op> gather_ops;            // linear node -> fused gather + GEMM launch
-  std::map<int, std::pair<int, int64_t>> hash_src;  // gather node -> (raw node, V) of the hash it absorbs
-  std::set<int> absorbed_hashes;           // hash_mod nodes recomputed by every consumer gather
-  std::map<int, Op> hash_ops;              // gather node -> launch reading the raw features
   ~Program() {
     int prev = 0;
     cudaGetDevice(&prev);
@@ -168,16 +162,6 @@ void build_op(Program& P, const Node& n, Op& op) {
       gather_sum((const int32_t*)T[in], T0, tb, b, (float*)T[me], B, F, R, st);
     };
     op.n_kernels = 1;
-    auto hs = P.hash_src.find(me);
-    if (hs != P.hash_src.end()) {
-      const int raw = hs->second.first;
-      const int64_t V = hs->second.second;
-      Op& h = P.hash_ops[me];
-      h.launch = [=](const Ptrs& T, cudaStream_t st) {
-        gather_sum(nullptr, T0, tb, b, (float*)T[me], B, F, R, st, (const int64_t*)T[raw], V);
-      };
-      h.n_kernels = 1;
-    }
   } else if (n.op == "gather_concat") {
     nargs(1, 1);
     need_dtype(n, argn(0).dtype, kI32, "ids");
@@ -193,16 +177,6 @@ void build_op(Program& P, const Node& n, Op& op) {
       gather_concat((const int32_t*)T[in], E, es, T[me], B, F, R, D, st);
     };
     op.n_kernels = 1;
-    auto hs = P.hash_src.find(me);
-    if (hs != P.hash_src.end()) {
-      const int raw = hs->second.first;
-      const int64_t V = hs->second.second;
-      Op& h = P.hash_ops[me];
-      h.launch = [=](const Ptrs& T, cudaStream_t st) {
-        gather_concat(nullptr, E, es, T[me], B, F, R, D, st, (const int64_t*)T[raw], V);
-      };
-      h.n_kernels = 1;
-    }
   } else if (n.op == "embed_seq") {
     nargs(1, 1);
     need_dtype(n, argn(0).dtype, kI32, "tokens");
@@ -232,19 +206,18 @@ void build_op(Program& P, const Node& n, Op& op) {
     if (xb && wb && K % 8 == 0 && N >= 16 && pair) {
       const char* bn_env = getenv("DUET_GEMM_BN");
       const int bn = bn_env ? atoi(bn_env) : tc2_pick_bn(M, N, K, sms);
-      const int np = tc2_pick_np(M, N, bn);
       const char* dbg_env = getenv("DUET_GEMM_DBG");
       const int dbg2 = dbg_env ? atoi(dbg_env) : 0;
       CUtensorMap tw = make_tmap_bf16_2d(W, N, K, bn / 2);
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
-        CUtensorMap ta = make_tmap_bf16_2d(T[in], M, K, 128 / np);
+        CUtensorMap ta = make_tmap_bf16_2d(T[in], M, K, 128);
         TcEpilogue ep;
         ep.bias = b;
         ep.out = T[me];
         ep.ldo = N;
         ep.act = act;
         ep.dbg = dbg2;
-        gemm_tc2_maps(ta, tw, M, N, K, bn, np, ep, yb, st);
+        gemm_tc2_maps(ta, tw, M, N, K, bn, ep, yb, st);
       };
     } else if (xb && wb && K % 8 == 0 && N >= 16) {
       const char* dbg_env = getenv("DUET_GEMM_DBG");
@@ -608,7 +581,7 @@ void build_op(Program& P, const Node& n, Op& op) {
         ep.out = T[dst];
         ep.ldo = s.Co;
         ep.act = act;
-        gemm_tc2_maps(ta, tw, (int)M, s.Co, (int)ldw, bn, 1, ep, 1, st);
+        gemm_tc2_maps(ta, tw, (int)M, s.Co, (int)ldw, bn, ep, 1, st);
       };
       op.n_kernels = 2;
     } else {
@@ -781,40 +754,6 @@ void build_op(Program& P, const Node& n, Op& op) {
   }
 }
 
-// hash_mod(%raw){V} whose every consumer is a gather (gather_concat / gather_sum reading it as ids)
-// and which is not a graph output: each gather hashes the raw int64 features itself (one int64 load
-// and a modulo per id), so the hash kernel and its [B, F] ids round trip leave the critical path
-// (c2: hash -> deep gather -> fc1 ...).  Valid under any placement: %raw is a graph input or an
-// earlier node, never produced by the gathers' subgraphs.  The node-level ops (duet_node_run) stay
-// unfused.  Opt-in (DUET_HASH_FUSE=1): measured on c2, p50 unchanged (38.9 vs 39.0 us; the deep
-// gather's int64 reads + modulo eat the saved launch) and e2e worse (63.5 vs 51.3 us: the raw
-// features then need a copy instead of the hash kernel's zero-copy PCIe read); c1 16.4 -> 18.5 us.
-void plan_hash_fusion(Program& P) {
-  static const bool on = getenv("DUET_HASH_FUSE") && atoi(getenv("DUET_HASH_FUSE")) == 1;
-  if (!on) return;
-  const Graph& g = *P.g;
-  std::vector<std::vector<int>> cons(g.nodes.size());
-  for (auto& n : g.nodes)
-    for (int u : n.inputs) cons[u].push_back(n.id);
-  std::set<int> outs(g.outputs.begin(), g.outputs.end());
-  for (auto& h : g.nodes) {
-    if (h.op != "hash_mod" || h.arg_nodes.size() != 1 || outs.count(h.id) || cons[h.id].empty()) continue;
-    const Node& raw = g.nodes[h.arg_nodes[0]];
-    if (raw.dtype != kI64 || raw.shape != h.shape) continue;
-    bool ok = true;
-    for (int c : cons[h.id]) {
-      const Node& cn = g.nodes[c];
-      ok = ok && (cn.op == "gather_concat" || cn.op == "gather_sum") && cn.arg_nodes.size() == 1 &&
-           cn.arg_nodes[0] == h.id;
-    }
-    if (!ok) continue;
-    const int64_t V = h.attr_int("V", 0);
-    if (V <= 0) continue;
-    P.absorbed_hashes.insert(h.id);
-    for (int c : cons[h.id]) P.hash_src[c] = {raw.id, V};
-  }
-}
-
 // add(%a, %b){act} whose later operand (topological rank) is a conv2d_bn with act=none consumed
 // only by this add: the conv's epilogue adds the other operand and applies the add's activation,
 // writing the add's buffer (ResNet BasicBlock tail; no extra HBM round trip).
@@ -839,55 +778,6 @@ void plan_residual_fusion(Program& P) {
   }
 }
 
-// gather_concat -> linear (the deep tower's first layer, SURVEY.md §8(a) A4 + A5): when the gather's
-// only consumer is a bf16 pair-GEMM linear with D = 64 rows and both sit in the same subgraph at
-// run time, the GEMM's producer warp gathers the embedding rows straight into the swizzled A stages
-// (tile::gather4 TMA) -- no [B, 64 F] round trip through HBM and one launch fewer.  The node-level
-// ops stay unfused (duet_node_run, or the two nodes in different subgraphs).  Opt-in
-// (DUET_GATHER_FUSE=1): measured slower than the two kernels (gemm_tc2.cu gemm_tc2_gather_ok).
-void plan_gather_fusion(Program& P, int sms) {
-  const Graph& g = *P.g;
-  std::vector<int> n_cons(g.nodes.size(), 0);
-  for (auto& n : g.nodes)
-    for (int u : n.inputs) n_cons[u]++;
-  std::set<int> outs(g.outputs.begin(), g.outputs.end());
-  for (auto& c : g.nodes) {
-    if (c.op != "linear" || c.arg_nodes.size() != 1 || c.params.size() != 2) continue;
-    const Node& x = g.nodes[c.arg_nodes[0]];
-    if (x.op != "gather_concat" || n_cons[x.id] != 1 || outs.count(x.id) || x.params.size() != 1 ||
-        P.hash_src.count(x.id))
-      continue;
-    const auto& e = g.params.at(x.params[0]);
-    const auto& w = g.params.at(c.params[0]);
-    if (e.dtype != kBF16 || w.dtype != kBF16 || c.dtype != kBF16 || e.shape.size() != 3 || e.shape[2] != 64) continue;
-    const int M = (int)x.shape[0], F = (int)e.shape[0], N = (int)w.shape[0], K = (int)w.shape[1];
-    const int64_t R = e.shape[1];
-    if (!gemm_tc2_gather_ok(M, N, K, F, R)) continue;
-    const char* bn_env = getenv("DUET_GEMM_BN");
-    const int bn = bn_env ? atoi(bn_env) : tc2_pick_bn(M, N, K, sms);
-    CUtensorMap tw = make_tmap_bf16_2d(P.param(c.params[0]), N, K, bn / 2);
-    CUtensorMap tE = make_tmap_gather4(P.param(x.params[0]), (int64_t)F * R);
-    const float* bias = (const float*)P.param(c.params[1]);
-    const int act = act_code(c.attr_str("act", "none"));
-    const int ids = x.arg_nodes[0], me = c.id;
-    Op op;
-    op.launch = [=](const Ptrs& T, cudaStream_t st) {
-      TcEpilogue ep;
-      ep.bias = bias;
-      ep.out = T[me];
-      ep.ldo = N;
-      ep.act = act;
-      ep.g_ids = (const int32_t*)T[ids];
-      ep.g_F = F;
-      ep.g_R = (int)R;
-      gemm_tc2_gather(tE, tw, M, N, K, bn, ep, st);
-    };
-    op.n_kernels = 1;
-    P.gather_fused[c.id] = x.id;
-    P.fused_gathers[x.id] = c.id;
-    P.gather_ops[c.id] = op;
-  }
-}
 
 std::shared_ptr<Program> ensure_program(Graph* g) {
   if (g->prog) return g->prog;
@@ -906,56 +796,20 @@ std::shared_ptr<Program> ensure_program(Graph* g) {
   for (auto& n : g->nodes) P->buf[n.id] = P->alloc(n.nbytes());
   P->ops.resize(g->nodes.size());
   plan_residual_fusion(*P);
-  plan_hash_fusion(*P);
   for (auto& n : g->nodes) build_op(*P, n, P->ops[n.id]);
-  plan_gather_fusion(*P, num_sms(dev));
   CK(cudaDeviceSynchronize());
   g->prog = P;
   return P;
 }
 
-// the gather is done by its consumer GEMM (plan_gather_fusion) when both run in subgraph s
-bool gather_absorbed(const Program& P, const Partition& part, int s, int v) {
-  auto it = P.fused_gathers.find(v);
-  return it != P.fused_gathers.end() && part.node_to_sg[v] == s && part.node_to_sg[it->second] == s;
-}
-const Op* gathering_linear(const Program& P, const Partition& part, int s, int v) {
-  auto it = P.gather_fused.find(v);
-  if (it == P.gather_fused.end() || part.node_to_sg[it->second] != s || part.node_to_sg[v] != s) return nullptr;
-  return &P.gather_ops.at(v);
-}
-
 void launch_subgraph(const Program& P, const Partition& part, int s, const Ptrs& T, cudaStream_t st) {
-  std::set<int> skip;
-  for (int v : part.sg_nodes[s]) {
-    if (skip.count(v) || gather_absorbed(P, part, s, v) || P.absorbed_hashes.count(v)) continue;
-    if (auto it = P.hash_ops.find(v); it != P.hash_ops.end()) {
-      it->second.launch(T, st);
-      continue;
-    }
-    if (const Op* go = gathering_linear(P, part, s, v)) {
-      go->launch(T, st);
-      continue;
-    }
+  for (int v : part.sg_nodes[s])
     if (P.ops[v].launch) P.ops[v].launch(T, st);
-  }
 }
 
 int subgraph_kernels(const Program& P, const Partition& part, int s) {
   int nk = 0;
-  std::set<int> skip;
-  for (int v : part.sg_nodes[s]) {
-    if (skip.count(v) || gather_absorbed(P, part, s, v) || P.absorbed_hashes.count(v)) continue;
-    if (P.hash_ops.count(v)) {
-      nk += 1;
-      continue;
-    }
-    if (gathering_linear(P, part, s, v)) {
-      nk += 1;
-      continue;
-    }
-    nk += P.ops[v].n_kernels;
-  }
+  for (int v : part.sg_nodes[s]) nk += P.ops[v].n_kernels;
   return nk;
 }
 
@@ -1157,9 +1011,6 @@ static void* direct_input_ptr(const Graph& g, const Node& in, const void* host) 
   if (uses != 1) return nullptr;
   const std::string& op = consumer->op;
   if (op != "hash_mod" && op != "gather_sum" && op != "gather_concat") return nullptr;
-  // a hash absorbed by its gathers (plan_hash_fusion) has several real readers of the input:
-  // one copy over PCIe beats each of them streaming it
-  if (g.prog && g.prog->absorbed_hashes.count(consumer->id)) return nullptr;
   return mapped_host_ptr(host);
 }
 

@@ -82,88 +82,6 @@ def test_gathers_and_hash_bit_exact():
     assert rel_err(wide.cpu().numpy(), o_wide) < 1e-6
 
 
-_GATHER_FUSED_SCRIPT = r'''
-import os, sys
-sys.path.insert(0, os.environ["REPO"])
-from tests.test_gpu_parity import gather_fused_case
-for case in [(300, 5, 1000, 136, "relu"), (2048, 26, 100_000, 1024, "relu"), (513, 8, 777, 64, "none"),
-             (4096, 26, 50_000, 512, "relu")]:
-    gather_fused_case(*case)
-    print("ok", case)
-'''
-
-
-def test_gather_fused_linear_opt_in():
-    """The opt-in gather_concat -> linear fusion (DUET_GATHER_FUSE=1; the switch is read once, so a
-    subprocess)."""
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    env = dict(os.environ, DUET_GATHER_FUSE="1", REPO=root)
-    r = subprocess.run([sys.executable, "-c", _GATHER_FUSED_SCRIPT], env=env, capture_output=True, text=True,
-                       timeout=300, cwd=root)
-    assert r.returncode == 0 and r.stdout.count("ok") == 4, r.stdout + r.stderr
-
-
-_HASH_FUSED_SCRIPT = r'''
-import os, sys
-sys.path.insert(0, os.environ["REPO"])
-import torch
-from tests.test_gpu_parity import test_config_small_parity, test_host_buffers_e2e_equal_device
-for cfg, dt in [("c1", "f32"), ("c2", "bf16"), ("c5", "bf16")]:
-    test_config_small_parity(cfg, dt)
-    test_host_buffers_e2e_equal_device(cfg)
-    print("ok", cfg)
-'''
-
-
-def test_hash_absorbed_by_gathers_opt_in():
-    """The opt-in hash_mod -> gathers fusion (DUET_HASH_FUSE=1, runtime.cu plan_hash_fusion): config
-    parity against the oracle (both schedules bit-identical) and host-buffer runs, in a subprocess
-    because the switch is read once."""
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    env = dict(os.environ, DUET_HASH_FUSE="1", REPO=root)
-    r = subprocess.run([sys.executable, "-c", _HASH_FUSED_SCRIPT], env=env, capture_output=True, text=True,
-                       timeout=600, cwd=root)
-    assert r.returncode == 0 and r.stdout.count("ok") == 3, r.stdout[-3000:] + r.stderr[-3000:]
-
-
-def gather_fused_case(B, F, R, N, act):
-    """gather_concat -> linear fused into one pair GEMM (tile::gather4 A producer, runtime.cu
-    plan_gather_fusion) == the unfused node kernels bit for bit, and == the float64 oracle."""
-    ir = (f"param @E : bf16[{F},{R},64]\nparam @W : bf16[{N},{64 * F}]\nparam @b : f32[{N}]\n"
-          f"%ids = input() : i32[{B},{F}]\n%x = gather_concat(%ids, @E) : bf16[{B},{64 * F}]\n"
-          f"%y = linear(%x, @W, @b) {{act={act}}} : bf16[{B},{N}]\noutput %y\n")
-    g_ = torch.Generator().manual_seed(B + F)
-    E = torch.randn(F, R, 64, generator=g_).to(torch.bfloat16)
-    Wt = ((torch.rand(N, 64 * F, generator=g_) * 2 - 1) / (64 * F) ** 0.5).to(torch.bfloat16)
-    b = torch.rand(N, generator=g_) * 0.2 - 0.1
-    ids = torch.randint(0, R, (B, F), generator=g_, dtype=torch.int32)
-    ids[0] = R - 1
-    g = duet.Graph(ir)
-    g.bind_all({"E": E.cuda(), "W": Wt.cuda(), "b": b.cuda()})
-    s = g.partition().profile_from_table([0], [[1000]]).schedule()
-    st = torch.cuda.Stream()
-    y = torch.empty(B, N, device="cuda", dtype=torch.bfloat16)
-    s.run([(0, st)], [ids.cuda()], [y])
-    assert s.launch_count() == 1  # one fused kernel
-    x = torch.empty(B, 64 * F, device="cuda", dtype=torch.bfloat16)
-    g.node_run("x", [ids.cuda()], x)
-    y2 = torch.empty_like(y)
-    g.node_run("y", [x], y2)
-    torch.cuda.synchronize()
-    assert torch.equal(y.view(torch.int16), y2.view(torch.int16))
-    rows = np.arange(B) if B <= 600 else np.random.default_rng(0).choice(B, 64, replace=False)
-    Ef = OF.to_f64(to_np(E), "bf16")
-    X = Ef[np.arange(F)[None, :], ids.numpy()[rows]].reshape(len(rows), -1)
-    want = OF.linear(X, OF.to_f64(to_np(Wt), "bf16"), b.double().numpy(), act)
-    assert rel_err(y.float().cpu().numpy()[rows], want) <= TOL["bf16"]
-
-
 def _oracle_outputs(wl, params, inputs):
     return OF.run(wl.ir, oracle_arrays(params), oracle_arrays(inputs))
 
