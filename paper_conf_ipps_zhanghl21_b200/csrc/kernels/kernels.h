@@ -104,6 +104,17 @@ int tc2_pick_bn(int M, int N, int K, int num_sms);
 void gemm_tc2_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
                    int out_bf16, cudaStream_t st);
 
+// ---- fp32 on the tensor cores (gemm_tf32.cu): 3xTF32 tcgen05 GEMM, 128 x bn tiles (bn 64 / 128) ----
+// A map [M, K] fp32 box 128 rows, W map [N, K] box bn rows (make_tmap_f32_2d: 32-column boxes);
+// epilogues EPI_BIAS_ACT (fp32 out) / EPI_LSTM / EPI_GRU (fp32 state, ep.kx in 32-wide k-blocks).
+CUtensorMap make_tmap_f32_2d(const void* base, int64_t rows, int64_t cols, int box_rows);
+bool tf32x3_ok(int K, int N);
+int tf32x3_pick_bn(int M, int N, int K, int num_sms);
+void gemm_tf32x3_maps(const CUtensorMap& ta, const CUtensorMap& tw, int M, int N, int K, int bn, const TcEpilogue& ep,
+                      int epi, cudaStream_t st, const CUtensorMap* tx = nullptr);
+void rnn_pack_f32(int kind, const float* Wih, const float* Whh, const float* bih, const float* bhh, float* Wcat,
+                  float* bias, int E, int Ep, int H, int U, int BN, int tiles, cudaStream_t st);
+
 // ---- SIMT fallbacks / small kernels (simt.cu) ----
 // Y[M,N] = act(X[M,K] W[N,K]^T + b) ; X/W dtype per flags; fp32 accumulate.
 void gemm_simt(const void* X, int x_bf16, const void* W, int w_bf16, const float* b, void* Y, int y_bf16, int M,
@@ -175,6 +186,13 @@ void fold_bn(const void* W, int bf16, const float* g, const float* beta, const f
 // Tap rectangle of a conv: the filter taps that touch the input for at least one output pixel.
 struct ConvTaps { int r0 = 0, nr = 1, s0 = 0, ns = 1; };
 ConvTaps conv_taps(const ConvShape& s);
+// fp32 implicit-GEMM conv (3xTF32; C % 32 == 0): tw = make_tmap_f32_2d(Wf [Co, kh*kw*C], Co, K, bn),
+// bn in {64, 128}; residual fp32 [M, Co] or null.  im2col_f32: explicit im2col for the other layers
+// (the 3-channel stem), rows padded to ldk (% 4 == 0) with zeros.
+bool conv_tf32_ok(const ConvShape& s);
+void conv_tf32x3(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
+                 const ConvShape& s, int act, int bn, cudaStream_t st);
+void im2col_f32(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStream_t st);
 // Launch plan: tile width bn, effective 64-wide k-blocks nkb (tap rectangle); ks is always 1.
 struct ConvPlan { int bn = 64, ks = 1, nkb = 0; };
 ConvPlan conv_tc_plan(const ConvShape& s, int num_sms);

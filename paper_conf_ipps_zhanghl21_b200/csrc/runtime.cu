@@ -19,6 +19,13 @@
 
 namespace duet {
 
+// fp32 contractions on the tensor cores (3xTF32, gemm_tf32.cu); DUET_TF32=0 keeps the CUDA-core
+// kernels (comparisons)
+static bool tf32_on() {
+  static const bool on = !(getenv("DUET_TF32") && atoi(getenv("DUET_TF32")) == 0);
+  return on;
+}
+
 // ------------------------------------------------------------------------------------------------
 // Program
 // ------------------------------------------------------------------------------------------------
@@ -243,6 +250,23 @@ void build_op(Program& P, const Node& n, Op& op) {
         if (splits > 1) gemm_splitk_reduce(ep, M, N, yb, st);
       };
       op.n_kernels = splits > 1 ? 2 : 1;
+    } else if (!xb && !wb && !yb && tf32x3_ok(K, N) && tf32_on()) {
+      // fp32 mode on the tensor cores: 3xTF32 (kernels/gemm_tf32.cu)
+      const char* bn_env = getenv("DUET_GEMM_BN");
+      const int bn = bn_env ? atoi(bn_env) : tf32x3_pick_bn(M, N, K, sms);
+      const char* dbg_env = getenv("DUET_GEMM_DBG");  // accumulator-split experiments (gemm_tf32.cu)
+      const int dbg = dbg_env ? atoi(dbg_env) : 0;
+      CUtensorMap tw = make_tmap_f32_2d(W, N, K, bn);
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        CUtensorMap ta = make_tmap_f32_2d(T[in], M, K, 128);
+        TcEpilogue ep;
+        ep.bias = b;
+        ep.out = T[me];
+        ep.ldo = N;
+        ep.act = act;
+        ep.dbg = dbg;
+        gemm_tf32x3_maps(ta, tw, M, N, K, bn, ep, EPI_BIAS_ACT, st);
+      };
     } else {
       op.launch = [=](const Ptrs& T, cudaStream_t st) { gemm_simt(T[in], xb, W, wb, b, T[me], yb, M, N, K, act, st); };
     }
@@ -463,6 +487,42 @@ void build_op(Program& P, const Node& n, Op& op) {
         }
       };
       op.n_kernels = S;
+    } else if (x.dtype == kF32 && E % 4 == 0 && H % 4 == 0 && tf32_on()) {
+      // fp32 mode on the tensor cores: the fused step of the bf16 path as a 3xTF32 GEMM
+      // (kernels/gemm_tf32.cu), one launch per step; x and h in fp32, K = [x_t (E, padded to 32) | h]
+      const int bn = 64;
+      const int U = bn / 4;
+      const int tiles = (H + U - 1) / U;
+      const int Np = tiles * bn;
+      const int Ep = (E + 31) / 32 * 32;
+      const int Kc = Ep + H;
+      float* Wcat = (float*)P.alloc((int64_t)Np * Kc * 4);
+      float* bias = (float*)P.alloc((int64_t)Np * 4);
+      rnn_pack_f32(kind, (const float*)Wih, (const float*)Whh, bih, bhh, Wcat, bias, E, Ep, H, U, bn, tiles, 0);
+      CK(cudaDeviceSynchronize());
+      CUtensorMap t_w = make_tmap_f32_2d(Wcat, Np, Kc, bn);
+      CUtensorMap t_h[2] = {make_tmap_f32_2d(hb[0], B, H, 128), make_tmap_f32_2d(hb[1], B, H, 128)};
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        CK(cudaMemsetAsync(hb[1], 0, (size_t)B * H * 4, st));
+        if (kind == EPI_LSTM) CK(cudaMemsetAsync(cst, 0, (size_t)B * H * 4, st));
+        CUtensorMap tx = make_tmap_f32_2d(T[in], (int64_t)S * B, E, 128);
+        for (int t = 0; t < S; ++t) {
+          TcEpilogue e2;
+          e2.bias = bias;
+          e2.c_state = cst;
+          e2.h_prev = hb[(t + 1) & 1];
+          e2.h_next = (t == S - 1 && !seq) ? T[me] : hb[t & 1];
+          e2.H = H;
+          e2.kx = Ep / 32;
+          e2.x_row0 = t * B;
+          // t = 0: h_{-1} = 0, so only the x_t part of K contributes
+          gemm_tf32x3_maps(t_h[(t + 1) & 1], t_w, B, Np, t == 0 ? Ep : Kc, bn, e2, kind, st, &tx);
+          if (seq)
+            CK(cudaMemcpyAsync((char*)T[me] + (size_t)t * B * H * 4, hb[t & 1], (size_t)B * H * 4,
+                               cudaMemcpyDeviceToDevice, st));
+        }
+      };
+      op.n_kernels = S;
     } else {
       // fp32 parity path (original PyTorch layout): G_x = x W_ih^T + folded bias, then SIMT steps
       std::vector<int32_t> ident(G * H);
@@ -519,7 +579,11 @@ void build_op(Program& P, const Node& n, Op& op) {
     const bool tma = bf && s.Co % 16 == 0 && conv_tma_ok(s);
     const bool stem = bf && !tma && res < 0 && !no_stem && conv_stem_ok(s);
     const bool cols = bf && !tma && !stem && s.Co >= 16 && s.Co % 8 == 0 && res < 0;
-    const int64_t ldw = (tma || cols || stem) ? (per_co + 7) / 8 * 8 : per_co;
+    // fp32 mode on the tensor cores (3xTF32, gemm_tf32.cu): implicit GEMM with im2col TMA when
+    // C % 32 == 0, else (the stem) explicit im2col + the 3xTF32 GEMM
+    const bool f32tc = !bf && tf32_on() && conv_tf32_ok(s);
+    const bool f32cols = !bf && tf32_on() && !f32tc && s.Co >= 16 && s.Co % 4 == 0 && res < 0;
+    const int64_t ldw = (tma || cols || stem) ? (per_co + 7) / 8 * 8 : f32cols ? (per_co + 3) / 4 * 4 : per_co;
     void* Wf = P.alloc((int64_t)s.Co * ldw * dtype_bytes(w.dtype));
     float* bias = (float*)P.alloc((int64_t)s.Co * 4);
     fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
@@ -557,6 +621,30 @@ void build_op(Program& P, const Node& n, Op& op) {
         conv_tc(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, K, act, plan, ctr, st);
       };
       op.n_kernels = 1;
+    } else if (f32tc) {
+      const int bn = tf32x3_pick_bn((int)std::min<int64_t>((int64_t)s.N * s.Ho * s.Wo, INT32_MAX), s.Co,
+                                    conv_taps(s).nr * conv_taps(s).ns * s.C, sms);
+      CUtensorMap tw = make_tmap_f32_2d(Wf, s.Co, ldw, bn);
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        conv_tf32x3(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, act, bn, st);
+      };
+      op.n_kernels = 1;
+    } else if (f32cols) {
+      const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
+      void* colbuf = P.alloc(M * ldw * 4);
+      const int bn = tf32x3_pick_bn((int)M, s.Co, (int)ldw, sms);
+      CUtensorMap tw = make_tmap_f32_2d(Wf, s.Co, ldw, bn);
+      CUtensorMap ta = make_tmap_f32_2d(colbuf, M, ldw, 128);
+      op.launch = [=](const Ptrs& T, cudaStream_t st) {
+        im2col_f32(T[in], colbuf, s, ldw, st);
+        TcEpilogue ep;
+        ep.bias = bias;
+        ep.out = T[dst];
+        ep.ldo = s.Co;
+        ep.act = act;
+        gemm_tf32x3_maps(ta, tw, (int)M, s.Co, (int)ldw, bn, ep, EPI_BIAS_ACT, st);
+      };
+      op.n_kernels = 2;
     } else if (stem) {
       void* Wk = P.alloc((int64_t)s.Co * 192 * 2);
       conv_stem_pack(Wf, ldw, Wk, s, 0);

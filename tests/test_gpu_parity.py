@@ -37,8 +37,11 @@ def _rand(shape, dt, scale=1.0, seed=0):
     (2048, 1024, 1664, "bf16", "bf16"),
     (77, 48, 72, "bf16", "f32"),
     (513, 272, 200, "bf16", "f32"),
-    (300, 136, 320, "f32", "f32"),
-    (5, 3, 7, "f32", "f32"),
+    (300, 136, 320, "f32", "f32"),      # fp32 on the tensor cores (3xTF32, gemm_tf32.cu)
+    (2048, 1024, 1664, "f32", "f32"),   # c2's fc1 in fp32: 128-wide tiles
+    (130, 17, 36, "f32", "f32"),        # ragged M / N, K one 32-wide block + 4
+    (4096, 64, 1024, "f32", "f32"),
+    (5, 3, 7, "f32", "f32"),            # K % 4 != 0, N < 16: CUDA-core path
     (128, 768, 3072, "bf16", "bf16"),   # split-K (12 splits of 4 k-blocks) + reduce
     (120, 136, 2500, "bf16", "f32"),    # split-K, ragged M / N / K
     (3, 768, 768, "bf16", "bf16"),      # MT-DNN task pooler at batch 3
@@ -271,29 +274,45 @@ def test_c2_full_size_sampled():
     (3, 12, 20, 64, 48, 3, 1, 1),     # halo kernel, W != H, ragged last band, Co < tile
 ])
 
-def test_conv_node(N, H, W, C, Co, k, stride, pad):
+def test_conv_node(N, H, W, C, Co, k, stride, pad, dt="bf16"):
     Ho, Wo = (H + 2 * pad - k) // stride + 1, (W + 2 * pad - k) // stride + 1
     ir = _single_node_graph(
-        f"%y = conv2d_bn(%x, @W, @g, @b, @m, @v) {{stride={stride}, pad={pad}, act=relu}} : bf16[{N},{Ho},{Wo},{Co}]",
-        {"W": ("bf16", (Co, k, k, C)), "g": ("f32", (Co,)), "b": ("f32", (Co,)), "m": ("f32", (Co,)),
-         "v": ("f32", (Co,))}, {"x": ("bf16", (N, H, W, C))})
-    x = _rand((N, H, W, C), "bf16", 1.0, 5)
-    Wt = _rand((Co, k, k, C), "bf16", (2.0 / (k * k * C)) ** 0.5, 6)
+        f"%y = conv2d_bn(%x, @W, @g, @b, @m, @v) {{stride={stride}, pad={pad}, act=relu}} : {dt}[{N},{Ho},{Wo},{Co}]",
+        {"W": (dt, (Co, k, k, C)), "g": ("f32", (Co,)), "b": ("f32", (Co,)), "m": ("f32", (Co,)),
+         "v": ("f32", (Co,))}, {"x": (dt, (N, H, W, C))})
+    x = _rand((N, H, W, C), dt, 1.0, 5)
+    Wt = _rand((Co, k, k, C), dt, (2.0 / (k * k * C)) ** 0.5, 6)
     g_ = (_rand((Co,), "f32", 0.5, 7) + 1.0)
     b_ = _rand((Co,), "f32", 0.1, 8)
     m_ = _rand((Co,), "f32", 0.1, 9)
     v_ = (_rand((Co,), "f32", 0.5, 10) + 1.0)
     g = duet.Graph(ir)
     g.bind_all({"W": Wt.cuda(), "g": g_.cuda(), "b": b_.cuda(), "m": m_.cuda(), "v": v_.cuda()})
-    y = torch.empty((N, Ho, Wo, Co), dtype=torch.bfloat16, device="cuda")
+    y = torch.empty((N, Ho, Wo, Co), dtype=torch.bfloat16 if dt == "bf16" else torch.float32, device="cuda")
     g.node_run("y", [x.cuda()], y)
     torch.cuda.synchronize()
     f = lambda t, d: OF.to_f64(to_np(t), d)
-    want = OF.conv2d_bn(f(x, "bf16"), f(Wt, "bf16"), f(g_, "f32"), f(b_, "f32"), f(m_, "f32"), f(v_, "f32"),
+    want = OF.conv2d_bn(f(x, dt), f(Wt, dt), f(g_, "f32"), f(b_, "f32"), f(m_, "f32"), f(v_, "f32"),
                         stride, pad, "relu")
-    err = rel_err(y.float().cpu().numpy(), want)
-    print(f"[parity] conv {N}x{H}x{W}x{C}->{Co} k{k}s{stride}: rel err {err:.3e}")
-    assert err <= TOL["bf16"], err
+    check(y.float().cpu().numpy(), want, TOL[dt], f"conv {N}x{H}x{W}x{C}->{Co} k{k}s{stride} {dt}")
+
+
+@pytest.mark.parametrize("N,H,W,C,Co,k,stride,pad", [
+    (2, 23, 19, 3, 64, 7, 2, 3),      # C % 32 != 0: explicit fp32 im2col + 3xTF32 GEMM
+    (1, 224, 224, 3, 64, 7, 2, 3),    # ResNet stem at full size
+    (2, 30, 16, 4, 48, 5, 2, 2),
+    (3, 14, 14, 64, 64, 3, 1, 1),     # 3xTF32 implicit GEMM (im2col TMA, 32-channel k-blocks)
+    (2, 15, 13, 128, 256, 3, 2, 1),   # stride 2, 128-wide tiles
+    (2, 9, 9, 64, 128, 1, 2, 0),      # 1x1 downsample
+    (4, 1, 1, 512, 512, 3, 1, 1),     # tap rectangle: centre tap only
+    (16, 2, 2, 256, 512, 3, 2, 1),
+    (30, 7, 7, 512, 256, 3, 1, 1),    # ragged last m tile, K = 4608
+    (2, 56, 56, 64, 64, 3, 1, 1),     # c4 layer-1 shape
+    (3, 12, 20, 32, 48, 3, 1, 1),     # one 32-channel block, Co < tile
+])
+def test_conv_node_f32(N, H, W, C, Co, k, stride, pad):
+    """fp32 mode on the tensor cores (gemm_tf32.cu) against the float64 oracle at the fp32 bar."""
+    test_conv_node(N, H, W, C, Co, k, stride, pad, dt="f32")
 
 _HALO_SCRIPT = r'''
 import os, sys
@@ -325,8 +344,12 @@ def test_conv_halo_all_shapes_forced():
     ("lstm", 5, 64, 40, 136, "bf16"),    # E padded to 64, H > one tile
     ("gru", 6, 200, 64, 72, "bf16"),
     ("gru", 4, 130, 24, 256, "bf16"),
-    ("lstm", 5, 33, 24, 40, "f32"),      # CUDA-core parity path
+    ("lstm", 5, 33, 24, 40, "f32"),      # fp32: 3xTF32 fused step (gemm_tf32.cu)
     ("gru", 5, 33, 24, 40, "f32"),
+    ("lstm", 6, 300, 64, 136, "f32"),    # 3 M tiles, H over several 16-unit tiles
+    ("gru", 5, 260, 100, 72, "f32"),     # E padded to 128
+    ("lstm", 4, 20, 23, 40, "f32"),      # E % 4 != 0: CUDA-core parity path
+    ("gru", 4, 20, 24, 42, "f32"),       # H % 4 != 0: CUDA-core parity path
 ])
 def test_rnn_node(kind, S, B, E, H, dt):
     G = 4 if kind == "lstm" else 3
@@ -358,7 +381,8 @@ def test_rnn_node(kind, S, B, E, H, dt):
     ("gru", 3, 4000, 136, 520, "bf16"),   # 128 x 256 tiles, ragged B, H and E
     ("lstm", 4, 2304, 128, 264, "bf16"),  # one 128 x 256 tile per CTA (90 tiles), ragged H
     ("gru", 3, 4096, 128, 256, "bf16"),   # one 128 x 256 tile per CTA (c5's b3 shape, GRU)
-    ("gru", 4, 33, 24, 40, "f32"),        # CUDA-core parity path
+    ("gru", 4, 33, 24, 40, "f32"),        # 3xTF32 fused step
+    ("lstm", 3, 40, 23, 40, "f32"),       # CUDA-core parity path
 ])
 def test_rnn_node_seq_output(kind, S, B, E, H, dt):
     rnn_seq_case(kind, S, B, E, H, dt)
