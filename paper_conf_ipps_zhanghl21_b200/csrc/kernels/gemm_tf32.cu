@@ -14,8 +14,9 @@
 // K = 16).  Warp roles (6 warps):
 //   warp 0      TMA producer: A/W k-blocks into a STAGES ring (full[s])
 //   warp 1      TMEM allocator + UMMA issuer: three kind::tf32 UMMAs per 8-deep k-step
-//   warps 2..5  split the landed stage in shared memory (a_big in place, a_small into the stage's
-//               second half; elementwise, so the swizzle is irrelevant), fence the generic-proxy
+//   warps 2..5  split the landed stage in shared memory (a_small into the stage's second half;
+//               a_big is the MMA's own truncating tf32 read of the fp32 operand; elementwise, so the
+//               swizzle is irrelevant), fence the generic-proxy
 //               stores for the tensor core (split[s]); after the mainloop: the fused epilogue
 // Epilogues (fp32 in and out): EPI_BIAS_ACT (+ optional residual), EPI_LSTM, EPI_GRU -- gemm_tc.cu's,
 // with the state (c, h_prev, h_next) in fp32 and full-precision expf / tanhf.
@@ -199,13 +200,16 @@ __global__ void __launch_bounds__(192, 1)
       ptx::mbar_wait(&full[s], (kb / Cfg::STAGES) & 1);
       uint4* big = reinterpret_cast<uint4*>(sA(s));
       uint4* small = big + kChunks;
+      // only the small parts are stored: kind::tf32 reads the top 19 bits of each fp32 operand
+      // (truncation), which IS a_big -- measured: the same error with and without clearing the
+      // low bits in place (tools/tf32_time.py), and 10% faster without the store
+      if (!(ep.dbg & 32))  // experiments: 32 = no split (mainloop timing; wrong results)
 #pragma unroll 4
-      for (int i = et; i < kChunks; i += kFSplitThreads) {
-        uint4 v = big[i], r;
-        split4(v, r);
-        big[i] = v;
-        small[i] = r;
-      }
+        for (int i = et; i < kChunks; i += kFSplitThreads) {
+          uint4 v = big[i], r;
+          split4(v, r);
+          small[i] = r;
+        }
       ptx::fence_async_smem();  // generic-proxy stores -> visible to the tensor core
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&split[s]);
@@ -417,25 +421,41 @@ PFN_cuTensorMapEncodeIm2col_v12000 encode_im2col() {
   return fn;
 }
 
-// cols[m, k] = x[n, ho*s-p+r, wo*s-p+q, c], k = (r, q, c), rows padded to ldk with zeros, fp32
+// cols[m, k] = x[n, ho*s-p+r, wo*s-p+q, c], k = (r, q, c), rows padded to ldk with zeros, fp32.
+// One thread per output row: (n, ho, wo) decoded once, k walked with incremental counters, the row
+// written as 16-B stores (as im2col_kernel, conv.cu).
 __global__ void im2col_f32_kernel(const float* __restrict__ x, float* __restrict__ cols, ConvShape s, int ldk) {
   ptx::pdl_wait();
   ptx::pdl_trigger();
   const int K = s.kh * s.kw * s.C;
-  const int64_t total = (int64_t)s.N * s.Ho * s.Wo * ldk;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t m = i / ldk;
-    const int k = (int)(i - m * ldk);
-    float v = 0.0f;
-    if (k < K) {
-      const int wo = (int)(m % s.Wo);
-      const int64_t q0 = m / s.Wo;
-      const int ho = (int)(q0 % s.Ho), n = (int)(q0 / s.Ho);
-      const int c = k % s.C, rq = k / s.C, q = rq % s.kw, r = rq / s.kw;
-      const int hi = ho * s.stride - s.pad + r, wi = wo * s.stride - s.pad + q;
-      if ((unsigned)hi < (unsigned)s.H && (unsigned)wi < (unsigned)s.W) v = x[(((int64_t)n * s.H + hi) * s.W + wi) * s.C + c];
+  const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
+  for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < M; m += (int64_t)gridDim.x * blockDim.x) {
+    const int wo = (int)(m % s.Wo);
+    const int64_t q0 = m / s.Wo;
+    const int ho = (int)(q0 % s.Ho), n = (int)(q0 / s.Ho);
+    const int hb = ho * s.stride - s.pad, wb = wo * s.stride - s.pad;
+    float4* dst = reinterpret_cast<float4*>(cols + m * ldk);
+    int c = 0, q = 0, r = 0;
+    for (int k0 = 0; k0 < ldk; k0 += 4) {
+      float v[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        v[e] = 0.0f;
+        if (k0 + e < K) {
+          const int hi = hb + r, wi = wb + q;
+          if ((unsigned)hi < (unsigned)s.H && (unsigned)wi < (unsigned)s.W)
+            v[e] = __ldg(x + (((int64_t)n * s.H + hi) * s.W + wi) * s.C + c);
+          if (++c == s.C) {
+            c = 0;
+            if (++q == s.kw) {
+              q = 0;
+              ++r;
+            }
+          }
+        }
+      }
+      dst[k0 / 4] = make_float4(v[0], v[1], v[2], v[3]);
     }
-    cols[i] = v;
   }
 }
 }  // namespace
@@ -488,7 +508,7 @@ void im2col_f32(const void* x, void* cols, const ConvShape& s, int64_t ldk, cuda
   const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
   if (!M) return;
   if (ldk % 4 || ldk >= INT32_MAX) fail(DUET_EUNSUPPORTED, "im2col_f32: ldk % 4 == 0 required");
-  launch_pdl(im2col_f32_kernel, dim3(grid_for(M * ldk, 256)), dim3(256), 0, st, (const float*)x, (float*)cols, s,
+  launch_pdl(im2col_f32_kernel, dim3(grid_for(M, 128, 16)), dim3(128), 0, st, (const float*)x, (float*)cols, s,
              (int)ldk);
   CK(cudaGetLastError());
 }

@@ -1,6 +1,6 @@
 """Per-node kernel times of a config (real intermediates; CUDA-graph replays of node_run).
 
-  python tools/node_times.py c2 [--flush]
+  python tools/node_times.py c2 [--flush] [--dt f32]
 
 Every node is made a graph output so one serial duet_run materialises all intermediates; then
 each node is timed alone: a CUDA graph of `iters` back-to-back duet_node_run launches, replayed
@@ -21,6 +21,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("config")
     ap.add_argument("--small", action="store_true")
+    ap.add_argument("--dt", default=None, choices=[None, "bf16", "f32"])
     ap.add_argument("--iters", type=int, default=20)
     ap.add_argument("--replays", type=int, default=20)
     ap.add_argument("--flush", action="store_true", help="flush L2 before every replay (1 launch per replay)")
@@ -31,7 +32,7 @@ def main():
     from paper_conf_ipps_zhanghl21_b200 import workloads as W
     from paper_conf_ipps_zhanghl21_b200.harness import materialize
 
-    wl = W.build(args.config, small=args.small)
+    wl = W.build(args.config, small=args.small, dt=args.dt)
     decl = {}
     for line in wl.ir.splitlines():
         m = re.match(r"%(\w+) = (\w+)\((.*?)\).*: (\w+)\[([\d,]*)\]", line)
