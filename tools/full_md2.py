@@ -2,6 +2,7 @@
 (read by bench.py for roofline.traffic: DRAM bytes per launch of each config's dominant kernel).
 
     python tools/full_md2.py r2 c5:b4_gru=gpurun_out/r2_full_gru1024_raw.csv ...
+    python tools/full_md2.py r2_tf32 --no-summary fc1_f32=gpurun_out/...raw.csv   (md only)
 """
 import csv
 import json
@@ -34,8 +35,9 @@ def read(path):
 
 
 def main():
-    tag = sys.argv[1]
-    items = [a.split("=", 1) for a in sys.argv[2:]]
+    args = [a for a in sys.argv[1:] if a != "--no-summary"]
+    tag = args[0]
+    items = [a.split("=", 1) for a in args[1:]]
     lines = [f"# {tag}: `ncu --set full --clock-control none` captures (one launch each, cold-cache replay)", ""]
     summary = {"tag": tag, "kernels": {}}
     for name, path in items:
@@ -50,7 +52,8 @@ def main():
                                     "tensor_pipe_pct": d.get("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed"),
                                     "kernel": d["kernel"][:120]}
     open(os.path.join(ROOT, "profiles", f"{tag}_full.md"), "w").write("\n".join(lines) + "\n")
-    json.dump(summary, open(os.path.join(ROOT, "profiles", "ncu_summary.json"), "w"), indent=1)
+    if "--no-summary" not in sys.argv:  # (extra captures: keep bench.py's per-config summary)
+        json.dump(summary, open(os.path.join(ROOT, "profiles", "ncu_summary.json"), "w"), indent=1)
     print("\n".join(lines))
 
 
