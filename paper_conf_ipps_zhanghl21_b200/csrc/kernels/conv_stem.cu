@@ -38,7 +38,8 @@ constexpr int A_ATOM_BYTES = ROWS * 128;
 constexpr int A_BYTES = ATOMS * A_ATOM_BYTES;  // 48 KB
 constexpr int NB = 8;               // builder warps (two threads per output pixel, kh rows split)
 constexpr int NE = 4;               // epilogue warps
-constexpr int THREADS = 32 * (NB + 1 + NE);
+constexpr int PW = NB + 1 + NE;     // patch producer warp (tile fetch + patch TMA), last
+constexpr int THREADS = 32 * (PW + 1);
 constexpr int NPMAX = 8;            // max patch buffers
 constexpr int BOXW = 256;           // patch box width (elements)
 constexpr int STEP = BOXW - SEG;    // element distance between consecutive boxes
@@ -93,8 +94,9 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint64_t* t_full = a_full + 4;        // [2] MMA commit -> epilogue
   uint64_t* t_empty = a_full + 6;       // [2] epilogue -> MMA
   uint64_t* w_full = a_full + 8;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(w_full + 1);
-  float* s_bias = reinterpret_cast<float*>(w_full + 2);
+  uint64_t* patch_empty = a_full + 9;   // [np] builders -> patch producer
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(patch_empty + NPMAX);
+  float* s_bias = reinterpret_cast<float*>(patch_empty + NPMAX + 1);
   // tile of local work item i: s_tile[i % 16] (-1 = no more work), written by the patch issuer,
   // published through ring_full[i % 16]; the MMA warp and the epilogue each read it and arrive on
   // ring_empty[i % 16] before the slot is reused
@@ -109,7 +111,10 @@ __global__ void __launch_bounds__(THREADS, 1)
   if (threadIdx.x == 0) {
     ptx::tma_prefetch(&tmX);
     ptx::tma_prefetch(&tmW);
-    for (int i = 0; i < g.np; ++i) ptx::mbar_init(&patch_full[i], 1);
+    for (int i = 0; i < g.np; ++i) {
+      ptx::mbar_init(&patch_full[i], 1);
+      ptx::mbar_init(&patch_empty[i], 1);
+    }
     for (int i = 0; i < 2; ++i) {
       ptx::mbar_init(&a_full[i], 1);
       ptx::mbar_init(&a_empty[i], 1);
@@ -170,19 +175,23 @@ __global__ void __launch_bounds__(THREADS, 1)
       ptx::tma_load_3d(&tmX, &patch_full[pb], dst + b * bbytes, b * STEP - g.L, ho * g.stride - g.pad, n);
   };
 
-  if (warp < NB) {
+  if (warp == PW) {
+    // ---------------- patch producer: tile fetch + patch TMA, np items ahead of the builders ----------------
+    // (its own warp since round 2: issued by builder thread 0, the tile counter's atomic round trip
+    // sat on the builders' critical path -- c4 stem 114 -> 88 us, c5 133 -> 104 us, CUDA-graph timing)
+    if (lane == 0) {
+      for (int i = 0;; ++i) {
+        if (i >= g.np) ptx::mbar_wait(&patch_empty[i % g.np], (uint32_t)(((i / g.np) - 1) & 1));
+        issue_patch(i);
+        if (s_tile[i & 15] < 0) break;
+      }
+    }
+  } else if (warp < NB) {
     // ---------------- builders: patch -> A (im2col in shared memory) ----------------
     const int m = threadIdx.x & (ROWS - 1);  // output pixel (UMMA row) of this thread
     const int rr = m / g.Wo, wo = m % g.Wo;   // output row within the tile, column
     const int kh_half = (g.kh + 1) / 2;
     const int r0 = threadIdx.x < ROWS ? 0 : kh_half, r1 = threadIdx.x < ROWS ? kh_half : g.kh;
-    if (threadIdx.x == 0) {
-      int i = 0;
-      for (; i < g.np; ++i) {
-        issue_patch(i);
-        if (s_tile[i & 15] < 0) break;
-      }
-    }
     // this pixel's window: box b, element offset o (even: 4-byte aligned words), box row rr*stride
     const int off = g.stride * g.C * wo + g.L - g.pad * g.C - g.d;
     const int src0 = (off / STEP) * bbytes + (off % STEP) * 2 + rr * g.stride * g.rowb;
@@ -210,10 +219,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       asm volatile("bar.sync 2, %0;" ::"n"(32 * NB) : "memory");  // A[p] built, patch[p] consumed
       if (threadIdx.x == 0) {
         ptx::mbar_arrive(&a_full[p]);
-        // the next item, unless the end was already issued among the items in flight
-        bool ended = false;
-        for (int k = i + 1; k < i + g.np; ++k) ended |= s_tile[k & 15] < 0;
-        if (!ended) issue_patch(i + g.np);
+        ptx::mbar_arrive(&patch_empty[pb]);
       }
     }
   } else if (warp == NB) {
@@ -307,16 +313,16 @@ StemGeom geom(const ConvShape& s, int act) {
   // off / STEP == b
   g.nbx = (s.stride * s.C * (s.Wo - 1) + g.L - s.pad * s.C - g.d) / STEP + 1;
   g.ksteps = (s.kh * SEG + 15) / 16;
-  const size_t fixed = 1024 + 2 * A_BYTES + (size_t)ATOMS * s.Co * 128 + (NPMAX + 9) * 8 + (size_t)s.Co * 4;
+  const size_t fixed = 1024 + 2 * A_BYTES + (size_t)ATOMS * s.Co * 128 + (2 * NPMAX + 10) * 8 + (size_t)s.Co * 4;
   const size_t pb = (size_t)g.nbx * g.bh * g.rowb;
-  g.np = (int)std::min<size_t>(NPMAX, (227 * 1024 - fixed) / pb);
+  g.np = (int)std::min<size_t>(NPMAX, (227 * 1024 - 512 - fixed) / pb);  // 512: the static tile ring
   if (g.np < 2) g.np = 2;  // (conv_stem_ok rejects shapes that do not fit two)
   return g;
 }
 
 size_t stem_smem(const StemGeom& g) {
-  return 1024 + 2 * A_BYTES + (size_t)ATOMS * g.Co * 128 + (size_t)g.np * g.nbx * g.bh * g.rowb + (NPMAX + 9) * 8 +
-         (size_t)g.Co * 4;
+  return 1024 + 2 * A_BYTES + (size_t)ATOMS * g.Co * 128 + (size_t)g.np * g.nbx * g.bh * g.rowb +
+         (2 * NPMAX + 10) * 8 + (size_t)g.Co * 4;
 }
 
 }  // namespace

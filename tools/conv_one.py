@@ -1,6 +1,8 @@
 """One conv2d_bn node at a given shape, for ncu / timing (bf16, NHWC, BN folded, ReLU).
 
     python tools/conv_one.py N H C Co k stride pad [reps] [residual]
+With CONV_ONE_GRAPH=1: a CUDA graph of 10 back-to-back launches per replay (no host latency in
+the figure; only the first launch of a replay starts cold).
 """
 import os
 import statistics
@@ -31,6 +33,25 @@ def main():
     flush = torch.empty(128 << 20, dtype=torch.float32, device="cuda")
     st = torch.cuda.Stream()
     ts = []
+    if os.environ.get("CONV_ONE_GRAPH") == "1":
+        with torch.cuda.stream(st):
+            g.node_run("y", [x], y, st)
+            st.synchronize()
+            gr = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gr, stream=st):
+                for _ in range(10):
+                    g.node_run("y", [x], y, torch.cuda.current_stream())
+        for i in range(reps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            with torch.cuda.stream(st):
+                e0.record(st)
+                gr.replay()
+                e1.record(st)
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1) * 1e3 / 10)
+        reps = -2
     for i in range(reps + 2):
         flush.zero_()
         torch.cuda.synchronize()
