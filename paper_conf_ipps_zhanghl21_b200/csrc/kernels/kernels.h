@@ -79,7 +79,8 @@ struct RnnPersistArgs {
                                                 // pre-swizzled [kh][Bp][64] (rnn_persist.cu)
   __nv_bfloat16* out = nullptr;       // [B, H] h_S
   __nv_bfloat16* seq = nullptr;       // optional [S, B, H]: every h_t (a lower stacked-RNN layer)
-  unsigned* counter = nullptr;        // grid-barrier counter, zeroed before each launch
+  unsigned* counter = nullptr;        // step counters, zeroed before each launch: [tiles_m] (msync)
+                                      // or [1] (grid barrier)
   float* c_state = nullptr;           // LSTM cell state [B, H] fp32 (several tiles per CTA only)
   int S = 0, B = 0, H = 0, kx = 0, kh = 0;
   int Bp = 0;                         // B padded to the 128-row tiles
@@ -87,6 +88,8 @@ struct RnnPersistArgs {
   int dbg = 0;                        // 1 = per-step timestamps (g_rp_trace)
   int stages = 0;                     // A-ring depth (set by the launcher)
   int pair = 0;                       // 1: CTA-pair kernel (rnn_pair_kernel; 256 x 256 pair tiles)
+  int msync = 1;                      // 1: step t+1 of a 128-row block waits only for that block's
+                                      // h_t (batch rows are independent recurrences); 0: grid barrier
   const void* wcat = nullptr;         // pair: packed weights [w_rows, w_cols] (for its 128-row box)
   int64_t w_rows = 0, w_cols = 0;
 };

@@ -237,16 +237,18 @@ __global__ void __launch_bounds__(kRThreads, 1)
         for (int j = 0; j < nkb; ++j, ++g) {
           const int s = g % STAGES;
           if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
-          if (j == kx && i == 0) {
-            // h_{t-1}: wait until every epilogue warp of every tile has released its slice (grid
-            // barrier), then order the generic-proxy writes it observed before this thread's
-            // async-proxy (TMA) reads
+          if (j == kx && (a.msync || i == 0)) {
+            // h_{t-1} of this tile's 128 batch rows: wait until every epilogue warp of every tile of
+            // the row block (m-tile sync; a.msync = 0: of the whole grid) has released its slice,
+            // then order the generic-proxy writes it observed before this thread's async-proxy
+            // (TMA) reads
             if (lane == 0) {
               // releases per tile and step: one per epilogue warp (one tile per CTA), one per tile
               // (several tiles per CTA: thousands of same-address releases per step serialised at
               // the L2 -- measured ~6-10 ns each, the whole step time at B = 4096)
-              const unsigned target = (unsigned)t * (unsigned)n_tiles * (MULTI ? 1u : (unsigned)kREpiWarps);
-              while (ld_acquire_gpu(a.counter) < target) {
+              const unsigned per = (unsigned)(a.msync ? a.tiles_n : n_tiles) * (MULTI ? 1u : (unsigned)kREpiWarps);
+              const unsigned* ctr = a.counter + (a.msync ? m0 / RBM : 0);
+              while (ld_acquire_gpu(ctr) < (unsigned)t * per) {
               }
               fence_proxy_async_global();
               if (trace && t < 64) trace[t * 16 + 0] = rp_gtimer();
@@ -409,7 +411,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
           // issues fence.proxy.async before its TMA reads
           fence_proxy_async_global();
           __syncwarp();
-          if (lane == 0) red_release_gpu_add(a.counter, 1u);
+          if (lane == 0) red_release_gpu_add(a.counter + (a.msync ? tile_m0(0) / RBM : 0), 1u);
           if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 3] = rp_gtimer();
         }
       }
@@ -525,7 +527,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
             if (threadIdx.x == 64) {
               // bar.sync orders the CTA's h stores before this thread's release, which is
               // cumulative at gpu scope (no separate __threadfence)
-              red_release_gpu_add(a.counter, 1u);
+              red_release_gpu_add(a.counter + (a.msync ? tile_m0(i) / RBM : 0), 1u);
               if (mtr && u < 64) mtr[u * 16 + 3] = rp_gtimer();
             }
           }
@@ -679,10 +681,11 @@ __global__ void __launch_bounds__(kRThreads, 1)
         for (int j = 0; j < nkb; ++j, ++g) {
           const int s = g % STAGES;
           if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
-          if (j == kx && i == 0) {
+          if (j == kx && (a.msync || i == 0)) {  // this CTA's 128 rows (m-tile sync) or the grid
             if (lane == 0) {
-              const unsigned target = (unsigned)t * (unsigned)n_tiles;
-              while (ld_acquire_gpu(a.counter) < target) {
+              const unsigned per = (unsigned)(a.msync ? a.tiles_n : n_tiles);
+              const unsigned* ctr = a.counter + (a.msync ? m0 / RBM : 0);
+              while (ld_acquire_gpu(ctr) < (unsigned)t * per) {
               }
               fence_proxy_async_global();
               if (mtr && t * my_tiles < 64) mtr[(t * my_tiles) * 16 + 0] = rp_gtimer();
@@ -849,7 +852,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
           fence_proxy_async_global();
           asm volatile("bar.sync 1, %0;" ::"n"(32 * kREpiWarps) : "memory");
           if (threadIdx.x == 64) {
-            red_release_gpu_add(a.counter, 1u);
+            red_release_gpu_add(a.counter + (a.msync ? tile_m0(i) / RBM : 0), 1u);
             if (mtr && u < 64) mtr[u * 16 + 3] = rp_gtimer();
           }
         }

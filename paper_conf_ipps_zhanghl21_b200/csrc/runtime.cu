@@ -409,7 +409,10 @@ void build_op(Program& P, const Node& n, Op& op) {
       const int grid = pair ? rnn_pair_grid(tiles, mt, sms) : std::min(rp_grid, tiles * mt);
       void* Wcat = P.alloc((int64_t)Np * Kc * 2);
       float* bias = (float*)P.alloc((int64_t)Np * 4);
-      unsigned* counter = (unsigned*)P.alloc(256);
+      // one step counter per 128-row block (the recurrence of batch rows [128 m, +128) depends on
+      // those rows' h only, so a row block's step t+1 waits for its own h_t, not the whole grid)
+      const int64_t ctr_bytes = ((int64_t)mt * 4 + 255) / 256 * 256;
+      unsigned* counter = (unsigned*)P.alloc(ctr_bytes);
       rnn_pack(kind, Wih, Whh, bih, bhh, Wcat, bias, E, Ep, H, U, bn, tiles, 0);
       CK(cudaDeviceSynchronize());
       CUtensorMap t_w = make_tmap_bf16_2d(Wcat, Np, Kc, bn);
@@ -435,11 +438,18 @@ void build_op(Program& P, const Node& n, Op& op) {
       ra.tiles_m = mt;
       ra.dbg = getenv("DUET_RNN_DBG") ? atoi(getenv("DUET_RNN_DBG")) : 0;
       ra.pair = pair ? 1 : 0;
+      // row-block step sync (measured, tools/msync_ab.sh): several
+      // tiles per CTA (c5's GRU512 14.3 -> 11.2, LSTM512 15.8 -> 11.8 us per step) and many row blocks
+      // (LSTM256 at B = 4096, 32 blocks of 4 CTAs: 6.7 -> 6.3); with 2 row blocks (c3's towers) the
+      // grid barrier measured faster (5.65 vs 5.87 us).  DUET_RNN_MSYNC: 0 never, 2 always.
+      static const int msync_env = getenv("DUET_RNN_MSYNC") ? atoi(getenv("DUET_RNN_MSYNC")) : 1;
+      const bool several = (int64_t)tiles * mt > grid;
+      ra.msync = msync_env == 2 || (msync_env == 1 && (several || mt >= 4)) ? 1 : 0;
       ra.wcat = Wcat;
       ra.w_rows = Np;
       ra.w_cols = Kc;
       op.launch = [=](const Ptrs& T, cudaStream_t st) {
-        CK(cudaMemsetAsync(counter, 0, sizeof(unsigned), st));
+        CK(cudaMemsetAsync(counter, 0, (size_t)mt * sizeof(unsigned), st));
         CUtensorMap tx = make_tmap_bf16_2d(T[in], (int64_t)S * B, E, 128);
         RnnPersistArgs r = ra;
         if (seq) {

@@ -411,6 +411,32 @@ def test_rnn_pair_lstm_forced():
     assert r.returncode == 0 and r.stdout.count("ok") == 3, r.stdout[-3000:] + r.stderr[-3000:]
 
 
+_MSYNC_SCRIPT = r'''
+import os, sys
+sys.path.insert(0, os.environ["REPO"])
+from tests.test_gpu_parity import rnn_seq_case
+for case in [("lstm", 6, 300, 64, 136, "bf16"), ("gru", 5, 1000, 64, 72, "bf16"), ("lstm", 4, 2304, 128, 264, "bf16"),
+             ("lstm", 4, 4096, 256, 512, "bf16"), ("gru", 4, 4000, 136, 520, "bf16")]:
+    rnn_seq_case(*case)
+    print("ok", case)
+'''
+
+
+@pytest.mark.parametrize("msync", ["0", "2"])
+def test_rnn_row_block_sync_forced(msync):
+    """The recurrence's step synchronisation both ways (DUET_RNN_MSYNC=2: every 128-row block waits
+    only for its own h_{t-1}; 0: one grid barrier), on one-tile (2 and 8 row blocks), several-tile
+    and CTA-pair launches; every h_t against the oracle.  A subprocess: the switch is read once."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, DUET_RNN_MSYNC=msync, REPO=root)
+    r = subprocess.run([sys.executable, "-c", _MSYNC_SCRIPT], env=env, capture_output=True, text=True, timeout=300,
+                       cwd=root)
+    assert r.returncode == 0 and r.stdout.count("ok") == 5, r.stdout[-3000:] + r.stderr[-3000:]
+
+
 def rnn_seq_case(kind, S, B, E, H, dt):
     """Stacked-RNN lower layer (seq=1, PAPER.md:89 Fig. 14): every h_t, [S, B, H] time-major."""
     G = 4 if kind == "lstm" else 3
