@@ -116,7 +116,7 @@ __global__ void gather_rows16_kernel(const IdSrc idx, const uint8_t* __restrict_
 // Same with a power-of-two number of 16-byte vectors per row and 32-bit index math (the generic
 // kernel's 64-bit divisions per vector dominated its issue time): VPR lanes per row, four rows in
 // flight per thread.
-template <int MODE, int VPR>
+template <int MODE, int VPR, int UNR = 4>
 __global__ void __launch_bounds__(256) gather_rows16p2_kernel(const IdSrc idx,
                                                               const uint8_t* __restrict__ tab,
                                                               uint8_t* __restrict__ out, int rows, int F,
@@ -126,10 +126,10 @@ __global__ void __launch_bounds__(256) gather_rows16p2_kernel(const IdSrc idx,
   constexpr int RB = VPR * 16;
   const int k = threadIdx.x & (VPR - 1);
   const int rows_per_pass = (int)(gridDim.x * blockDim.x) / VPR;
-  for (int r0 = (int)(blockIdx.x * blockDim.x + threadIdx.x) / VPR; r0 < rows; r0 += 4 * rows_per_pass) {
-    uint4 val[4];
+  for (int r0 = (int)(blockIdx.x * blockDim.x + threadIdx.x) / VPR; r0 < rows; r0 += UNR * rows_per_pass) {
+    uint4 val[UNR];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < UNR; ++u) {
       const int r = r0 + u * rows_per_pass;
       if (r < rows) {
         int64_t trow;
@@ -143,7 +143,7 @@ __global__ void __launch_bounds__(256) gather_rows16p2_kernel(const IdSrc idx,
       }
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < UNR; ++u) {
       const int r = r0 + u * rows_per_pass;
       if (r < rows) *reinterpret_cast<uint4*>(out + (int64_t)r * RB + k * 16) = val[u];
     }
@@ -241,13 +241,17 @@ static void gather_rows(int mode, const IdSrc idx, const void* tab, int esize, v
   int64_t rb = (int64_t)D * esize;
   bool vec = (rb % 16 == 0) && ((uintptr_t)tab % 16 == 0) && ((uintptr_t)out % 16 == 0);
   const int vpr16 = (int)(rb / 16);
-  if (vec && rows < (1LL << 30) && (vpr16 == 4 || vpr16 == 8 || vpr16 == 16)) {
+  if (vec && rows < (1LL << 30) && (vpr16 == 4 || vpr16 == 8 || vpr16 == 16 || vpr16 == 32)) {
+    // (8 rows in flight per thread measured slower than 4 at every c3-c5 embedding shape)
     const int g = grid_for((rows * vpr16 + 3) / 4, 256, 16);
 #define DUET_G16(M, V)                                                                                             \
   if (mode == M && vpr16 == V)                                                                                     \
     launch_pdl(gather_rows16p2_kernel<M, V>, dim3(g), dim3(256), 0, st, idx, (const uint8_t*)tab, (uint8_t*)out,  \
                (int)rows, F, R, B, S);
-    DUET_G16(0, 4) DUET_G16(0, 8) DUET_G16(0, 16) DUET_G16(1, 4) DUET_G16(1, 8) DUET_G16(1, 16)
+    // 512-byte rows (E = 256 bf16: c3-c5's token embeddings) took the generic kernel's 64-bit
+    // divisions until round 2: c5's b2_x 32.8 -> 16.1 us
+    DUET_G16(0, 4) DUET_G16(0, 8) DUET_G16(0, 16) DUET_G16(0, 32) DUET_G16(1, 4) DUET_G16(1, 8) DUET_G16(1, 16)
+    DUET_G16(1, 32)
 #undef DUET_G16
   } else if (vec) {
     int vpr = (int)(rb / 16);

@@ -161,6 +161,32 @@ __global__ void avgpool_kernel(const T* x, T* y, int N, int HW, int C) {
   }
 }
 
+// global average pool for small maps (HW < 8, e.g. c5's 1x1 layer-4 output), NHWC bf16, C % 8 == 0:
+// one thread per (image, 8-channel chunk), 16-byte loads, the HW positions summed in order in fp32
+// (the same order as avgpool_kernel; the scalar kernel took 16 us for c5's 4 MB)
+__global__ void avgpool_small8_kernel(const uint4* __restrict__ x, uint4* __restrict__ y, int N, int HW, int C8) {
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
+  const int total = N * C8;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += gridDim.x * blockDim.x) {
+    const int n = i / C8, c8 = i - n * C8;
+    float acc[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) acc[e] = 0.0f;
+    for (int j = 0; j < HW; ++j) {
+      const uint4 v = __ldg(x + ((size_t)n * HW + j) * C8 + c8);
+      const __nv_bfloat16* b = reinterpret_cast<const __nv_bfloat16*>(&v);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] += __bfloat162float(b[e]);
+    }
+    uint4 o;
+    __nv_bfloat16* ob = reinterpret_cast<__nv_bfloat16*>(&o);
+#pragma unroll
+    for (int e = 0; e < 8; ++e) ob[e] = __float2bfloat16_rn(acc[e] / (float)HW);
+    y[i] = o;
+  }
+}
+
 int warp_rows_grid(int B) { return (B + 7) / 8; }
 
 // NHWC bf16 maxpool, 8 channels (16 B) per thread, 32-bit index math (C % 8 == 0)
@@ -394,6 +420,12 @@ void avgpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, 
   if (!total) return;
   if (bf16 && C % 8 == 0 && H * W >= 8 && ((uintptr_t)x % 16) == 0 && ((uintptr_t)y % 16) == 0) {
     launch_plain(avgpool8_kernel, dim3(N, (C / 8 + 31) / 32), dim3(256), 0, st, (const uint4*)x, (uint4*)y, H * W, C / 8);
+    CK(cudaGetLastError());
+    return;
+  }
+  if (bf16 && C % 8 == 0 && total / 8 < INT32_MAX && ((uintptr_t)x % 16) == 0 && ((uintptr_t)y % 16) == 0) {
+    launch_plain(avgpool_small8_kernel, dim3(grid_for(total / 8, 256)), dim3(256), 0, st, (const uint4*)x, (uint4*)y, N,
+                 H * W, C / 8);
     CK(cudaGetLastError());
     return;
   }

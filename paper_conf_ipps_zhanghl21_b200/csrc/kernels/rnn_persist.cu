@@ -194,6 +194,10 @@ __global__ void __launch_bounds__(kRThreads, 1)
   auto tile_n0 = [&](int i) { return ((int)(blockIdx.x + i * gridDim.x) % a.tiles_n) * BN; };
   auto tile_m0 = [&](int i) { return ((int)(blockIdx.x + i * gridDim.x) / a.tiles_n) * RBM; };
   const int cta = blockIdx.x;
+  // packed k-block of the j-th load of a step: x blocks in order, then the h blocks rotated by
+  // a.hrot * CTA (all CTAs reading the same 16 KB h block at once queue on the same L2 lines)
+  const int hrot = kh > 0 ? (a.hrot * cta) % kh : 0;
+  auto kblk = [&](int j) { return j < kx ? j : kx + (j - kx + hrot) % kh; };
   unsigned long long* trace = (a.dbg & 1) && !MULTI && cta < 128 ? g_rp_trace + (size_t)cta * 64 * 16 : nullptr;
   // several tiles per CTA: stamps per work unit u = t * my_tiles + i < 64 (tools/rnn_trace_multi.py):
   // 0 barrier observed (i = 0), 7 first A load issued, 11 first W load issued, 1 first stage landed,
@@ -262,7 +266,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
             if (j < kx) {
               ptx::tma_load_2d(&tmX, &full[s], sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
             } else {  // h_{t-1}: one contiguous, pre-swizzled 16 KB block (see hs_index)
-              const __nv_bfloat16* src = a.hbuf[(t - 1) & 1] + ((size_t)(j - kx) * a.Bp + m0) * RBK;
+              const __nv_bfloat16* src = a.hbuf[(t - 1) & 1] + ((size_t)(kblk(j) - kx) * a.Bp + m0) * RBK;
               ptx::bulk_g2s(sA + s * R_A_BYTES, src, R_A_BYTES, &full[s]);
             }
           }
@@ -292,7 +296,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
             if (lane == 0) {
               ptx::mbar_arrive_expect_tx(&full[s], C::B_BYTES);
               // packed weight columns: [x part (kx blocks) | h part (kh blocks)] -> column block j
-              ptx::tma_load_2d(&tmW, &full[s], sB + s * C::B_BYTES, j * RBK, n0);
+              ptx::tma_load_2d(&tmW, &full[s], sB + s * C::B_BYTES, kblk(j) * RBK, n0);
             }
             __syncwarp();
           }
@@ -326,7 +330,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
             if (j == kx) mtr[u * 16 + 4] = rp_gtimer();
           }
           const uint64_t da = da0 + (uint64_t)((s * R_A_BYTES) >> 4);
-          const uint64_t db = db0 + (uint64_t)(((WRES ? j : s) * C::B_BYTES) >> 4);
+          const uint64_t db = db0 + (uint64_t)(((WRES ? kblk(j) : s) * C::B_BYTES) >> 4);
           if (!(a.dbg & 16))
 #pragma unroll
             for (int k = 0; k < RBK / 16; ++k) ptx::umma_bf16_elect(d, da + 2 * k, db + 2 * k, idesc, (j | k) != 0);
@@ -637,6 +641,9 @@ __global__ void __launch_bounds__(kRThreads, 1)
   const uint32_t rank = crank & 1;
   const uint32_t leader = crank & ~1u;
   const int pair = (int)blockIdx.x >> 1, n_pairs = (int)gridDim.x >> 1;
+  // h k-blocks rotated per pair (both CTAs of a pair load the same order; see rnn_persist_kernel)
+  const int hrot = kh > 0 ? (a.hrot * pair) % kh : 0;
+  auto kblk = [&](int j) { return j < kx ? j : kx + (j - kx + hrot) % kh; };
   const int n_ptiles = a.tiles_n * (a.tiles_m >> 1);
   const int n_tiles = a.tiles_n * a.tiles_m;  // 128-row CTA tiles (grid-barrier releases per step)
   const int my_tiles = (n_ptiles - 1 - pair) / n_pairs + 1;
@@ -699,7 +706,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
             if (j < kx) {
               ptx::tma_load_2d_2sm(&tmX, fb, sA + s * R_A_BYTES, j * RBK, t * a.B + m0);
             } else {  // pre-swizzled 16 KB h block through a SWIZZLE_NONE map (bytes land as stored)
-              ptx::tma_load_2d_2sm(((t - 1) & 1) ? &tmH1 : &tmH0, fb, sA + s * R_A_BYTES, 0, (j - kx) * a.Bp + m0);
+              ptx::tma_load_2d_2sm(((t - 1) & 1) ? &tmH1 : &tmH0, fb, sA + s * R_A_BYTES, 0, (kblk(j) - kx) * a.Bp + m0);
             }
           }
           __syncwarp();
@@ -720,7 +727,7 @@ __global__ void __launch_bounds__(kRThreads, 1)
           if (lane == 0) {
             const uint32_t fb = full_l0 + s * 8;
             if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * kPWBytes);
-            ptx::tma_load_2d_2sm(&tmW, fb, sB + s * kPWBytes, j * RBK, n0 + (int)rank * (BN / 2));
+            ptx::tma_load_2d_2sm(&tmW, fb, sB + s * kPWBytes, kblk(j) * RBK, n0 + (int)rank * (BN / 2));
           }
           __syncwarp();
         }

@@ -445,6 +445,8 @@ void build_op(Program& P, const Node& n, Op& op) {
       static const int msync_env = getenv("DUET_RNN_MSYNC") ? atoi(getenv("DUET_RNN_MSYNC")) : 1;
       const bool several = (int64_t)tiles * mt > grid;
       ra.msync = msync_env == 2 || (msync_env == 1 && (several || mt >= 4)) ? 1 : 0;
+      static const int hrot_env = getenv("DUET_RNN_HROT") ? atoi(getenv("DUET_RNN_HROT")) : 1;
+      ra.hrot = hrot_env;
       ra.wcat = Wcat;
       ra.w_rows = Np;
       ra.w_cols = Kc;

@@ -314,6 +314,32 @@ def test_conv_node_f32(N, H, W, C, Co, k, stride, pad):
     """fp32 mode on the tensor cores (gemm_tf32.cu) against the float64 oracle at the fp32 bar."""
     test_conv_node(N, H, W, C, Co, k, stride, pad, dt="f32")
 
+@pytest.mark.parametrize("N,H,W,C", [
+    (5, 1, 1, 512),     # c5's layer-4 map: the small-map average pool is a per-chunk copy
+    (3, 2, 3, 64),      # HW < 8: small-map kernel
+    (2, 7, 7, 512),     # c4's layer-4 map (HW >= 8: split-HW kernel)
+    (3, 9, 5, 24),      # C % 8 == 0 (3 chunks)
+    (2, 3, 3, 20),      # C % 8 != 0: scalar kernel
+])
+def test_pool_nodes(N, H, W, C):
+    """Global average pool and 3x3/2 max pool nodes against the oracle (bf16 storage)."""
+    Hp, Wp = (H - 1) // 2 + 1, (W - 1) // 2 + 1
+    ir = "\n".join([f"%x = input() : bf16[{N},{H},{W},{C}]", f"%a = avgpool(%x) : bf16[{N},{C}]",
+                     f"%y = maxpool(%x) {{k=3, stride=2, pad=1}} : bf16[{N},{Hp},{Wp},{C}]", "output %a",
+                     "output %y"]) + "\n"
+    x = _rand((N, H, W, C), "bf16", 2.0, 41)
+    g = duet.Graph(ir)
+    a = torch.empty((N, C), dtype=torch.bfloat16, device="cuda")
+    y = torch.empty((N, Hp, Wp, C), dtype=torch.bfloat16, device="cuda")
+    g.node_run("a", [x.cuda()], a)
+    g.node_run("y", [x.cuda()], y)
+    torch.cuda.synchronize()
+    xf = OF.to_f64(to_np(x), "bf16")
+    check(a.float().cpu().numpy(), OF.avgpool(xf), TOL["bf16"], f"avgpool {N}x{H}x{W}x{C}")
+    # a max of bf16 values is one of them: exact
+    np.testing.assert_array_equal(y.float().cpu().numpy(), OF.maxpool(xf, 3, 2, 1))
+
+
 _HALO_SCRIPT = r'''
 import os, sys
 sys.path.insert(0, os.environ["REPO"])
