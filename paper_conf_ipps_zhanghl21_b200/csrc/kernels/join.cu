@@ -268,6 +268,61 @@ __global__ void maxpool3s2_kernel(const uint4* __restrict__ x, uint4* __restrict
   }
 }
 
+// ResNet maxpool (3x3, stride 2, pad 1), NHWC bf16, C % 8 == 0, staged (round 2): a CTA pools
+// output rows [ho0, ho0 + k) of one image from the input rows they read, [2 ho0 - 1, 2 ho0 + 2k),
+// which are contiguous in NHWC: ONE bulk copy into shared memory, then the nine taps per 16-byte
+// output chunk come from there (the per-thread nine-load kernel above reached ~0.5 of HBM).  Every
+// window holds its centre pixel, so the max starts from it (no -inf padding needed).
+__device__ __forceinline__ uint4 bmax8(uint4 a, uint4 b) {
+  uint32_t* pa = reinterpret_cast<uint32_t*>(&a);
+  const uint32_t* pb = reinterpret_cast<const uint32_t*>(&b);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    __nv_bfloat162 r = __hmax2(*reinterpret_cast<const __nv_bfloat162*>(&pa[q]), *reinterpret_cast<const __nv_bfloat162*>(&pb[q]));
+    pa[q] = *reinterpret_cast<uint32_t*>(&r);
+  }
+  return a;
+}
+__global__ void maxpool3s2_rows_kernel(const uint4* __restrict__ x, uint4* __restrict__ y, int H, int W, int C8, int Ho,
+                                       int Wo, int k) {
+  extern __shared__ __align__(128) uint4 srows[];
+  __shared__ __align__(8) uint64_t bar;
+  const int bands = (Ho + k - 1) / k;
+  const int n = blockIdx.x / bands, ho0 = (blockIdx.x % bands) * k, ho1 = min(Ho, ho0 + k);
+  const int r0 = max(0, 2 * ho0 - 1), r1 = min(H, 2 * ho1);
+  const uint32_t bytes = (uint32_t)((r1 - r0) * W * C8 * 16);
+  if (threadIdx.x == 0) {
+    ptx::mbar_init(&bar, 1);
+    ptx::fence_mbar_init();
+  }
+  __syncthreads();
+  ptx::pdl_wait();
+  ptx::pdl_trigger();
+  if (threadIdx.x == 0) {
+    ptx::mbar_arrive_expect_tx(&bar, bytes);
+    ptx::bulk_g2s(srows, x + ((size_t)n * H + r0) * W * C8, bytes, &bar);
+  }
+  ptx::mbar_wait(&bar, 0);
+  const int total = (ho1 - ho0) * Wo * C8;
+  uint4* yo = y + ((size_t)n * Ho + ho0) * Wo * C8;
+  for (int i = threadIdx.x; i < total; i += blockDim.x) {
+    const int c8 = i % C8, t = i / C8, wo = t % Wo, ho = ho0 + t / Wo;
+    uint4 m = srows[((2 * ho - r0) * W + 2 * wo) * C8 + c8];
+#pragma unroll
+    for (int r = -1; r <= 1; ++r) {
+      const int hi = 2 * ho + r;
+      if (hi < r0 || hi >= r1) continue;
+#pragma unroll
+      for (int q = -1; q <= 1; ++q) {
+        const int wi = 2 * wo + q;
+        if (wi < 0 || wi >= W || (r == 0 && q == 0)) continue;
+        m = bmax8(m, srows[((hi - r0) * W + wi) * C8 + c8]);
+      }
+    }
+    yo[i] = m;
+  }
+}
+
 // global average pool, NHWC bf16, C % 8 == 0: block = (image n, 32 chunks of 8 channels); its 8
 // warps split the HW positions (warp w takes j = w, w + 8, ...), lane = channel chunk, 4 loads in
 // flight per lane, then the 8 partial sums are added in warp order in shared memory (fixed order:
@@ -394,6 +449,22 @@ void maxpool_nhwc(const void* x, void* y, int bf16, int N, int H, int W, int C, 
   if (!total) return;
   const bool vec = bf16 && C % 8 == 0 && total / 8 < INT32_MAX && (int64_t)N * H * W * C / 8 < INT32_MAX &&
                    ((uintptr_t)x % 16) == 0 && ((uintptr_t)y % 16) == 0;
+  const int64_t row_bytes = (int64_t)W * C * 2;
+  if (vec && k == 3 && s == 2 && p == 1 && 3 * row_bytes <= 64 * 1024) {
+    // output rows per CTA: the most whose input rows fit in 64 KB of shared memory
+    const int kr = std::max(1, std::min(Ho, (int)((64 * 1024 / row_bytes - 1) / 2)));
+    const int bands = (Ho + kr - 1) / kr;
+    const size_t smem = (size_t)std::min<int64_t>(H, 2 * kr + 1) * row_bytes;
+    static size_t attr = 0;
+    if (smem > attr) {
+      CK(cudaFuncSetAttribute(maxpool3s2_rows_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      attr = smem;
+    }
+    launch_plain(maxpool3s2_rows_kernel, dim3((unsigned)((int64_t)N * bands)), dim3(256), smem, st, (const uint4*)x,
+                 (uint4*)y, H, W, C / 8, Ho, Wo, kr);
+    CK(cudaGetLastError());
+    return;
+  }
   if (vec && k == 3 && s == 2 && p == 1) {
     launch_plain(maxpool3s2_kernel, dim3(grid_for(total / 8, 256, 16)), dim3(256), 0, st, (const uint4*)x, (uint4*)y, N, H,
                  W, C / 8, Ho, Wo);

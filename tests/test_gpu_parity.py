@@ -320,6 +320,9 @@ def test_conv_node_f32(N, H, W, C, Co, k, stride, pad):
     (2, 7, 7, 512),     # c4's layer-4 map (HW >= 8: split-HW kernel)
     (3, 9, 5, 24),      # C % 8 == 0 (3 chunks)
     (2, 3, 3, 20),      # C % 8 != 0: scalar kernel
+    (2, 112, 112, 64),  # c4's max pool input: staged bands of output rows
+    (5, 16, 16, 64),    # c5's: a whole image per CTA
+    (3, 15, 9, 64),     # odd H / W: the last window is clipped
 ])
 def test_pool_nodes(N, H, W, C):
     """Global average pool and 3x3/2 max pool nodes against the oracle (bf16 storage)."""
