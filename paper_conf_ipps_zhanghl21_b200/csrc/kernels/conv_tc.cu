@@ -352,11 +352,17 @@ void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void
     CUtensorMap tx = make_tmap_im2col(x, s);
     switch (bn) {
       case 64: {
-        // two CTAs per SM for the 64-channel layers (2 stages each): measured c5 layer 1 (8x8x64,
-        // B = 4096) 70.6 -> 56.9 us, c5 p50 -2.5% (two runs each); DUET_CONV_OCC=1: one CTA, 4 stages
-        static const int occ = getenv("DUET_CONV_OCC") ? atoi(getenv("DUET_CONV_OCC")) : 2;
+        // several CTAs per SM for the 64-channel layers: their tiles are bound by per-tile TMA round
+        // trips, and independent CTAs (each its own ring, MMA warp and epilogue) overlap them.
+        // Measured (conv_one, CUDA graphs, same box; profiles/r2_conv_occ.log): c5 layer 1 (4096 x
+        // 8x8x64) 1 CTA 70.6, 2 CTAs 37.6, 3 CTAs with one-k-block stages 32.8, 4 CTAs 33.5 us;
+        // c4 layer 1 (64 x 56x56x64) 31.5 / 26.9 / 28.2 us (the SMEM-halo kernel 30.0).
+        // DUET_CONV_OCC: 1, 2 (two-k-block stages), 4 = that many CTAs; default 3
+        static const int occ = getenv("DUET_CONV_OCC") ? atoi(getenv("DUET_CONV_OCC")) : 3;
+        if (occ == 1) return launch_conv_tma<64>(tx, tw, a, st);
         if (occ == 2) return launch_conv_tma<64, 2>(tx, tw, a, st);
-        return launch_conv_tma<64>(tx, tw, a, st);
+        if (occ == 4) return launch_conv_tma<64, 4, 1>(tx, tw, a, st);
+        return launch_conv_tma<64, 3, 1>(tx, tw, a, st);
       }
       // (two CTAs per SM with one-k-block stages for 128-wide tiles measured -9% .. +18% across
       // the c4 / c5 shapes and c4 p50 unchanged: not used, profiles/r2_conv.md)

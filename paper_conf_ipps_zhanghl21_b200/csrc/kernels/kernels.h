@@ -205,17 +205,6 @@ int conv_tc_pick_bn(const ConvShape& s, int num_sms);
 void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
              const ConvShape& s, int K, int act, const ConvPlan& p, unsigned* ctr, cudaStream_t st);
 bool conv_tma_ok(const ConvShape& s);
-// Halo implicit-GEMM 3x3/s1/p1 conv (conv_halo.cu): input tile + zero halo loaded once per
-// 64-channel block, the nine taps read from shared memory.
-struct HaloPlan {
-  bool ok = false;
-  int bn = 64, hb = 0, ni = 1, Hs = 0, bands = 1, a_bytes = 0, box_bytes = 0, a_stages = 2, b_stages = 0, bres = 0,
-      smem = 0;
-  int64_t units = 0;
-};
-HaloPlan conv_halo_plan(const ConvShape& s, int num_sms, bool force = false);
-void conv_halo(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y, const ConvShape& s,
-               int act, const HaloPlan& p, unsigned* ctr, cudaStream_t st);  // ctr: as conv_tc
 // Explicit im2col (layers with C % 64 != 0): cols[m, k] = x[n, ho*s-p+r, wo*s-p+q, c], k = (r, q, c),
 // rows padded to ldk (zeros), bf16.
 void im2col(const void* x, void* cols, const ConvShape& s, int64_t ldk, cudaStream_t st);

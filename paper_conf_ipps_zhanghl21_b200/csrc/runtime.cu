@@ -600,22 +600,8 @@ void build_op(Program& P, const Node& n, Op& op) {
     float* bias = (float*)P.alloc((int64_t)s.Co * 4);
     fold_bn(P.param(n.params[0]), bf, (const float*)P.param(n.params[1]), (const float*)P.param(n.params[2]),
             (const float*)P.param(n.params[3]), (const float*)P.param(n.params[4]), Wf, bias, s.Co, per_co, ldw, 0);
-    // DUET_CONV_HALO: 0 = never, 2 = wherever eligible (tests), default = where measured faster
-    static const int halo_mode = getenv("DUET_CONV_HALO") ? atoi(getenv("DUET_CONV_HALO")) : 1;
-    const HaloPlan halo = (tma && halo_mode) ? conv_halo_plan(s, sms, halo_mode == 2) : HaloPlan{};
     static const bool conv_dyn = !(getenv("DUET_CONV_DYN") && atoi(getenv("DUET_CONV_DYN")) == 0);
-    if (halo.ok) {
-      CUtensorMap tw = make_tmap_bf16_2d(Wf, s.Co, ldw, halo.bn);
-      unsigned* ctr = nullptr;
-      if (conv_dyn) {
-        ctr = (unsigned*)P.alloc(2 * sizeof(unsigned));
-        CK(cudaMemset(ctr, 0, 2 * sizeof(unsigned)));
-      }
-      op.launch = [=](const Ptrs& T, cudaStream_t st) {
-        conv_halo(tw, T[in], bias, res >= 0 ? T[res] : nullptr, T[dst], s, act, halo, ctr, st);
-      };
-      op.n_kernels = 1;
-    } else if (tma) {
+    if (tma) {
       ConvPlan plan = conv_tc_plan(s, sms);
       if (const char* f = getenv("DUET_CONV_BN")) {  // tile-width sweeps (tools/plan_sweep.sh)
         const int fb = atoi(f);

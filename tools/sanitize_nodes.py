@@ -25,7 +25,7 @@ def node(ir, params, args, out_shape, out_dt=torch.bfloat16):
 
 
 def main():
-    which = sys.argv[1:] or ["gemm", "rnn", "conv", "stem", "conv7", "halo", "c2"]
+    which = sys.argv[1:] or ["gemm", "rnn", "conv", "stem", "conv7", "c2"]
     gen = torch.Generator().manual_seed(0)
     r = lambda *s, sc=1.0: ((torch.rand(*s, generator=gen) * 2 - 1) * sc).to(torch.bfloat16)
     if "gemm" in which:
@@ -43,8 +43,7 @@ def main():
               "bhh": torch.zeros(3 * H)}, [r(S, B, E)], (B, H))
         print("rnn ok", flush=True)
     for key, (N_, H_, C, Co, k, s, p) in (("conv", (2, 14, 64, 64, 3, 1, 1)), ("stem", (1, 64, 3, 64, 7, 2, 3)),
-                                              ("conv7", (16, 7, 512, 512, 3, 1, 1)),
-                                              ("halo", (2, 56, 64, 64, 3, 1, 1))):
+                                              ("conv7", (16, 7, 512, 512, 3, 1, 1))):
         if key not in which:
             continue
         Ho, Wo = (H_ + 2 * p - k) // s + 1, (H_ + 2 * p - k) // s + 1
