@@ -1,7 +1,7 @@
 """DUET on B200 — benchmark (driver contract: one JSON line on rank 0).
 
 Headline workload: BASELINE.json configs[4] (c5, the 8-way heterogeneous ensemble, batch 4096), the
-largest configuration that fits one GPU; `per_config` adds c1-c4 (configs[0..3]) measured the same
+largest configuration that fits one GPU; `per_config` adds c1-c4 (configs[0..3]) and c6 (MT-DNN) measured the same
 way in the same run (BASELINE.json:2 "per model").  A *step* = one inference of one batch through
 the whole hot path, executed by libduet's greedy-correction schedule on CUDA-stream slots (one
 CUDA-graph replay).
@@ -53,7 +53,7 @@ def parse():
     ap.add_argument("--config", default="c5", choices=["c1", "c2", "c3", "c4", "c5", "c6"],
                     help="c1-c5 = BASELINE.json configs[0..4]; c6 = MT-DNN (SURVEY.md §8(f) N4(b), not a BASELINE config)")
     ap.add_argument("--per-config", default="auto",
-                    help="comma list of extra configs measured in the same run ('auto': c1-c4 beside a c5 headline "
+                    help="comma list of extra configs measured in the same run ('auto': c1-c4 and c6 beside a c5 headline "
                          "at N = 1; 'none')")
     ap.add_argument("--slots", type=int, default=2, help="CUDA-stream slots on the GPU")
     ap.add_argument("--dtype", default=None, choices=[None, "bf16", "f32"])
@@ -495,7 +495,7 @@ def bench_single(args):
     extra = {}
     pcs = args.per_config
     if pcs == "auto":
-        pcs = "c1,c2,c3,c4" if (args.config == "c5" and world == 1) else "none"
+        pcs = "c1,c2,c3,c4,c6" if (args.config == "c5" and world == 1) else "none"
     if pcs != "none" and rank == 0:
         for c in [c for c in pcs.split(",") if c and c != args.config]:
             torch.cuda.empty_cache()
