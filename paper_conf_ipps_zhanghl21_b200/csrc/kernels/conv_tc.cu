@@ -366,7 +366,21 @@ void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void
       }
       // (two CTAs per SM with one-k-block stages for 128-wide tiles measured -9% .. +18% across
       // the c4 / c5 shapes and c4 p50 unchanged: not used, profiles/r2_conv.md)
-      case 128: return launch_conv_tma<128>(tx, tw, a, st);
+      case 128: {
+        // two CTAs per SM (one-k-block stages) once the tiles outnumber the SMs (with fewer, the
+        // second CTA of an SM only halves the first's share): c5 layer 3 (4096 x 2x2x256) 26.1 ->
+        // 21.8 us, layer 2 27.5 -> 24.7, c4 layer 3 25.7 -> 21.9, layer 2 22.4 -> 21.3; c4 layer 4
+        // (100 tiles) 25.2 -> 33.0 with two, so it keeps one (profiles/r2_conv_occ128.log).
+        // DUET_CONV_OCC128: 1 / 2 force one / two CTAs per SM
+        static const int occ128 = getenv("DUET_CONV_OCC128") ? atoi(getenv("DUET_CONV_OCC128")) : 0;
+        const int64_t M = (int64_t)s.N * s.Ho * s.Wo;
+        const int64_t tiles = ((M + CBM - 1) / CBM) * ((s.Co + 127) / 128);
+        int dev = 0;
+        cudaGetDevice(&dev);
+        const bool two = occ128 == 2 || (occ128 == 0 && tiles > num_sms(dev));
+        if (two) return launch_conv_tma<128, 2, 1>(tx, tw, a, st);
+        return launch_conv_tma<128>(tx, tw, a, st);
+      }
       case 256: return launch_conv_tma<256>(tx, tw, a, st);
     }
   }
