@@ -1219,7 +1219,15 @@ Schedule* schedule_measured(const Partition* p, const Profile* pr, const duet_sc
   fill_inputs(*P, home);
   for (int s = 0; s < p->n_sg(); ++s) launch_subgraph(*P, *p, s, P->buf, home);  // real data everywhere
   CK(cudaStreamSynchronize(home));
-  std::vector<cudaEvent_t> ev(opts.samples + 1);
+  // Each timed replay starts with a cold L2 (a 256 MB write first, outside the timed interval), as
+  // bench.py times every step: a candidate is judged under the condition its latency is reported
+  // for (back-to-back warm replays favoured assignments whose inputs stay cached).
+  // DUET_MEASURE_FLUSH=0: back-to-back replays.
+  static const bool cold = !(getenv("DUET_MEASURE_FLUSH") && atoi(getenv("DUET_MEASURE_FLUSH")) == 0);
+  static void* flush_buf = nullptr;
+  const size_t flush_bytes = (size_t)256 << 20;
+  if (cold && !flush_buf) CK(cudaMalloc(&flush_buf, flush_bytes));
+  std::vector<cudaEvent_t> ev(2 * opts.samples + 1);
   for (auto& e : ev) CK(cudaEventCreate(&e));
   std::map<std::vector<int>, int64_t> memo;
   static const bool log = getenv("DUET_MEASURE_LOG") != nullptr;
@@ -1238,15 +1246,25 @@ Schedule* schedule_measured(const Partition* p, const Profile* pr, const duet_sc
     std::vector<double> ns;
     try {
       for (int w = 0; w < opts.warmup; ++w) CK(cudaGraphLaunch(E.exec, home));
-      CK(cudaEventRecord(ev[0], home));
-      for (int k = 0; k < opts.samples; ++k) {
-        CK(cudaGraphLaunch(E.exec, home));
-        CK(cudaEventRecord(ev[k + 1], home));
+      if (cold) {
+        for (int k = 0; k < opts.samples; ++k) {
+          CK(cudaMemsetAsync(flush_buf, k & 0xff, flush_bytes, home));
+          CK(cudaEventRecord(ev[2 * k], home));
+          CK(cudaGraphLaunch(E.exec, home));
+          CK(cudaEventRecord(ev[2 * k + 1], home));
+        }
+      } else {
+        CK(cudaEventRecord(ev[0], home));
+        for (int k = 0; k < opts.samples; ++k) {
+          CK(cudaGraphLaunch(E.exec, home));
+          CK(cudaEventRecord(ev[k + 1], home));
+        }
       }
       CK(cudaStreamSynchronize(home));
       for (int k = 0; k < opts.samples; ++k) {
         float ms = 0;
-        CK(cudaEventElapsedTime(&ms, ev[k], ev[k + 1]));
+        if (cold) CK(cudaEventElapsedTime(&ms, ev[2 * k], ev[2 * k + 1]));
+        else CK(cudaEventElapsedTime(&ms, ev[k], ev[k + 1]));
         ns.push_back(ms * 1e6);
       }
     } catch (...) {
