@@ -414,8 +414,15 @@ __global__ void __launch_bounds__(kRThreads, 1)
           // are ordered before the release-add by __syncwarp; the consumer acquires the counter and
           // issues fence.proxy.async before its TMA reads
           fence_proxy_async_global();
-          __syncwarp();
-          if (lane == 0) red_release_gpu_add(a.counter + (a.msync ? tile_m0(0) / RBM : 0), 1u);
+          if (a.ctarel) {
+            // one release per CTA (counting its eight warps): an eighth of the same-address atomics
+            // at the counter's L2 slice; bar.sync orders every warp's stores before it (cumulative)
+            asm volatile("bar.sync 1, %0;" ::"n"(32 * kREpiWarps) : "memory");
+            if (threadIdx.x == 64) red_release_gpu_add(a.counter + (a.msync ? tile_m0(0) / RBM : 0), (unsigned)kREpiWarps);
+          } else {
+            __syncwarp();
+            if (lane == 0) red_release_gpu_add(a.counter + (a.msync ? tile_m0(0) / RBM : 0), 1u);
+          }
           if (trace && t < 64 && threadIdx.x == 64) trace[t * 16 + 3] = rp_gtimer();
         }
       }

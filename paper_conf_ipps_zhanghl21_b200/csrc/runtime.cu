@@ -447,6 +447,11 @@ void build_op(Program& P, const Node& n, Op& op) {
       ra.msync = msync_env == 2 || (msync_env == 1 && (several || mt >= 4)) ? 1 : 0;
       static const int hrot_env = getenv("DUET_RNN_HROT") ? atoi(getenv("DUET_RNN_HROT")) : 1;
       ra.hrot = hrot_env;
+      // one release per CTA instead of one per epilogue warp (same-address atomics at the counter's
+      // L2 slice): c3 tower 393 -> 374 us, c4 GRU 587 -> 567, c5 LSTM256 424 -> 404
+      // (profiles/r2_ctarel_ab.log); DUET_RNN_CTAREL=0 restores per-warp releases
+      static const int ctarel_env = getenv("DUET_RNN_CTAREL") ? atoi(getenv("DUET_RNN_CTAREL")) : 1;
+      ra.ctarel = ctarel_env;
       ra.wcat = Wcat;
       ra.w_rows = Np;
       ra.w_cols = Kc;
