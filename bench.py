@@ -249,6 +249,20 @@ def load_peaks():
         return 6650.0, 1590.0, 1590.0, "fallback"
 
 
+def node_executed(wl, node):
+    """FLOP the kernels actually issue for one launch of `node`: the algorithmic count with the
+    recurrences' padding -- four gate blocks for GRU too (n_x and n_h kept apart), batch
+    rows padded to the 128-row tiles, E padded to 64 -- (GEMMs: the algorithmic count)."""
+    op, args, _, shape = node_decl(wl, node)
+    if op in ("lstm", "gru"):
+        _, _, _, xs = node_decl(wl, args[0])
+        S, B, E = xs
+        H = shape[-1]
+        Bp, Ep = -(-B // 128) * 128, -(-E // 64) * 64
+        return 2 * S * Bp * 4 * H * (Ep + H)
+    return node_work(wl, node)
+
+
 def roofline(torch, cfg, wl, sess, flush):
     node = DOMINANT.get(cfg)
     if node is None:
@@ -270,7 +284,10 @@ def roofline(torch, cfg, wl, sess, flush):
             "frac_vs_sustained": round(achieved / sustained, 4),
             "algorithmic_per_launch": work, "ms_per_launch": round(cold_ms, 5), "timing": "cold (L2 flushed)",
             "warm_ms_per_launch": round(warm_ms, 5),
-            "warm_frac": round(work / (warm_ms / 1e3) / 1e12 / burst, 4)}
+            "warm_frac": round(work / (warm_ms / 1e3) / 1e12 / burst, 4),
+            # secondary: the rate on the FLOP the kernel issues (GRU's fourth gate block, tile padding)
+            "executed_per_launch": node_executed(wl, node),
+            "frac_executed": round(node_executed(wl, node) / (cold_ms / 1e3) / 1e12 / peak, 4)}
 
 
 # ---------------------------------------------------------------------------------------------
