@@ -272,6 +272,8 @@ def test_c2_full_size_sampled():
     (3, 28, 28, 128, 128, 3, 1, 1),   # layer-2 shape
     (7, 8, 8, 64, 64, 3, 1, 1),       # c5 layer-1 shape
     (3, 12, 20, 64, 48, 3, 1, 1),     # W != H, Co < tile
+    (32, 28, 28, 128, 128, 3, 1, 1),  # 196 128-wide tiles > SMs: two CTAs per SM
+    (64, 14, 14, 256, 256, 3, 1, 1),  # c4 layer 3 (two CTAs per SM)
 ])
 
 def test_conv_node(N, H, W, C, Co, k, stride, pad, dt="bf16"):
