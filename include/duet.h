@@ -266,6 +266,17 @@ void duet_schedule_destroy(duet_schedule_t* s);
 duet_status duet_run(duet_schedule_t* s, const duet_slot* slots, int n_slots, const duet_tensor* inputs,
                      int n_in, duet_tensor* outputs, int n_out);
 
+/* Device trace of the executor (§IV-D: the executor starts a subgraph once its
+ * predecessors finish).  With tracing on, later duet_run calls of this schedule record a timing
+ * event at the fork and around every subgraph on its slot stream (a separate cached graph; the
+ * untraced graph is unchanged).  duet_schedule_trace waits for the last traced run and writes, per
+ * subgraph, start_ns[i] / end_ns[i] = its first kernel's start / last kernel's end in ns after the
+ * fork (event resolution ~0.5 us); n_sg must equal the partition's subgraph count.  DUET_ESTATE
+ * when the last run was not traced.  Either array may be NULL.  tools/trace_json.py writes them
+ * as a Chrome trace; tests check start(v) >= end(u) on every partition edge. */
+duet_status duet_schedule_set_trace(duet_schedule_t* s, int on);
+duet_status duet_schedule_trace(const duet_schedule_t* s, int64_t* start_ns, int64_t* end_ns, int32_t n_sg);
+
 /* Number of kernel launches one duet_run of this schedule performs (for the bench's
  * "gpu_launches" claim).  Valid after the first duet_run. */
 duet_status duet_schedule_launch_count(const duet_schedule_t* s, int64_t* n_kernels);

@@ -273,6 +273,20 @@ duet_status duet_run(duet_schedule_t* s, const duet_slot* slots, int n_slots, co
   });
 }
 
+duet_status duet_schedule_set_trace(duet_schedule_t* s, int on) {
+  return guard([&] {
+    need(s, "schedule");
+    s->s->trace = on ? 1 : 0;
+  });
+}
+
+duet_status duet_schedule_trace(const duet_schedule_t* s, int64_t* start_ns, int64_t* end_ns, int32_t n_sg) {
+  return guard([&] {
+    need(s, "schedule");
+    schedule_trace_export(s->s.get(), start_ns, end_ns, n_sg);
+  });
+}
+
 duet_status duet_schedule_launch_count(const duet_schedule_t* s, int64_t* n_kernels) {
   return guard([&] {
     need(s, "schedule");

@@ -114,6 +114,7 @@ struct Schedule {
   int64_t makespan = 0;
   int fell_back = 0;
   int64_t measured_ns = -1;         // measured mode: device latency of slot_of (else -1)
+  int trace = 0;                    // 1: duet_run records per-subgraph start / end events
   std::shared_ptr<ExecCache> exec;  // captured CUDA graphs (runtime.cu)
   ~Schedule();
 };
@@ -135,6 +136,8 @@ Profile* profile_on_device(const Partition* p, const duet_slot* slots, int n_slo
 void run_schedule(Schedule* s, const duet_slot* slots, int n_slots, const duet_tensor* in, int n_in,
                   duet_tensor* out, int n_out);
 int64_t schedule_launch_count(const Schedule* s);
+// per-subgraph [start, end) of the last traced duet_run, ns after its fork (waits for that run)
+void schedule_trace_export(const Schedule* s, int64_t* start_ns, int64_t* end_ns, int n);
 void node_run(Graph* g, const std::string& node, const duet_tensor* args, int n_args, duet_tensor* out,
               void* stream);
 void destroy_program(Program* p);

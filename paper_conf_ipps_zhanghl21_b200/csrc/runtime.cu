@@ -929,12 +929,18 @@ struct ExecEntry {
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t exec = nullptr;
   std::vector<cudaEvent_t> events;
+  // trace (Schedule::trace): timing events at the fork and around every subgraph (also in events),
+  // recorded as external event-record nodes of the graph (a plain record during capture only
+  // expresses a dependency)
+  cudaEvent_t t_fork = nullptr;
+  std::vector<cudaEvent_t> t_start, t_end;
 };
 
 struct ExecCache {
   int device = 0;
   std::vector<ExecEntry> entries;
   int64_t launches = 0;
+  int last = -1;  // entry of the last duet_run (trace export)
   std::weak_ptr<Program> prog;
   ~ExecCache() {
     int prev = 0;
@@ -975,6 +981,19 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
   std::vector<cudaEvent_t> done(n);
   for (int s = 0; s < n; ++s) done[s] = mk();
   cudaEvent_t fork = mk();
+  auto mk_timed = [&]() {
+    cudaEvent_t ev;
+    CK(cudaEventCreate(&ev));
+    E.events.push_back(ev);
+    return ev;
+  };
+  if (S.trace) {
+    E.t_fork = mk_timed();
+    for (int s = 0; s < n; ++s) {
+      E.t_start.push_back(mk_timed());
+      E.t_end.push_back(mk_timed());
+    }
+  }
   // subgraph-level predecessors
   std::vector<std::vector<int>> preds(n);
   for (auto& kv : part.edges)
@@ -1007,6 +1026,7 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
   CK(cudaStreamBeginCapture(home, cudaStreamCaptureModeRelaxed));
   try {
     CK(cudaEventRecord(fork, home));
+    if (S.trace) CK(cudaEventRecordWithFlags(E.t_fork, home, cudaEventRecordExternal));
     // pinned-host inputs/outputs are memcpy nodes of the same graph: one launch per inference
     for (size_t c = 0; c < h2d.size(); ++c) {
       CK(cudaStreamWaitEvent(side[c], fork, 0));
@@ -1033,8 +1053,10 @@ static ExecEntry capture(const Program& P, const Schedule& S, const std::vector<
       for (int u : preds[s])
         if (streams[S.slot_of[u]] != st) CK(cudaStreamWaitEvent(st, done[u], 0));
       for (int c : copies_of[s]) CK(cudaStreamWaitEvent(st, copied[c], 0));
+      if (S.trace) CK(cudaEventRecordWithFlags(E.t_start[s], st, cudaEventRecordExternal));
       launch_subgraph(P, part, s, T, st);
       nk += subgraph_kernels(P, part, s);
+      if (S.trace) CK(cudaEventRecordWithFlags(E.t_end[s], st, cudaEventRecordExternal));
       CK(cudaEventRecord(done[s], st));
       last_on[q] = s;
     }
@@ -1176,6 +1198,7 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
   for (auto st : streams) key.push_back((void*)st);
   for (auto& c : h2d) key.push_back(const_cast<void*>(c.src));
   for (auto& c : d2h) key.push_back(c.dst);
+  key.push_back((void*)(intptr_t)S->trace);
   ExecEntry* hit = nullptr;
   for (auto& e : S->exec->entries)
     if (e.key == key) hit = &e;
@@ -1194,7 +1217,24 @@ void run_schedule(Schedule* S, const duet_slot* slots, int n_slots, const duet_t
     S->exec->entries.push_back(std::move(E));
     hit = &S->exec->entries.back();
   }
+  S->exec->last = (int)(hit - S->exec->entries.data());
   CK(cudaGraphLaunch(hit->exec, home));
+}
+
+void schedule_trace_export(const Schedule* s, int64_t* start_ns, int64_t* end_ns, int n) {
+  if (!s->exec || s->exec->last < 0) fail(DUET_ESTATE, "no duet_run of this schedule yet");
+  const ExecEntry& E = s->exec->entries[s->exec->last];
+  if (!E.t_fork) fail(DUET_ESTATE, "the last duet_run was not traced (duet_schedule_set_trace)");
+  if (n != (int)E.t_start.size()) fail(DUET_EINVAL, "trace: n must equal the subgraph count");
+  DeviceGuard dg(s->exec->device);
+  for (int i = 0; i < n; ++i) {
+    CK(cudaEventSynchronize(E.t_end[i]));
+    float a = 0, b = 0;
+    CK(cudaEventElapsedTime(&a, E.t_fork, E.t_start[i]));
+    CK(cudaEventElapsedTime(&b, E.t_fork, E.t_end[i]));
+    if (start_ns) start_ns[i] = (int64_t)((double)a * 1e6);
+    if (end_ns) end_ns[i] = (int64_t)((double)b * 1e6);
+  }
 }
 
 // ------------------------------------------------------------------------------------------------

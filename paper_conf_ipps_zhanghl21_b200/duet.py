@@ -99,6 +99,8 @@ _sig = {
     "duet_schedule_destroy": (None, [_P]),
     "duet_run": (C.c_int, [_P, C.POINTER(Slot), C.c_int, C.POINTER(Tensor), C.c_int, C.POINTER(Tensor), C.c_int]),
     "duet_schedule_launch_count": (C.c_int, [_P, C.POINTER(C.c_int64)]),
+    "duet_schedule_set_trace": (C.c_int, [_P, C.c_int]),
+    "duet_schedule_trace": (C.c_int, [_P, C.POINTER(C.c_int64), C.POINTER(C.c_int64), C.c_int32]),
     "duet_node_run": (C.c_int, [_P, C.c_char_p, C.POINTER(Tensor), C.c_int, C.POINTER(Tensor), _P]),
 }
 for _name, (_res, _args) in _sig.items():
@@ -339,6 +341,16 @@ class Schedule:
         sa = make_slots(slots)
         ia, oa = _tensor_array(inputs), _tensor_array(outputs)
         _check(_lib.duet_run(self._h, sa, len(slots), ia, len(inputs), oa, len(outputs)))
+
+    def set_trace(self, on: bool = True) -> None:
+        _check(_lib.duet_schedule_set_trace(self._h, int(on)))
+
+    def trace(self) -> tuple:
+        """(start_ns, end_ns) per subgraph of the last traced duet_run, relative to its fork."""
+        n = self.prof.part.n_sg
+        a, b = np.zeros(n, np.int64), np.zeros(n, np.int64)
+        _check(_lib.duet_schedule_trace(self._h, _np_ptr(a, C.c_int64), _np_ptr(b, C.c_int64), n))
+        return a, b
 
     def launch_count(self) -> int:
         n = C.c_int64()

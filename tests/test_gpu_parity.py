@@ -713,3 +713,39 @@ def test_bench_contract_keys():
     c2 = d["per_config"]["c2"]
     assert c2["workload"] == "c2_wide_deep" and c2["roofline"]["frac"] > 0 and c2["speedup_vs_serial"] > 0
     assert c2["e2e"]["h2d_bytes_per_step"] == 2048 * 26 * 8
+
+
+@pytest.mark.parametrize("cfg", ["c2", "c4", "c5"])
+def test_executor_trace_dependencies(cfg):
+    """The executor's dependency contract on the device (§IV-D): with tracing on,
+    duet_run records each subgraph's start / end; every partition edge u -> v has start(v) >=
+    end(u), subgraphs on one slot never overlap, and the traced run's outputs equal the untraced
+    run's bit for bit (tracing adds event nodes only)."""
+    import os
+    import sys
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools"))
+    import trace_json as TJ
+    wl = W.build(cfg, small=True)
+    sess = Session(wl, n_slots=2, profile=FAST_PROFILE)
+    inputs = list(materialize(wl.inputs, "cuda").values())
+    for sched in (sess.schedule(), sess.prof.schedule(mode=duet.ROUND_ROBIN)):
+        ref = sess.outputs()
+        sess.run(sched, inputs, ref)
+        torch.cuda.synchronize()
+        with pytest.raises(duet.DuetError):
+            sched.trace()  # the last run was not traced
+        sched.set_trace(True)
+        outs = sess.outputs()
+        sess.run(sched, inputs, outs)
+        torch.cuda.synchronize()
+        start, end = sched.trace()
+        assert (end >= start).all() and (start >= 0).all()
+        assert TJ.violations(sess, start, end) == []
+        slot_of = sched.export()["slot_of"]
+        for d in set(slot_of):
+            iv = sorted((int(start[s]), int(end[s])) for s in range(len(slot_of)) if slot_of[s] == d)
+            assert all(b[0] >= a[1] for a, b in zip(iv, iv[1:])), iv
+        for r, o in zip(ref, outs):
+            assert torch.equal(r.cpu(), o.cpu())
+        sched.set_trace(False)
+
