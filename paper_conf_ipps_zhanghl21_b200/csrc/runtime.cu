@@ -1339,6 +1339,77 @@ Schedule* schedule_measured(const Partition* p, const Profile* pr, const duet_sc
     throw;
   }
   for (auto e : ev) cudaEventDestroy(e);
+  // Final verification against measurement noise (round 2): each candidate above was timed once,
+  // at a different moment (clocks drift under the power cap), and Step 3 keeps the minimum of noisy
+  // figures.  The K fastest assignments measured (the result included) are timed again, interleaved
+  // over R rounds so that drift hits them alike, and the lowest median is kept.  The reported
+  // assignment is still one Step 3 evaluated.  DUET_MEASURE_REFINE: K (default 4; <= 1: off).
+  static const int refine_k = getenv("DUET_MEASURE_REFINE") ? atoi(getenv("DUET_MEASURE_REFINE")) : 4;
+  if (refine_k > 1 && memo.size() > 1 && S->fell_back == 0) {
+    std::vector<std::pair<int64_t, std::vector<int>>> ranked;
+    for (auto& kv : memo) ranked.push_back({kv.second, kv.first});
+    std::sort(ranked.begin(), ranked.end());
+    std::vector<std::vector<int>> cands;
+    for (size_t i = 0; i < ranked.size() && (int)cands.size() < refine_k; ++i) cands.push_back(ranked[i].second);
+    if (std::find(cands.begin(), cands.end(), S->slot_of) == cands.end()) cands.push_back(S->slot_of);
+    const int rounds = 6, per = std::max(5, opts.samples / rounds);
+    std::vector<ExecEntry> ents;
+    std::vector<std::vector<double>> got(cands.size());
+    std::vector<cudaEvent_t> e2(2 * per);
+    for (auto& e : e2) CK(cudaEventCreate(&e));
+    auto cleanup = [&]() {
+      for (auto& E : ents) {
+        cudaGraphExecDestroy(E.exec);
+        cudaGraphDestroy(E.graph);
+        for (auto e : E.events) cudaEventDestroy(e);
+      }
+      for (auto e : e2) cudaEventDestroy(e);
+    };
+    try {
+      for (auto& a : cands) {
+        Schedule T;
+        T.p = p;
+        T.pr = pr;
+        T.slot_of = a;
+        for (int s = 0; s < p->n_sg(); ++s) T.order.push_back(s);
+        int64_t nk = 0;
+        ents.push_back(capture(*P, T, streams, P->buf, {}, {}, &nk));
+      }
+      for (int r = 0; r < rounds; ++r)
+        for (size_t c = 0; c < cands.size(); ++c) {
+          CK(cudaGraphLaunch(ents[c].exec, home));  // warm the graph, then cold timed replays
+          for (int k = 0; k < per; ++k) {
+            if (cold) CK(cudaMemsetAsync(flush_buf, k & 0xff, flush_bytes, home));
+            CK(cudaEventRecord(e2[2 * k], home));
+            CK(cudaGraphLaunch(ents[c].exec, home));
+            CK(cudaEventRecord(e2[2 * k + 1], home));
+          }
+          CK(cudaStreamSynchronize(home));
+          for (int k = 0; k < per; ++k) {
+            float ms = 0;
+            CK(cudaEventElapsedTime(&ms, e2[2 * k], e2[2 * k + 1]));
+            got[c].push_back(ms * 1e6);
+          }
+        }
+    } catch (...) {
+      cleanup();
+      delete S;
+      throw;
+    }
+    cleanup();
+    size_t best = 0;
+    std::vector<int64_t> med(cands.size());
+    for (size_t c = 0; c < cands.size(); ++c) {
+      med[c] = lower_median(got[c]);
+      if (med[c] < med[best]) best = c;
+    }
+    if (log)
+      for (size_t c = 0; c < cands.size(); ++c)
+        fprintf(stderr, "[refine] candidate %zu first %lld ns, interleaved %lld ns%s\n", c,
+                (long long)memo[cands[c]], (long long)med[c], c == best ? " (kept)" : "");
+    S->slot_of = cands[best];
+    S->measured_ns = med[best];
+  }
   if (mo) {
     mo->measured_ns = S->measured_ns;
     mo->evaluations = (int32_t)memo.size();

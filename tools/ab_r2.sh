@@ -32,5 +32,7 @@ case "$1" in
     for sh in "64 112 112 64" "4096 16 16 64"; do python tools/pool_time.py $sh; done ;;
   embed)   # token-embedding gathers (tools/embed_time.py)                       -> r2_embed_ab.log
     for sh in "32 4096 256" "64 4096 128" "16 4096 256" "64 256 256" "64 64 256"; do python tools/embed_time.py $sh; done ;;
-  *) echo "usage: bash tools/ab_r2.sh msync|ctarel|hrot|conv_occ|conv_occ128|conv_cfg|measure_flush|slots|pool|embed"; exit 1 ;;
+  refine)  # interleaved re-measurement of the 4 best candidates (4) vs Step 3's first figures (0)
+    for r in 1 2 3; do for m in 4 0; do for c in c5 c4; do echo -n "$c refine=$m: "; DUET_MEASURE_REFINE=$m cfg_line $c; done; done; done ;;
+  *) echo "usage: bash tools/ab_r2.sh msync|ctarel|hrot|conv_occ|conv_occ128|conv_cfg|measure_flush|slots|pool|embed|refine"; exit 1 ;;
 esac
