@@ -16,8 +16,8 @@ def main():
     tag = sys.argv[2]
     cfgs = list(res)
     print(f"# Scheduler comparison on B200, {tag} (SURVEY.md §8(f) N2; PAPER.md:88 Fig. 13)\n")
-    print(f"`python tools/fig13.py --configs {','.join(cfgs)}` on one B200, 2 stream slots, full sizes, bf16, the final "
-          f"kernels of round 1 (automatic RNN gate-tile width).  Per scheduler: measured p50 of its assignment (ms; CUDA "
+    print(f"`python tools/fig13.py --configs {','.join(cfgs)}` on one B200, 2 stream slots, full sizes, bf16, the library "
+          f"at the time of the run (automatic RNN gate-tile width).  Per scheduler: measured p50 of its assignment (ms; CUDA "
           f"events on the home stream, 50 replays, inputs resident, L2 warm) and, in brackets, the C3 model makespan "
           f"from the device profile.  Fallback disabled so every scheduler's own placement runs.  Raw: "
           f"`{tag}_fig13.json`.\n")
