@@ -956,11 +956,12 @@ bool launch_rp_pair(const CUtensorMap& tx, RnnPersistArgs a, int grid, cudaStrea
 }  // namespace
 
 bool rnn_pair_ok(int kind, int bn, int B, int tiles_n, int tiles_m, int sms) {
-  // DUET_RNN_PAIR: 0 = never, 2 = LSTM too (tests), default = GRU only -- measured against the
-  // one-CTA kernel on one box: GRU1024 at B = 4096 571 -> 542 us, GRU512 447 -> 447, LSTM512
-  // 503 -> 537
-  static const int mode = getenv("DUET_RNN_PAIR") ? atoi(getenv("DUET_RNN_PAIR")) : 1;
-  if (mode == 0 || (kind == EPI_LSTM && mode != 2)) return false;
+  // DUET_RNN_PAIR: 0 = never, 1 = GRU only, default 2 = GRU and LSTM -- measured against the
+  // one-CTA kernel on one box: GRU1024 at B = 4096 571 -> 542 us, GRU512 447 -> 447; LSTM512 503 ->
+  // 537 with the grid barrier, 417 -> 406 us once steps synchronise per row block (round 2,
+  // DESIGN.md "Persistent recurrence")
+  static const int mode = getenv("DUET_RNN_PAIR") ? atoi(getenv("DUET_RNN_PAIR")) : 2;
+  if (mode == 0 || (kind == EPI_LSTM && mode == 1)) return false;
   // under Nsight Compute (which exports NV_NSIGHT_INJECTION_TRANSPORT_TYPE / NV_TPS_LAUNCH_TOKEN to
   // the profiled process) the cooperative cluster launch fails with cudaErrorLaunchFailure although
   // 74 pairs are reported co-resident; profiled runs take the one-CTA kernel (same tiles per CTA,
