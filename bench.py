@@ -161,6 +161,9 @@ def node_decl(wl, name):
     raise KeyError(name)
 
 
+# recurrence gate-tile widths tried by harness.tuned_session (0 = automatic); BENCH_TILES overrides
+TILE_CANDIDATES = tuple(int(x) for x in os.environ.get("BENCH_TILES", "0,128").split(","))
+
 DOMINANT = {  # config -> node whose single launch dominates a step
     "c2": "fc1",      # 2048x1024x1664 pair GEMM
     "c3": "lstmA",    # one tower's persistent LSTM (S = 64)
@@ -402,7 +405,7 @@ def make_session(args, cfg, local, batch=None):
     tile_ns = None
     if args.sched == "measured" and W.rnn_nodes(wl) and args.rnn_tiles:
         sess, duet_s, tile_ns, base = tuned_session(wl, n_slots=args.slots, device=local, profile=prof_opts,
-                                                    tile_candidates=(0, 128))
+                                                    tile_candidates=TILE_CANDIDATES)
     else:
         sess = base = Session(wl, n_slots=args.slots, device=local, profile=prof_opts)
         duet_s = None
