@@ -34,5 +34,7 @@ case "$1" in
     for sh in "32 4096 256" "64 4096 128" "16 4096 256" "64 256 256" "64 64 256"; do python tools/embed_time.py $sh; done ;;
   refine)  # interleaved re-measurement of the 4 best candidates (4) vs Step 3's first figures (0)
     for r in 1 2 3; do for m in 4 0; do for c in c5 c4; do echo -n "$c refine=$m: "; DUET_MEASURE_REFINE=$m cfg_line $c; done; done; done ;;
-  *) echo "usage: bash tools/ab_r2.sh msync|ctarel|hrot|conv_occ|conv_occ128|conv_cfg|measure_flush|slots|pool|embed|refine"; exit 1 ;;
+  lstm_pair)  # LSTM on the CTA-pair recurrence (2, default) vs GRU only (1)     -> r2_lstm_pair_ab.log
+    for m in 2 1 2 1; do for sh in "lstm 4096 512 256 32" "gru 4096 512 256 32"; do DUET_RNN_PAIR=$m python tools/rnn_time.py $sh | sed "s/^/pair=$m /"; done; done ;;
+  *) echo "usage: bash tools/ab_r2.sh msync|ctarel|hrot|conv_occ|conv_occ128|conv_cfg|measure_flush|slots|pool|embed|refine|lstm_pair"; exit 1 ;;
 esac
