@@ -89,6 +89,7 @@ struct RnnPersistArgs {
   int stages = 0;                     // A-ring depth (set by the launcher)
   int pair = 0;                       // 1: CTA-pair kernel (rnn_pair_kernel; 256 x 256 pair tiles)
   int ctarel = 1;                     // one-tile path: one counter release per CTA (else per epilogue warp)
+  int issue2 = 1;                     // one-CTA kernel: second A / W issuer warps (odd ring stages)
   int hrot = 1;                       // h k-block load order rotated by hrot * CTA (0: all CTAs in order)
   int msync = 1;                      // 1: step t+1 of a 128-row block waits only for that block's
                                       // h_t (batch rows are independent recurrences); 0: grid barrier

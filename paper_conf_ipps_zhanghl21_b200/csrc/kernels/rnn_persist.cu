@@ -44,8 +44,14 @@ constexpr int RBM = 128;
 constexpr int RBK = 64;
 constexpr int R_A_BYTES = RBM * RBK * 2;
 constexpr int kREpiWarps = 8;
-constexpr int kRThreads = 64 + 32 * kREpiWarps + 32;  // + W producer warp (last)
+constexpr int kRThreads = 64 + 32 * kREpiWarps + 32 + 32;  // + W producer, second A issuer
 constexpr int kWWarp = 2 + kREpiWarps;
+// Second TMA issuer (round 2, a.issue2): one thread's bulk / tensor copies into an SM complete in
+// issue order at ~16 KB per 0.37 us (~44 GB/s) whatever their size, so the x / h stream gets a
+// second issuing warp that takes the odd ring stages (measured on the c3 tower with the resident-W
+// warp issuing every other h block: 381 -> 336 us).  (A thirteenth
+// warp would round the register budget down to 128 per thread: spills.)
+constexpr int kA2Warp = kWWarp + 1;
 
 template <int BN>
 struct RCfg {
@@ -58,10 +64,10 @@ struct RCfg {
 // Shared-memory plan: [A ring: stages x 16 KB][W: resident (kx + kh blocks) or a ring of `stages`
 // blocks][barriers][bias].  W is resident when it fits next to a ring of >= 6 A stages.
 constexpr int kRSmemBudget = 227 * 1024;
-inline int rp_plan(int bn, int nkw, bool* wres) {
+inline int rp_plan(int bn, int nkw, bool* wres, int min_res_stages = 6) {
   const int bb = bn * RBK * 2, extra = 1024 + 512 + bn * 4;
   const int res_stages = (kRSmemBudget - extra - nkw * bb) / R_A_BYTES;
-  if (res_stages >= 6) {
+  if (res_stages >= min_res_stages) {
     *wres = true;
     return res_stages > 10 ? 10 : res_stages;
   }
@@ -231,17 +237,26 @@ __global__ void __launch_bounds__(kRThreads, 1)
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
-  if (warp == 0) {
+  if (warp == 0 || warp == kA2Warp) {
     // ---------------- A producer: x_t blocks, [grid barrier], h_{t-1} blocks per (step, tile) ------
+    // (a.issue2: warp 0 issues the even ring stages, kA2Warp the odd ones; each acquires the step
+    // counter before the first h block it issues.  Measured against three issuers rotating A + W
+    // stages: two A issuers beside the W warp won on every shape, profiles/r2_issue_ab.log)
+    const int par = warp == 0 ? 0 : 1;
+    const bool two = a.issue2 != 0;
     int g = 0;
-    for (int t = 0; t < S; ++t) {
+    for (int t = 0; t < S && (two || par == 0); ++t) {
       const int nkb = kx + (t > 0 ? kh : 0);  // h_{-1} = 0: step 0 has only the x part
+      bool waited = false;
       for (int i = 0; i < my_tiles; ++i) {
         const int m0 = tile_m0(i);
+        if (a.msync) waited = false;
         for (int j = 0; j < nkb; ++j, ++g) {
+          if (two && (g & 1) != par) continue;
           const int s = g % STAGES;
           if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
-          if (j == kx && (a.msync || i == 0)) {
+          if (j >= kx && !waited) {
+            waited = true;
             // h_{t-1} of this tile's 128 batch rows: wait until every epilogue warp of every tile of
             // the row block (m-tile sync; a.msync = 0: of the whole grid) has released its slice,
             // then order the generic-proxy writes it observed before this thread's async-proxy
@@ -594,7 +609,10 @@ void launch_rp_any(const CUtensorMap& tx, const CUtensorMap& th0, const CUtensor
   if (multi) return launch_rp_multi<BN, KIND>(tx, th0, th1, tw, a, grid, st);
   static const int wres_env = getenv("DUET_RNN_WRES") ? atoi(getenv("DUET_RNN_WRES")) : 1;
   bool wres = false;
-  a.stages = rp_plan(BN, a.kx + a.kh, &wres);
+  // with two x / h issuers a resident W pays even next to a 4-stage ring (c4's GRU1024: 160 KB of
+  // weights); with one, W streams unless >= 6 stages fit (round 1: 7.72 -> 7.54 us only)
+  static const int min_res = getenv("DUET_RNN_WRES_MIN") ? atoi(getenv("DUET_RNN_WRES_MIN")) : 4;
+  a.stages = rp_plan(BN, a.kx + a.kh, &wres, a.issue2 ? min_res : 6);
   if (wres && !wres_env) {  // streamed W (comparisons)
     wres = false;
     a.stages = (192 * 1024) / (R_A_BYTES + RCfg<BN>::B_BYTES);
@@ -685,17 +703,24 @@ __global__ void __launch_bounds__(kRThreads, 1)
   const uint32_t tmem = *tmem_slot;
   const uint32_t full_l0 = ptx::mapa(ptx::smem_u32(&full[0]), leader);
 
-  if (warp == 0) {
+  if (warp == 0 || warp == kA2Warp) {
     // ---------------- A producer: own 128 rows of x_t, [grid barrier], h_{t-1} ----------------
+    // (a.issue2: warp 0 the even ring stages, kA2Warp the odd ones, as in rnn_persist_kernel)
+    const int par = warp == 0 ? 0 : 1;
+    const bool two = a.issue2 != 0;
     int g = 0;
-    for (int t = 0; t < S; ++t) {
+    for (int t = 0; t < S && (two || par == 0); ++t) {
       const int nkb = kx + (t > 0 ? kh : 0);
+      bool waited = false;
       for (int i = 0; i < my_tiles; ++i) {
         const int m0 = tile_m0(i);
+        if (a.msync) waited = false;
         for (int j = 0; j < nkb; ++j, ++g) {
+          if (two && (g & 1) != par) continue;
           const int s = g % STAGES;
           if (g >= STAGES) wait_sleep(&empty[s], ((g / STAGES) - 1) & 1);
-          if (j == kx && (a.msync || i == 0)) {  // this CTA's 128 rows (m-tile sync) or the grid
+          if (j >= kx && !waited) {  // this CTA's 128 rows (m-tile sync) or the grid
+            waited = true;
             if (lane == 0) {
               const unsigned per = (unsigned)(a.msync ? a.tiles_n : n_tiles);
               const unsigned* ctr = a.counter + (a.msync ? m0 / RBM : 0);

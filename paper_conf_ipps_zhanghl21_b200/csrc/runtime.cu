@@ -447,6 +447,8 @@ void build_op(Program& P, const Node& n, Op& op) {
       ra.msync = msync_env == 2 || (msync_env == 1 && (several || mt >= 4)) ? 1 : 0;
       static const int hrot_env = getenv("DUET_RNN_HROT") ? atoi(getenv("DUET_RNN_HROT")) : 1;
       ra.hrot = hrot_env;
+      static const int issue2_env = getenv("DUET_RNN_ISSUE2") ? atoi(getenv("DUET_RNN_ISSUE2")) : 1;
+      ra.issue2 = issue2_env;
       // one release per CTA instead of one per epilogue warp (same-address atomics at the counter's
       // L2 slice): c3 tower 393 -> 374 us, c4 GRU 587 -> 567, c5 LSTM256 424 -> 404
       // (profiles/r2_ctarel_ab.log); DUET_RNN_CTAREL=0 restores per-warp releases
