@@ -32,7 +32,11 @@ __device__ __forceinline__ unsigned long long gtimer() {
 
 constexpr int BM2 = 128;  // rows per CTA (256 per pair)
 constexpr int kEpiThreads2 = 256;           // 8 epilogue warps
-constexpr int kThreads2 = 64 + kEpiThreads2;  // + TMA producer warp + MMA warp
+constexpr int kThreads2 = 64 + kEpiThreads2 + 32;  // + TMA producer warp + MMA warp + W issuer
+// Round 2: the W stream has its own issuing warp (warp kWIss2): one thread's copies complete in issue
+// order at ~0.37 us per request, and the single producer issued 2 A + 2 W requests per stage
+// (the same finding there).  ep.dbg & 64: one issuer (A/B).
+constexpr int kWIss2 = 2 + kEpiThreads2 / 32;
 constexpr int BK2 = 64;   // one SWIZZLE_128B atom of K
 constexpr int KB2 = 2;    // k-blocks per pipeline stage: halves barrier round trips per FLOP
 constexpr int A2_ATOM = BM2 * BK2 * 2;
@@ -84,7 +88,7 @@ __global__ void __launch_bounds__(kThreads2, 1)
     ptx::tma_prefetch(&tmA);
     ptx::tma_prefetch(&tmW);
     for (int s = 0; s < C::STAGES; ++s) {
-      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&full[s], (ep.dbg & 64) ? 1 : 2);  // A issuer + W issuer (each the pair's bytes)
       ptx::mbar_init(&empty[s], 1);
     }
     ptx::mbar_init(tmem_full, 1);
@@ -94,12 +98,13 @@ __global__ void __launch_bounds__(kThreads2, 1)
   ptx::cluster_sync_relaxed();
   if (tr && threadIdx.x == 0) trace[12] = gtimer();
   const uint32_t full_leader0 = ptx::mapa(ptx::smem_u32(&full[0]), crank & ~1u);
-  if (warp == 0 && lane == 0 && !(ep.dbg & 2)) {
+  const bool split = !(ep.dbg & 64);  // A on warp 0, W on warp kWIss2
+  if (warp == (split ? kWIss2 : 0) && lane == 0 && !(ep.dbg & 2)) {
     // weights are graph parameters, never written by the previous kernel: their first stages
     // stream in while the previous kernel drains (programmatic dependent launch)
     for (int kb = 0; kb < npre; ++kb) {
       const uint32_t fb = full_leader0 + kb * 8;
-      if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, 2 * C::STAGE);
+      if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, split ? 2 * C::B_BYTES : 2 * C::STAGE);
       if (tr && kb == 0) trace[2] = gtimer();
 #pragma unroll
       for (int h = 0; h < KB2; ++h)
@@ -126,7 +131,27 @@ __global__ void __launch_bounds__(kThreads2, 1)
   if (tr && threadIdx.x == 0) trace[1] = gtimer();
   ptx::pdl_trigger();
 
-  if (warp == 0) {
+  if (split && (warp == 0 || warp == kWIss2)) {
+    // two issuers: warp 0 the A k-blocks of every stage, warp kWIss2 the W k-blocks (after the
+    // pre-loaded stages); each arrives on the leader's full barrier with the pair's bytes
+    if (lane == 0 && !(ep.dbg & 2)) {
+      const bool isA = warp == 0;
+      for (int kb = isA ? 0 : npre; kb < nk; ++kb) {
+        const int s = kb % C::STAGES;
+        if (kb >= C::STAGES) ptx::mbar_wait(&empty[s], ((kb / C::STAGES) - 1) & 1);
+        const uint32_t fb = full_leader0 + s * 8;
+        if (rank == 0) ptx::mbar_arrive_expect_tx_cl(fb, isA ? 2 * A2_BYTES : 2 * C::B_BYTES);
+#pragma unroll
+        for (int h = 0; h < KB2; ++h) {
+          if (isA)
+            ptx::tma_load_2d_2sm(&tmA, fb, sA + s * A2_BYTES + h * A2_ATOM, (kb * KB2 + h) * BK2, m0);
+          else
+            ptx::tma_load_2d_2sm(&tmW, fb, sB + s * C::B_BYTES + h * C::B_ATOM, (kb * KB2 + h) * BK2,
+                                 n0 + (int)rank * C::BH);
+        }
+      }
+    }
+  } else if (warp == 0) {
     if (lane == 0) {
       for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % C::STAGES;
@@ -175,6 +200,8 @@ __global__ void __launch_bounds__(kThreads2, 1)
       ptx::umma_commit_2sm_elect(tmem_full, pair_mask);
       if (tr && lane == 0) trace[4] = gtimer();
     }
+  } else if (warp == kWIss2) {
+    // (single-issuer mode: idle)
   } else {
     // epilogue warps 2..9: warp w reads TMEM lanes 32 (w % 4) .. +32 (hardware lane-quarter
     // rule); the two warps of a quarter split the columns.  Bias of this tile -> smem first
