@@ -57,12 +57,21 @@ struct ConvArgs {
   int r0, s0, ns;      // tap rectangle: rows r0.., columns s0 .. s0 + ns - 1
   unsigned* ctr;       // [2] dynamic tile counter + exit count (zero between launches; the last
                        // CTA to finish fetching resets both), or null: static tile = block + j grid
+  int dbg;             // 1: one producer thread issues A and W (comparisons; DUET_CONV_ISS=1)
 };
 
 // TMA-im2col variant (C % 64 == 0): one thread streams both operands; A tile = 128 consecutive
 // output pixels x 64 channels of filter tap (r, s) loaded by one im2col TMA.
+// ISS2 (round 2): the weights of each stage are issued by their own warp (warp 6, a third reader of the
+// tile ring): one thread's copies complete in issue order, and the producer issued an im2col A box
+// and a W box per k-block (the same finding)
+template <int OCC>
+constexpr bool conv_iss2() { return OCC <= 2; }  // three CTAs per SM: 224 threads would cap registers
+template <int OCC>
+constexpr int conv_threads() { return conv_iss2<OCC>() ? 224 : 192; }
+
 template <int BN, int OCC, int KB>
-__global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constant__ CUtensorMap tmX,
+__global__ void __launch_bounds__(conv_threads<OCC>(), OCC) conv_tma_kernel(const __grid_constant__ CUtensorMap tmX,
                                                             const __grid_constant__ CUtensorMap tmW, const ConvArgs a) {
   using C = ConvCfg<BN, OCC, KB>;
   constexpr int CA_BYTES = C::CA_BYTES;
@@ -93,7 +102,7 @@ __global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constan
     ptx::tma_prefetch(&tmX);
     ptx::tma_prefetch(&tmW);
     for (int i = 0; i < C::STAGES; ++i) {
-      ptx::mbar_init(&full[i], 1);
+      ptx::mbar_init(&full[i], (conv_iss2<OCC>() && !(a.dbg & 1)) ? 2 : 1);  // A producer (+ W issuer)
       ptx::mbar_init(&empty[i], 1);
     }
     for (int i = 0; i < 2; ++i) {
@@ -102,7 +111,7 @@ __global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constan
     }
     for (int i = 0; i < 4; ++i) {
       ptx::mbar_init(&tile_full[i], 1);
-      ptx::mbar_init(&tile_empty[i], 2);
+      ptx::mbar_init(&tile_empty[i], (conv_iss2<OCC>() && !(a.dbg & 1)) ? 3 : 2);  // MMA, epilogue (+ W issuer)
     }
     ptx::fence_mbar_init();
   }
@@ -124,6 +133,7 @@ __global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constan
   // other stream slot's persistent recurrence holds most SMs) keeps taking
   // tiles instead of owning a fixed share that waits for the late CTAs' SMs.  The producer fetches
   // tile j into s_tile[j % 4]; the MMA warp and the epilogue read it from there.
+  const bool iss2 = conv_iss2<OCC>() && !(a.dbg & 1);
   if (warp == 0) {
     if (lane == 0) {
       int64_t g = 0;
@@ -153,7 +163,7 @@ __global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constan
           const int st = (int)(g % C::STAGES);
           const int64_t use = g / C::STAGES;
           if (use >= 1) ptx::mbar_wait(&empty[st], (uint32_t)((use - 1) & 1));
-          ptx::mbar_arrive_expect_tx(&full[st], C::STAGE);
+          ptx::mbar_arrive_expect_tx(&full[st], iss2 ? CA_BYTES : C::STAGE);
 #pragma unroll
           for (int h = 0; h < KB; ++h) {
             const int kbi = it * KB + h;
@@ -163,10 +173,44 @@ __global__ void __launch_bounds__(192, OCC) conv_tma_kernel(const __grid_constan
             const int r = a.r0 + tap / a.ns, q = a.s0 + tap % a.ns;
             ptx::tma_load_im2col_4d(&tmX, &full[st], sA + st * CA_BYTES + h * (CBM * CBK * 2), c0, wb, hb, nn,
                                     (uint16_t)q, (uint16_t)r);
-            const int wcol = valid ? (r * s.kw + q) * s.C + c0 : a.K;  // column K: all out of bounds -> zeros
+            if (!iss2) {
+              const int wcol = valid ? (r * s.kw + q) * s.C + c0 : a.K;  // column K: all out of bounds -> zeros
+              ptx::tma_load_2d(&tmW, &full[st], sB + st * C::B_BYTES + h * C::B_ATOM, wcol, n0);
+            }
+          }
+        }
+      }
+    }
+  } else if (warp == 6) {
+    // W issuer: the same tiles (a third reader of the tile ring) and the same stage sequence
+    // (single-producer comparisons, a.dbg & 1: idle)
+    int64_t g = 0;
+    for (int j = 0; iss2; ++j) {
+      const int slot = j & 3;
+      ptx::mbar_wait(&tile_full[slot], (uint32_t)((j >> 2) & 1));
+      const int u = s_tile[slot];
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&tile_empty[slot]);
+      if (u < 0) break;
+      const int n0 = (int)((int64_t)u % tiles_n) * BN;
+      for (int it = 0; it < nk; ++it, ++g) {
+        const int st = (int)(g % C::STAGES);
+        const int64_t use = g / C::STAGES;
+        if (use >= 1) ptx::mbar_wait(&empty[st], (uint32_t)((use - 1) & 1));
+        if (lane == 0) {
+          ptx::mbar_arrive_expect_tx(&full[st], C::B_BYTES);
+#pragma unroll
+          for (int h = 0; h < KB; ++h) {
+            const int kbi = it * KB + h;
+            const bool valid = kbi < a.nkb;
+            const int kv = valid ? kbi : a.nkb - 1;
+            const int tap = kv / cb, c0 = (kv - tap * cb) * 64;
+            const int r = a.r0 + tap / a.ns, q = a.s0 + tap % a.ns;
+            const int wcol = valid ? (r * s.kw + q) * s.C + c0 : a.K;
             ptx::tma_load_2d(&tmW, &full[st], sB + st * C::B_BYTES + h * C::B_ATOM, wcol, n0);
           }
         }
+        __syncwarp();
       }
     }
   } else if (warp == 1) {
@@ -279,7 +323,7 @@ void launch_conv_tma(const CUtensorMap& tx, const CUtensorMap& tw, const ConvArg
   int dev = 0;
   cudaGetDevice(&dev);
   const int grid = (int)std::min<int64_t>(units, (int64_t)OCC * num_sms(dev));
-  launch_pdl_if(pdl_on(true), kern, dim3(grid), dim3(192), C::SMEM, st, tx, tw, a);
+  launch_pdl_if(pdl_on(true), kern, dim3(grid), dim3(conv_threads<OCC>()), C::SMEM, st, tx, tw, a);
 }
 
 
@@ -345,8 +389,9 @@ CUtensorMap make_tmap_im2col(const void* x, const ConvShape& s) {
 void conv_tc(const CUtensorMap& tw, const void* x, const float* bias, const void* residual, void* y,
              const ConvShape& s, int K, int act, const ConvPlan& p, unsigned* ctr, cudaStream_t st) {
   const ConvTaps t = conv_taps(s);
+  static const int iss_env = getenv("DUET_CONV_ISS") ? atoi(getenv("DUET_CONV_ISS")) : 2;
   ConvArgs a{(const __nv_bfloat16*)x, bias, (const __nv_bfloat16*)residual, (__nv_bfloat16*)y, s, K, act,
-             p.nkb, t.r0, t.s0, t.ns, ctr};
+             p.nkb, t.r0, t.s0, t.ns, ctr, iss_env == 1 ? 1 : 0};
   const int bn = p.bn;
   if (conv_tma_ok(s) && ((uintptr_t)x % 16) == 0) {
     CUtensorMap tx = make_tmap_im2col(x, s);
