@@ -40,8 +40,10 @@ struct TileCfg {
   static constexpr int SMEM = STAGES * (A_STAGE_BYTES + B_STAGE_BYTES) + 1024 + 256 + BN * 4;
 };
 
+// Round 2: W k-blocks on their own issuing warp (warp 6; one thread's copies complete in issue order,
+// DESIGN.md "Persistent recurrence"); ep.dbg & 64: one producer (comparisons)
 template <int BN, int EPI, typename OutT>
-__global__ void __launch_bounds__(192, 1)
+__global__ void __launch_bounds__(224, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                    const __grid_constant__ CUtensorMap tmX, const TcEpilogue ep, int M, int N, int K) {
   using Cfg = TileCfg<BN>;
@@ -71,12 +73,13 @@ __global__ void __launch_bounds__(192, 1)
     ptx::tma_prefetch(&tmW);
     if (ep.kx) ptx::tma_prefetch(&tmX);
     for (int s = 0; s < Cfg::STAGES; ++s) {
-      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&full[s], (ep.dbg & 66) ? 1 : 2);  // A producer (+ W issuer)
       ptx::mbar_init(&empty[s], 1);
     }
     ptx::mbar_init(tmem_full, 1);
     ptx::fence_mbar_init();
   }
+  const bool wsplit = !(ep.dbg & 66);
   // wait for the previous kernel BEFORE taking tensor memory: a PDL-dependent CTA that holds TMEM
   // while it waits can starve a co-resident kernel of another stream (observed as a hang with
   // two slots)
@@ -100,13 +103,24 @@ __global__ void __launch_bounds__(192, 1)
         if (ep.dbg & 2) {
           ptx::mbar_arrive(&full[s]);
         } else {
-          ptx::mbar_arrive_expect_tx(&full[s], A_STAGE_BYTES + Cfg::B_STAGE_BYTES);
+          ptx::mbar_arrive_expect_tx(&full[s], A_STAGE_BYTES + (wsplit ? 0 : Cfg::B_STAGE_BYTES));
           if (kb < ep.kx)  // fused RNN step: x_t part of K
             ptx::tma_load_2d(&tmX, &full[s], sA + s * A_STAGE_BYTES, kb * BK, ep.x_row0 + m0);
           else
             ptx::tma_load_2d(&tmA, &full[s], sA + s * A_STAGE_BYTES, (kb - ep.kx) * BK, m0);
-          ptx::tma_load_2d(&tmW, &full[s], sB + s * Cfg::B_STAGE_BYTES, kb * BK, n0);
+          if (!wsplit) ptx::tma_load_2d(&tmW, &full[s], sB + s * Cfg::B_STAGE_BYTES, kb * BK, n0);
         }
+      }
+    }
+  } else if (warp == 6) {
+    // W issuer (weights: graph parameters, independent of the previous kernel)
+    if (lane == 0 && wsplit) {
+      for (int i = 0; i < nk; ++i) {
+        const int s = i % Cfg::STAGES;
+        const int kb = kb0 + i;
+        if (i >= Cfg::STAGES) ptx::mbar_wait(&empty[s], ((i / Cfg::STAGES) - 1) & 1);
+        ptx::mbar_arrive_expect_tx(&full[s], Cfg::B_STAGE_BYTES);
+        ptx::tma_load_2d(&tmW, &full[s], sB + s * Cfg::B_STAGE_BYTES, kb * BK, n0);
       }
     }
   } else if (warp == 1) {
@@ -299,7 +313,7 @@ void launch_tc(const CUtensorMap& a, const CUtensorMap& w, const CUtensorMap& x,
     attr_done = true;
   }
   dim3 grid((N + BN - 1) / BN, (M + BM - 1) / BM, ep.splits > 1 ? ep.splits : 1);
-  launch_pdl_if(pdl_on(true), kern, grid, dim3(192), Cfg::SMEM, st, a, w, x, ep, M, N, K);
+  launch_pdl_if(pdl_on(true), kern, grid, dim3(224), Cfg::SMEM, st, a, w, x, ep, M, N, K);
 }
 
 // Fused recurrent weights: row r' = tile*BN + g*U + j' <-> (gate block g, unit j = tile*U + j');
